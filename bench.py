@@ -1,0 +1,382 @@
+#!/usr/bin/env python
+"""Benchmark of the recursive-block SpTRSV on B200 (BASELINE.json metric:
+"SpTRSV solve GFLOPS (2*nnz/t) and HBM GB/s % of peak; preprocess ms").
+
+One step = one sptrsv_solve of the whole hot path (permute-in, every triangle
+and square segment of Alg 7, permute-out) over one RHS batch of the workload.
+Default workload: BASELINE.json configs[1] = C2 (IC(0) factor of the 2D
+5-point Laplacian, n = 1M, single RHS, fp64).  Inputs are resident in HBM when
+the timed region starts; L2 (126 MB) is flushed between timed solves with a
+256 MB write (the C2 working set, 56 MB, would otherwise stay in L2).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl ours|reference]
+
+Multi-GPU (torchrun, one process per GPU): the plan is replicated and every
+rank solves its own right-hand side(s) -- independent RHS columns, no
+collective on the data path ("scaling": "weak").
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "SpTRSV solve GFLOPS (2*nnz*nrhs/t)"
+DEFAULT_NRHS = {"C1": 1, "C2": 1, "C3": 1, "C4": 1, "C5": 512}
+WORKLOAD = {
+    "C1": "C1 random lower triangle n=1000 ~5 nnz/row fp64",
+    "C2": "C2 IC(0) factor of 2D 5-point Laplacian 1000x1000 (n=1M, nnz=2.998M) fp64",
+    "C3": "C3 layered power-law L n=4M ~20 nnz/row 2815 levels fp64",
+    "C4": "C4 supernodal factor n=500K w=64 dense tiles fp64",
+    "C5": "C5 random L n=2M ~10 nnz/row, 512 RHS fp64",
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--nrhs", type=int, default=None)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--selector", default="B200", choices=["B200", "PAPER"])
+    ap.add_argument("--variant", default="REC", choices=["REC", "COL", "ROW"])
+    ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
+    ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0, help="oracle baseline budget")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                     timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([v.strip() for v in out.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def start(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+
+    def stop(self):
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=10)
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for nm, v in zip(names, r[5:9]):
+                if v.strip().lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+def algorithmic_bytes(n, nnz, nrhs, vb):
+    """Compulsory traffic of any CSR SpTRSV: read L once,
+    read b once, write x once."""
+    return nnz * (vb + 4) + 4 * (n + 1) + 2 * n * nrhs * vb
+
+
+def seg_alg_bytes(seg, nrhs, vb):
+    """Algorithmic bytes of one segment launch: its matrix
+    entries (value + column), its row pointers, and its vector traffic."""
+    m = seg["row1"] - seg["row0"]
+    if seg["kind"] == "TRI":
+        off = seg["nnz"] - m
+        return off * (vb + 4) + (m + 1) * 4 + m * vb + 2 * m * nrhs * vb  # + diag, b in, x out
+    nz = seg["nnz"]
+    rows = m - seg["empty_rows"]
+    ncols = seg["col1"] - seg["col0"]
+    return nz * (vb + 4) + (rows + 1) * 4 + ncols * nrhs * vb + 2 * rows * nrhs * vb
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+def load_traffic(kernel_impl: str):
+    """dram bytes per launch of the dominant kernel from the committed ncu
+    summary (profiles/ncu_summary.json), else None."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        d = json.load(open(p))
+        return d.get("dram_bytes_per_launch", {}).get(kernel_impl)
+    except Exception:
+        return None
+
+
+def cpu_baseline(M, b, budget_s):
+    """Oracle (Alg 1, plain C, fp64) on the host, 1 thread per RHS column
+    group; repeated full solves until ~budget_s of CPU work (bounded sample)."""
+    from oracle import numeric as on
+    nrhs = b.shape[0]
+    threads = 1 if nrhs == 1 else min(nrhs, len(os.sched_getaffinity(0)))
+    if nrhs > 1:
+        # bounded sample: the first columns only, as many as threads x 2
+        cols = min(nrhs, threads * 2)
+        bs = np.ascontiguousarray(b[:cols])
+    else:
+        cols, bs = 1, b
+    x, dt, used = on.solve_timed(M, bs, threads=threads)
+    reps, tot = 1, dt
+    while tot < budget_s and reps < 10000:
+        _, dt, used = on.solve_timed(M, bs, threads=threads)
+        tot += dt
+        reps += 1
+    per = tot / reps
+    gflops = 2.0 * M.nnz * cols / per / 1e9
+    sample = (f"{reps} full solves of the workload matrix x {cols} of {nrhs} RHS column(s), "
+              f"{tot:.1f} s of CPU time")
+    return {"value": gflops, "unit": "GFLOPS", "cores": used, "kind": "oracle", "sample": sample,
+            "ms_per_solve": per * 1e3}
+
+
+def run_reference(args):
+    """--impl reference: the oracle, as it stands, timed on the host cores."""
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return
+    from workloads import generators as g
+    from oracle import numeric as on
+    nrhs = args.nrhs or DEFAULT_NRHS[args.config]
+    M, b = g.gen_config(args.config, nrhs=nrhs)
+    threads = 1 if nrhs == 1 else min(nrhs, len(os.sched_getaffinity(0)))
+    cols = nrhs if nrhs == 1 else min(nrhs, threads * 2)
+    bs = np.ascontiguousarray(b[:cols])
+    for _ in range(args.warmup):
+        on.solve_timed(M, bs, threads=threads)
+    ts = []
+    for _ in range(args.steps):
+        _, dt, used = on.solve_timed(M, bs, threads=threads)
+        ts.append(dt)
+    t = float(np.mean(ts))
+    val = 2.0 * M.nnz * cols / t / 1e9
+    line = {"metric": METRIC, "value": val, "unit": "GFLOPS", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": WORKLOAD[args.config], "n": M.n, "nnz": M.nnz, "nrhs_timed": cols},
+            "cpu_baseline": {"value": val, "unit": "GFLOPS", "cores": used, "kind": "oracle",
+                             "sample": f"{args.steps} full solves x {cols} RHS column(s)"},
+            "e2e": {"value": val, "unit": "GFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+
+    ws, rank, local = dist_env()
+    if ws > 1:
+        dist.init_process_group("nccl")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+
+    import paper_conf_icpp_lun020_b200 as sp
+    from workloads import generators as g
+
+    nrhs = args.nrhs or DEFAULT_NRHS[args.config]
+    tdt = torch.float64 if args.dtype == "f64" else torch.float32
+    vb = 8 if args.dtype == "f64" else 4
+    M, b_np = g.gen_config(args.config, nrhs=nrhs)
+    if rank:
+        b_np = g.gen_rhs(M.n, nrhs, seed=g.SEED_BASE + int(args.config[1:]) + 1000 + rank)
+    val = M.val if args.dtype == "f64" else M.val.astype(np.float32)
+
+    # preprocess (analysis + upload): one warm-up, median of 3
+    kw = dict(selector=args.selector, variant=args.variant)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, val, **kw)
+    pre = []
+    for _ in range(3):
+        t0 = time.perf_counter()
+        p2 = sp.sptrsv_analyse(M.row_ptr, M.col_idx, val, **kw)
+        torch.cuda.synchronize()
+        pre.append((time.perf_counter() - t0) * 1e3)
+        p2.free()
+    preprocess_ms = float(np.median(pre))
+    info = plan.info()
+    segs = plan.segments()
+
+    B = torch.from_numpy(b_np).to(dev, tdt).T  # (n, nrhs) column-major
+    if nrhs == 1:
+        B = B[:, 0].contiguous()
+    X = torch.empty_like(B)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    for _ in range(args.warmup):
+        if not args.no_flush:
+            flush.zero_()
+        sp.sptrsv_solve(plan, B, X, stream=stream)
+    torch.cuda.synchronize()
+
+    # ---------------- timed region: K solves, CUDA events on the solve stream
+    plan.set_profiling(True)
+    seg_acc = None
+    clocks = ClockSampler(local)
+    clocks.start()
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    for i in range(args.steps):
+        if not args.no_flush:
+            flush.zero_()
+        starts[i].record(stream)
+        sp.sptrsv_solve(plan, B, X, stream=stream)
+        ends[i].record(stream)
+        st = plan.seg_times()  # synchronises on the last segment event
+        seg_acc = st if seg_acc is None else seg_acc + st
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+    t_local = float(np.sum(step_ms)) / 1e3
+    if ws > 1:
+        tt = torch.tensor([t_local], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_max = float(tt.item())
+    else:
+        t_max = t_local
+    plan.set_profiling(False)
+
+    flops_step = 2.0 * M.nnz * nrhs
+    value = ws * flops_step * args.steps / t_max / 1e9
+    ms_per_step = t_max / args.steps * 1e3
+
+    # ---------------- roofline of the dominant kernel
+    peak, peak_kind = load_peaks()
+    seg_mean = seg_acc / args.steps  # [perm-in, seg..., perm-out]
+    names = ["permute_in"] + [f"seg{i}:{s['impl']}" for i, s in enumerate(segs)] + ["permute_out"]
+    dom = int(np.argmax(seg_mean))
+    if 1 <= dom <= len(segs):
+        dseg = segs[dom - 1]
+        dbytes = seg_alg_bytes(dseg, nrhs, vb)
+        dimpl = dseg["impl"]
+    else:
+        dbytes = M.n * 4 + 2 * M.n * nrhs * vb
+        dimpl = "PERMUTE"
+    achieved = dbytes / (seg_mean[dom] / 1e3) / 1e9
+    tr = load_traffic(dimpl)
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": tr, "kernel": names[dom], "share_of_step": float(seg_mean[dom] / seg_mean.sum()),
+                "peak_source": f"{peak_kind} copy bandwidth (MEASURED_PEAKS.json hbm_gbs)"}
+    whole_bytes = algorithmic_bytes(M.n, M.nnz, nrhs, vb)
+    whole = {"achieved_gbs": whole_bytes / (ms_per_step / 1e3) / 1e9, "frac": whole_bytes / (ms_per_step / 1e3) / 1e9 / peak,
+             "alg_bytes": whole_bytes}
+
+    # ---------------- end to end through the C ABI with host buffers
+    Bh = torch.from_numpy(b_np.astype(np.float64 if vb == 8 else np.float32)).pin_memory().T
+    if nrhs == 1:
+        Bh = Bh[:, 0].contiguous().pin_memory()
+    Xh = torch.empty_like(Bh).pin_memory() if nrhs == 1 else torch.empty(nrhs, M.n, dtype=tdt).pin_memory().T
+    for _ in range(2):
+        sp.sptrsv_solve(plan, Bh, Xh, stream=stream)
+    e2e_ms = []
+    for _ in range(max(3, min(args.steps, 20))):
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        sp.sptrsv_solve(plan, Bh, Xh, stream=stream)  # H2D + solve + D2H (+ sync)
+        e1.record(stream)
+        e1.synchronize()
+        e2e_ms.append(e0.elapsed_time(e1))
+    e2e_t = float(np.mean(e2e_ms)) / 1e3
+    if ws > 1:
+        tt = torch.tensor([e2e_t], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        e2e_t = float(tt.item())
+    e2e = {"value": ws * flops_step / e2e_t / 1e9, "unit": "GFLOPS", "h2d_bytes_per_step": M.n * nrhs * vb,
+           "d2h_bytes_per_step": M.n * nrhs * vb, "ms_per_step": e2e_t * 1e3}
+
+    # ---------------- parity of the timed result (sampled for multi-RHS)
+    parity = None
+    if rank == 0:
+        from oracle import numeric as on
+        cols = list(range(nrhs)) if nrhs <= 4 else [0, nrhs // 2, nrhs - 1]
+        xs = X.double().cpu().numpy()
+        xs = xs[None] if xs.ndim == 1 else xs.T[cols]
+        ref = on.solve(M, b_np[cols], threads=min(len(cols), 8))
+        parity = {"rel_err": on.rel_err(xs, ref), "tol": 1e-10 if vb == 8 else 1e-4,
+                  "columns_checked": len(cols)}
+
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(M, b_np, args.cpu_seconds)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "GFLOPS", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
+            "config": {"workload": WORKLOAD[args.config], "n": M.n, "nnz": M.nnz, "nrhs": nrhs,
+                       "selector": args.selector, "variant": args.variant, "depth": info["depth"],
+                       "segments": len(segs), "l2": "flushed (256 MB write) between timed solves"
+                       if not args.no_flush else "not flushed", "parallelism": f"rhs-replicas x{ws}"},
+            "preprocess_ms": preprocess_ms,
+            "hbm_whole_solve": whole,
+            "roofline": roofline,
+            "segment_ms": {nm: float(v) for nm, v in zip(names, seg_mean)},
+            "e2e": e2e,
+            "gpu_launches": int(info["launches_per_solve"]) * args.steps,
+            "clocks": clk,
+            "parity": parity,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,443 @@
+// Host-side preprocessing of the recursive-block SpTRSV (the "analysis" of
+// sptrsv_analyse).  Deterministic: the same input always gives the same plan,
+// bit for bit, on any machine and thread count (needed for replicated plans
+// across ranks).
+//
+// Steps, in the paper's order (see DESIGN.md sec. 3 for the numbered readings):
+//   validate            Alg 1 layout: diagonal last in each CSR row
+//   levels              Alg 2 (L77-L87): level(i) = 1 + max level of its dependencies
+//   reorder             Sec 3.3 (L231-L233): stable sort of every triangle by level
+//   recursive split     Alg 6 (L184-L195), mid = lo + floor(m/2); depth rule L299
+//   COL / ROW variants  Alg 4 (L149-L159) / Alg 5 (L166-L176), same leaves (L182)
+//   blocked storage     Sec 3.3 (L229, L235-L241): triangles and squares in
+//                       execution order, diagonal separate, CSR or DCSR
+//   features + Alg 7    Sec 3.4 (L252-L296)
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <functional>
+#include <numeric>
+#include <thread>
+
+#include "internal.h"
+
+namespace sptrsv {
+
+namespace {
+
+// Run f(lo, hi) over [0, n) split into contiguous chunks on `threads` threads.
+void parallel_for(int64_t n, int threads, const std::function<void(int64_t, int64_t)>& f) {
+  if (threads <= 1 || n < 65536) {
+    f(0, n);
+    return;
+  }
+  std::vector<std::thread> th;
+  for (int t = 0; t < threads; ++t) {
+    int64_t a = n * t / threads, b = n * (t + 1) / threads;
+    th.emplace_back([=, &f] { f(a, b); });
+  }
+  for (auto& x : th) x.join();
+}
+
+struct LowerCSR {
+  int32_t n = 0;
+  std::vector<int64_t> rp;
+  std::vector<int32_t> ci;
+  std::vector<char> val;
+};
+
+Error validate(int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, const char* val, size_t vb,
+               sptrsv_fill_t fill) {
+  if (rp[0] != 0) return {SPTRSV_ERROR_INVALID_VALUE, "row_ptr[0] != 0"};
+  if ((int64_t)rp[n] != nnz) return {SPTRSV_ERROR_INVALID_VALUE, "nnz != row_ptr[n]"};
+  for (int32_t i = 0; i < n; ++i) {
+    int64_t s = rp[i], e = rp[i + 1];
+    if (e < s || e > nnz) return {SPTRSV_ERROR_INVALID_VALUE, "row_ptr not monotone at row " + std::to_string(i)};
+    for (int64_t q = s; q < e; ++q) {
+      int32_t c = ci[q];
+      if (c < 0 || c >= n) return {SPTRSV_ERROR_INVALID_VALUE, "column index out of range in row " + std::to_string(i)};
+      if (q > s && c <= ci[q - 1]) return {SPTRSV_ERROR_UNSORTED, "columns not strictly increasing in row " + std::to_string(i)};
+    }
+    bool zero;
+    if (fill == SPTRSV_LOWER) {
+      if (e > s && ci[e - 1] > i) return {SPTRSV_ERROR_NOT_TRIANGULAR, "entry above the diagonal in row " + std::to_string(i)};
+      if (e == s || ci[e - 1] != i) return {SPTRSV_ERROR_ZERO_PIVOT, "missing diagonal in row " + std::to_string(i)};
+      const char* d = val + (size_t)(e - 1) * vb;
+      zero = vb == 8 ? (*(const double*)d == 0.0) : (*(const float*)d == 0.0f);
+    } else {
+      if (e > s && ci[s] < i) return {SPTRSV_ERROR_NOT_TRIANGULAR, "entry below the diagonal in row " + std::to_string(i)};
+      if (e == s || ci[s] != i) return {SPTRSV_ERROR_ZERO_PIVOT, "missing diagonal in row " + std::to_string(i)};
+      const char* d = val + (size_t)s * vb;
+      zero = vb == 8 ? (*(const double*)d == 0.0) : (*(const float*)d == 0.0f);
+    }
+    if (zero) return {SPTRSV_ERROR_ZERO_PIVOT, "zero diagonal in row " + std::to_string(i)};
+  }
+  return {SPTRSV_SUCCESS, ""};
+}
+
+// Lower CSR of the input; UPPER is mapped to J U J (i -> n-1-i, reading R19):
+// row n-1-i of the result is row i of U read backwards, so its columns are
+// ascending and the diagonal (first in U's row) becomes last.
+LowerCSR to_lower(int32_t n, const int32_t* rp, const int32_t* ci, const char* val, size_t vb,
+                  sptrsv_fill_t fill) {
+  LowerCSR L;
+  L.n = n;
+  int64_t nnz = rp[n];
+  L.rp.resize((size_t)n + 1);
+  L.ci.resize((size_t)nnz);
+  L.val.resize((size_t)nnz * vb);
+  if (fill == SPTRSV_LOWER) {
+    for (int32_t i = 0; i <= n; ++i) L.rp[i] = rp[i];
+    std::memcpy(L.ci.data(), ci, (size_t)nnz * 4);
+    std::memcpy(L.val.data(), val, (size_t)nnz * vb);
+    return L;
+  }
+  L.rp[0] = 0;
+  for (int32_t r = 0; r < n; ++r) {
+    int32_t i = n - 1 - r;
+    L.rp[r + 1] = L.rp[r] + (rp[i + 1] - rp[i]);
+  }
+  for (int32_t r = 0; r < n; ++r) {
+    int32_t i = n - 1 - r;
+    int64_t o = L.rp[r];
+    for (int64_t q = (int64_t)rp[i + 1] - 1; q >= rp[i]; --q, ++o) {
+      L.ci[o] = n - 1 - ci[q];
+      std::memcpy(&L.val[(size_t)o * vb], val + (size_t)q * vb, vb);
+    }
+  }
+  return L;
+}
+
+// Reading R2: largest d with d == 0 or floor(n / 2^d) >= T.
+int32_t depth_rule(int64_t n, int64_t T) {
+  int32_t d = 0;
+  while ((n >> (d + 1)) >= T) ++d;
+  return d;
+}
+
+// Reading R1b: a forced depth keeps at least one row per leaf.
+int32_t clamp_depth(int64_t n, int32_t d) {
+  if (n <= 1) return 0;
+  int32_t lg = 0;
+  while ((int64_t(1) << (lg + 1)) <= n) ++lg;
+  return std::min(d, lg);
+}
+
+struct Reorderer {
+  const LowerCSR& L;
+  bool reorder;
+  std::vector<int32_t> perm, old2new, leaf_level;
+
+  explicit Reorderer(const LowerCSR& l, bool re) : L(l), reorder(re) {
+    perm.resize(L.n);
+    old2new.resize(L.n);
+    leaf_level.assign(L.n, 0);
+    std::iota(perm.begin(), perm.end(), 0);
+    std::iota(old2new.begin(), old2new.end(), 0);
+  }
+
+  // Levels of the triangle rows/cols [lo,hi) of the current P L P^T (only
+  // dependencies inside the triangle count, reading R5), then a stable
+  // counting sort of its rows by level (ties keep the current order, R4).
+  // Writes the (sorted) levels into leaf_level[lo,hi); returns nlevels.
+  int32_t node_reorder(int32_t lo, int32_t hi) {
+    int32_t m = hi - lo;
+    if (m == 0) return 0;
+    std::vector<int32_t> lev((size_t)m);
+    int32_t nl = 0;
+    for (int32_t r = lo; r < hi; ++r) {
+      int32_t o = perm[r];
+      int32_t lv = 0;
+      for (int64_t q = L.rp[o], e = L.rp[o + 1] - 1; q < e; ++q) {  // off-diagonals
+        int32_t c = old2new[L.ci[q]];
+        if (c >= lo) lv = std::max(lv, lev[c - lo] + 1);
+      }
+      lev[r - lo] = lv;
+      nl = std::max(nl, lv + 1);
+    }
+    if (reorder) {
+      std::vector<int32_t> cnt((size_t)nl + 1, 0);
+      for (int32_t k = 0; k < m; ++k) cnt[lev[k] + 1]++;
+      for (int32_t l = 0; l < nl; ++l) cnt[l + 1] += cnt[l];
+      std::vector<int32_t> np((size_t)m);
+      for (int32_t k = 0; k < m; ++k) np[cnt[lev[k]]++] = perm[lo + k];
+      for (int32_t k = 0; k < m; ++k) {
+        perm[lo + k] = np[k];
+        old2new[np[k]] = lo + k;
+      }
+      std::sort(lev.begin(), lev.end());
+    }
+    std::copy(lev.begin(), lev.end(), leaf_level.begin() + lo);
+    return nl;
+  }
+};
+
+}  // namespace
+
+static int32_t select_tri(int32_t nlevels, int32_t npr) {
+  // Alg 7, PAPER.md:L270-L278 (branch order: reading R12)
+  if (nlevels == 1) return SPTRSV_K_COMPLETELY_PARALLEL;
+  if (nlevels > 20000) return SPTRSV_K_NEAR_SERIAL;
+  if ((npr == 1 && nlevels <= 100) || (npr <= 15 && nlevels <= 20)) return SPTRSV_K_LEVEL_SET;
+  return SPTRSV_K_SYNC_FREE;
+}
+
+static int32_t select_sq(int32_t npr, int64_t empty, int64_t m) {
+  // Alg 7, PAPER.md:L281-L292 with L258's thresholds; emptyratio compared in
+  // integers (reading R9)
+  if (npr <= 12) return (2 * empty <= m) ? SPTRSV_K_SCALAR_CSR : SPTRSV_K_SCALAR_DCSR;
+  return (20 * empty <= 3 * m) ? SPTRSV_K_VECTOR_CSR : SPTRSV_K_VECTOR_DCSR;
+}
+
+Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx,
+                   const void* val_v) {
+  const char* val = (const char*)val_v;
+  const size_t vb = p.vbytes;
+  int threads = p.opts.threads > 0 ? p.opts.threads : (int)std::max(1u, std::thread::hardware_concurrency());
+  threads = std::min(threads, 64);
+
+  Error e = validate(n, nnz, row_ptr, col_idx, val, vb, p.fill);
+  if (e.status) return e;
+  LowerCSR L = to_lower(n, row_ptr, col_idx, val, vb, p.fill);
+  p.n = n;
+  p.nnz = nnz;
+
+  // ---- depth (L299) ----
+  p.min_block_rows = p.opts.min_block_rows > 0 ? p.opts.min_block_rows : (int64_t)20 * p.sm_count * 128;
+  if (p.opts.depth >= 0)
+    p.depth = clamp_depth(n, p.opts.depth);
+  else
+    p.depth = n ? depth_rule(n, p.min_block_rows) : 0;
+
+  // ---- recursive reordering: every node, root and leaves (reading R3) ----
+  // Siblings are independent once their parent is reordered (each only reads
+  // dependencies inside its own range), so one depth level runs in parallel.
+  Reorderer R(L, p.opts.reorder == 0);
+  std::vector<int32_t> leaf_nl;
+  std::vector<std::pair<int32_t, int32_t>> nodes = {{0, n}};
+  for (int32_t d = 0; d <= p.depth && n > 0; ++d) {
+    std::vector<int32_t> nl(nodes.size());
+    if (nodes.size() == 1 || threads == 1) {
+      for (size_t k = 0; k < nodes.size(); ++k) nl[k] = R.node_reorder(nodes[k].first, nodes[k].second);
+    } else {
+      std::vector<std::thread> th;
+      int T = std::min<int>(threads, (int)nodes.size());
+      for (int t = 0; t < T; ++t)
+        th.emplace_back([&, t] {
+          for (size_t k = t; k < nodes.size(); k += T) nl[k] = R.node_reorder(nodes[k].first, nodes[k].second);
+        });
+      for (auto& x : th) x.join();
+    }
+    if (d == p.depth) {
+      leaf_nl = nl;
+      break;
+    }
+    std::vector<std::pair<int32_t, int32_t>> next;
+    for (auto& nd : nodes) {
+      int32_t mid = nd.first + (nd.second - nd.first) / 2;  // reading R1
+      next.push_back({nd.first, mid});
+      next.push_back({mid, nd.second});
+    }
+    nodes.swap(next);
+  }
+
+  // ---- final P L P^T, columns sorted (reading R6) ----
+  p.p_rp.assign((size_t)n + 1, 0);
+  for (int32_t r = 0; r < n; ++r) {
+    int32_t o = R.perm[r];
+    p.p_rp[r + 1] = p.p_rp[r] + (L.rp[o + 1] - L.rp[o]);
+  }
+  p.p_ci.resize((size_t)nnz);
+  p.p_val.resize((size_t)nnz * vb);
+  parallel_for(n, threads, [&](int64_t a, int64_t b) {
+    std::vector<std::pair<int32_t, int64_t>> tmp;
+    for (int64_t r = a; r < b; ++r) {
+      int32_t o = R.perm[r];
+      int64_t s = L.rp[o], len = L.rp[o + 1] - s;
+      tmp.resize((size_t)len);
+      for (int64_t k = 0; k < len; ++k) tmp[k] = {R.old2new[L.ci[s + k]], s + k};
+      std::sort(tmp.begin(), tmp.end());
+      int64_t d0 = p.p_rp[r];
+      for (int64_t k = 0; k < len; ++k) {
+        p.p_ci[d0 + k] = tmp[k].first;
+        std::memcpy(&p.p_val[(size_t)(d0 + k) * vb], &L.val[(size_t)tmp[k].second * vb], vb);
+      }
+    }
+  });
+  p.diag_new.resize((size_t)n * vb);
+  for (int32_t r = 0; r < n; ++r)
+    std::memcpy(&p.diag_new[(size_t)r * vb], &p.p_val[(size_t)(p.p_rp[r + 1] - 1) * vb], vb);
+
+  p.perm.resize(n);
+  for (int32_t k = 0; k < n; ++k) p.perm[k] = p.fill == SPTRSV_LOWER ? R.perm[k] : n - 1 - R.perm[k];
+  p.leaf_level = R.leaf_level;
+
+  // ---- segment geometry in execution order ----
+  struct Geo { int32_t kind, r0, r1, c0, c1, leaf; };
+  std::vector<Geo> geo;
+  std::vector<std::pair<int32_t, int32_t>> leaves = nodes;  // in order
+  if (n > 0) {
+    if (p.opts.variant == SPTRSV_VARIANT_REC) {
+      std::function<void(int32_t, int32_t, int32_t)> rec = [&](int32_t lo, int32_t hi, int32_t d) {
+        if (d == 0) {
+          int32_t li = (int32_t)(std::lower_bound(leaves.begin(), leaves.end(), std::make_pair(lo, hi)) - leaves.begin());
+          geo.push_back({0, lo, hi, lo, hi, li});
+          return;
+        }
+        int32_t mid = lo + (hi - lo) / 2;
+        rec(lo, mid, d - 1);
+        geo.push_back({1, mid, hi, lo, mid, -1});
+        rec(mid, hi, d - 1);
+      };
+      rec(0, n, p.depth);
+    } else {
+      int32_t K = (int32_t)leaves.size();
+      for (int32_t k = 0; k < K; ++k) {
+        int32_t s = leaves[k].first, e2 = leaves[k].second;
+        if (p.opts.variant == SPTRSV_VARIANT_COL) {  // Alg 4, reading R16
+          geo.push_back({0, s, e2, s, e2, k});
+          if (k != K - 1) geo.push_back({1, e2, n, s, e2, -1});
+        } else {  // Alg 5, reading R17
+          if (k != 0) geo.push_back({1, s, e2, 0, s, -1});
+          geo.push_back({0, s, e2, s, e2, k});
+        }
+      }
+    }
+  }
+
+  // ---- extract blocks, features, Alg 7 ----
+  p.segs.resize(geo.size());
+  auto build_seg = [&](size_t si) {
+    const Geo& g = geo[si];
+    Segment& S = p.segs[si];
+    sptrsv_seg_info_t& I = S.info;
+    I.kind = g.kind;
+    I.row0 = g.r0; I.row1 = g.r1; I.col0 = g.c0; I.col1 = g.c1;
+    int32_t m = g.r1 - g.r0;
+    S.rp.assign((size_t)m + 1, 0);
+    std::vector<int64_t> lo_idx((size_t)m), hi_idx((size_t)m);
+    for (int32_t k = 0; k < m; ++k) {
+      int32_t r = g.r0 + k;
+      const int32_t* rb = p.p_ci.data() + p.p_rp[r];
+      const int32_t* re = p.p_ci.data() + p.p_rp[r + 1];
+      int32_t cend = g.kind == 0 ? r : g.c1;  // TRI: off-diagonals only
+      const int32_t* a = std::lower_bound(rb, re, g.c0);
+      const int32_t* b = std::lower_bound(a, re, cend);
+      lo_idx[k] = a - p.p_ci.data();
+      hi_idx[k] = b - p.p_ci.data();
+    }
+    int64_t tot = 0, empty = 0;
+    for (int32_t k = 0; k < m; ++k) {
+      int64_t c = hi_idx[k] - lo_idx[k];
+      tot += c;
+      empty += (c == 0);
+    }
+    if (g.kind == 0) {
+      I.nnz = tot + m;  // the diagonal counts (reading R8)
+      I.nnz_per_row = m ? (int32_t)(I.nnz / m) : 0;
+      I.nlevels = leaf_nl[g.leaf];
+      I.empty_rows = 0;
+      I.kernel = select_tri(I.nlevels, I.nnz_per_row);
+      I.format = I.kernel == SPTRSV_K_COMPLETELY_PARALLEL ? SPTRSV_FMT_DIAG : SPTRSV_FMT_CSR;
+      S.in_degree.resize(m);
+      for (int32_t k = 0; k < m; ++k) S.in_degree[k] = (int32_t)(hi_idx[k] - lo_idx[k]);
+      S.level_ptr.assign((size_t)I.nlevels + 1, 0);
+      for (int32_t k = 0; k < m; ++k) S.level_ptr[p.leaf_level[g.r0 + k] + 1]++;
+      int32_t mx = 0;
+      for (int32_t l = 0; l < I.nlevels; ++l) {
+        mx = std::max(mx, S.level_ptr[l + 1]);
+        S.level_ptr[l + 1] += S.level_ptr[l];
+      }
+      I.max_level_rows = mx;
+      S.nzr = m;
+    } else {
+      I.nnz = tot;
+      I.nnz_per_row = m ? (int32_t)(tot / m) : 0;
+      I.empty_rows = (int32_t)empty;
+      I.nlevels = 0;
+      I.kernel = select_sq(I.nnz_per_row, empty, m);
+      I.format = (I.kernel == SPTRSV_K_SCALAR_DCSR || I.kernel == SPTRSV_K_VECTOR_DCSR) ? SPTRSV_FMT_DCSR
+                                                                                        : SPTRSV_FMT_CSR;
+    }
+    // storage
+    bool dcsr = g.kind == 1 && I.format == SPTRSV_FMT_DCSR;
+    S.ci.resize((size_t)tot);
+    S.val.resize((size_t)tot * vb);
+    if (dcsr) {
+      S.nzr = (int32_t)(m - empty);
+      S.rows.resize(S.nzr);
+      S.rp.assign((size_t)S.nzr + 1, 0);
+    } else {
+      S.nzr = m;
+    }
+    int64_t o = 0;
+    int32_t jr = 0;
+    for (int32_t k = 0; k < m; ++k) {
+      int64_t a = lo_idx[k], b = hi_idx[k];
+      if (dcsr) {
+        if (b == a) continue;
+        S.rows[jr] = g.r0 + k;
+      }
+      std::memcpy(&S.ci[o], &p.p_ci[a], (size_t)(b - a) * 4);
+      std::memcpy(&S.val[(size_t)o * vb], &p.p_val[(size_t)a * vb], (size_t)(b - a) * vb);
+      o += b - a;
+      if (dcsr)
+        S.rp[++jr] = (int32_t)o;
+      else
+        S.rp[k + 1] = (int32_t)o;
+    }
+  };
+  if (threads > 1 && geo.size() > 1) {
+    std::vector<std::thread> th;
+    int T = std::min<int>(threads, (int)geo.size());
+    for (int t = 0; t < T; ++t)
+      th.emplace_back([&, t] {
+        for (size_t k = t; k < geo.size(); k += T) build_seg(k);
+      });
+    for (auto& x : th) x.join();
+  } else {
+    for (size_t k = 0; k < geo.size(); ++k) build_seg(k);
+  }
+  choose_impls(p);
+  return {SPTRSV_SUCCESS, ""};
+}
+
+// Which sm_100a kernel runs each segment.  PAPER: the Alg 7 label's own kernel
+// (L247-L250).  B200: a cost model over the same features.
+void choose_impls(Plan& p) {
+  for (auto& S : p.segs) {
+    auto& I = S.info;
+    if (I.kind == 0) {
+      int impl;
+      switch (I.kernel) {
+        case SPTRSV_K_COMPLETELY_PARALLEL: impl = SPTRSV_IMPL_TRI_DIAG; break;
+        case SPTRSV_K_LEVEL_SET: impl = SPTRSV_IMPL_TRI_LEVELSET; break;
+        case SPTRSV_K_NEAR_SERIAL: impl = SPTRSV_IMPL_TRI_CHAIN; break;
+        default: impl = SPTRSV_IMPL_TRI_SYNCFREE; break;
+      }
+      if (p.opts.selector == SPTRSV_SELECT_B200 && I.nlevels > 1) {
+        int64_t m = I.row1 - I.row0;
+        // narrow levels: one CTA walks the level chain with bar.sync (no
+        // cross-SM flag round trips); wide levels: all SMs
+        if (I.max_level_rows <= 2048 || (m / std::max(1, I.nlevels)) <= 256)
+          impl = SPTRSV_IMPL_TRI_CHAIN;
+        else if (I.nlevels <= 20)
+          impl = SPTRSV_IMPL_TRI_LEVELSET;
+        else
+          impl = SPTRSV_IMPL_TRI_SYNCFREE;
+      }
+      if (p.opts.force_tri_impl >= SPTRSV_IMPL_TRI_LEVELSET && p.opts.force_tri_impl <= SPTRSV_IMPL_TRI_CHAIN)
+        impl = p.opts.force_tri_impl;
+      if (p.opts.force_tri_impl == SPTRSV_IMPL_TRI_DIAG && I.nlevels <= 1) impl = SPTRSV_IMPL_TRI_DIAG;
+      I.impl = impl;
+    } else {
+      int impl = (I.kernel == SPTRSV_K_VECTOR_CSR || I.kernel == SPTRSV_K_VECTOR_DCSR) ? SPTRSV_IMPL_SQ_VECTOR
+                                                                                      : SPTRSV_IMPL_SQ_SCALAR;
+      if (p.opts.force_sq_impl == SPTRSV_IMPL_SQ_SCALAR || p.opts.force_sq_impl == SPTRSV_IMPL_SQ_VECTOR)
+        impl = p.opts.force_sq_impl;
+      I.impl = impl;
+    }
+  }
+}
+
+}  // namespace sptrsv

@@ -1,0 +1,289 @@
+// The C ABI (include/sptrsv.h): argument checking, status codes, ownership.
+#include <cuda_runtime.h>
+
+#include <chrono>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+
+#define SPTRSV_EXPORT extern "C" __attribute__((visibility("default")))
+
+namespace sptrsv {
+Error seg_times(Plan& p, float* ms, int32_t cap, int32_t* count);
+Error device_info(int* sm_count, int* major, int* minor);
+
+static thread_local std::string g_last_error;
+void set_last_error(const std::string& msg) { g_last_error = msg; }
+
+static sptrsv_status_t fail(const Error& e) {
+  set_last_error(e.msg);
+  return e.status;
+}
+static sptrsv_status_t fail(sptrsv_status_t s, const std::string& msg) {
+  set_last_error(msg);
+  return s;
+}
+}  // namespace sptrsv
+
+struct sptrsv_plan_s {
+  sptrsv::Plan p;
+};
+
+using namespace sptrsv;
+
+SPTRSV_EXPORT void sptrsv_opts_default(sptrsv_opts_t* o) {
+  if (!o) return;
+  std::memset(o, 0, sizeof(*o));
+  o->variant = SPTRSV_VARIANT_REC;
+  o->depth = -1;
+  o->min_block_rows = 0;
+  o->reorder = 0;
+  o->selector = SPTRSV_SELECT_B200;
+  o->force_tri_impl = -1;
+  o->force_sq_impl = -1;
+  o->host_only = 0;
+  o->sm_count = 0;
+  o->threads = 0;
+  o->device = -1;
+}
+
+static bool host_copy_if_device(const void* src, size_t bytes, std::vector<char>& dst, const void** out,
+                                Error* err) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, src) == cudaSuccess &&
+      (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged)) {
+    dst.resize(bytes);
+    cudaError_t e = cudaMemcpy(dst.data(), src, bytes, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) {
+      *err = {SPTRSV_ERROR_CUDA, std::string("copying CSR to host: ") + cudaGetErrorString(e)};
+      return false;
+    }
+    *out = dst.data();
+    return true;
+  }
+  cudaGetLastError();
+  *out = src;
+  return true;
+}
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_analyse(int32_t n, int64_t nnz, const int32_t* row_ptr,
+                                             const int32_t* col_idx, const void* val, sptrsv_dtype_t dtype,
+                                             sptrsv_fill_t fill, const sptrsv_opts_t* opts, void* stream,
+                                             sptrsv_plan_t* plan_out) {
+  if (!plan_out) return fail(SPTRSV_ERROR_INVALID_VALUE, "plan_out is NULL");
+  *plan_out = nullptr;
+  auto t0 = std::chrono::steady_clock::now();
+  if (n < 0 || nnz < 0) return fail(SPTRSV_ERROR_INVALID_VALUE, "n < 0 or nnz < 0");
+  if (nnz >= (int64_t(1) << 31)) return fail(SPTRSV_ERROR_NOT_SUPPORTED, "nnz >= 2^31");
+  if (dtype != SPTRSV_R64F && dtype != SPTRSV_R32F) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad dtype");
+  if (fill != SPTRSV_LOWER && fill != SPTRSV_UPPER) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad fill");
+  if (!row_ptr || (nnz > 0 && (!col_idx || !val))) return fail(SPTRSV_ERROR_INVALID_VALUE, "NULL CSR array");
+  sptrsv_opts_t o;
+  if (opts)
+    o = *opts;
+  else
+    sptrsv_opts_default(&o);
+  if (o.variant < 0 || o.variant > 2) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad variant");
+  if (o.reorder < 0 || o.reorder > 1) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad reorder");
+  if (o.selector < 0 || o.selector > 1) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad selector");
+  if (o.min_block_rows < 0) return fail(SPTRSV_ERROR_INVALID_VALUE, "min_block_rows < 0");
+
+  sptrsv_plan_s* P = new (std::nothrow) sptrsv_plan_s();
+  if (!P) return fail(SPTRSV_ERROR_ALLOC, "host allocation failed");
+  Plan& p = P->p;
+  p.opts = o;
+  p.dtype = dtype;
+  p.fill = fill;
+  p.vbytes = dtype == SPTRSV_R64F ? 8 : 4;
+
+  std::vector<char> hrp, hci, hval;
+  const void *rp_h = row_ptr, *ci_h = col_idx, *val_h = val;
+  if (!o.host_only) {
+    if (o.device >= 0) {
+      cudaError_t ce0 = cudaSetDevice(o.device);
+      if (ce0 != cudaSuccess) {
+        delete P;
+        return fail(SPTRSV_ERROR_CUDA, std::string("cudaSetDevice: ") + cudaGetErrorString(ce0));
+      }
+    }
+    int sms = 0, major = 0, minor = 0;
+    Error e = device_info(&sms, &major, &minor);
+    if (e.status) {
+      delete P;
+      return fail(e);
+    }
+    if (major != 10 || minor != 0) {
+      delete P;
+      return fail(SPTRSV_ERROR_NOT_SUPPORTED, "device is sm_" + std::to_string(major * 10 + minor) +
+                                                  "; this library is built for sm_100a (B200) only");
+    }
+    p.sm_count = o.sm_count > 0 ? o.sm_count : sms;
+    Error ce{SPTRSV_SUCCESS, ""};
+    if (!host_copy_if_device(row_ptr, (size_t)(n + 1) * 4, hrp, &rp_h, &ce) ||
+        (nnz > 0 && !host_copy_if_device(col_idx, (size_t)nnz * 4, hci, &ci_h, &ce)) ||
+        (nnz > 0 && !host_copy_if_device(val, (size_t)nnz * p.vbytes, hval, &val_h, &ce))) {
+      delete P;
+      return fail(ce);
+    }
+  } else {
+    p.sm_count = o.sm_count > 0 ? o.sm_count : 148;
+  }
+  Error e = analyse_host(p, n, nnz, (const int32_t*)rp_h, (const int32_t*)ci_h, val_h);
+  if (e.status) {
+    delete P;
+    return fail(e);
+  }
+  if (!o.host_only) {
+    e = upload(p, stream);
+    if (e.status) {
+      release(p);
+      delete P;
+      return fail(e);
+    }
+  }
+  p.analyse_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  *plan_out = P;
+  return SPTRSV_SUCCESS;
+}
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_solve(sptrsv_plan_t plan, const void* b, int64_t ldb, void* x, int64_t ldx,
+                                           int32_t nrhs, sptrsv_layout_t layout, void* stream) {
+  if (!plan) return fail(SPTRSV_ERROR_INVALID_VALUE, "plan is NULL");
+  Plan& p = plan->p;
+  if (p.opts.host_only) return fail(SPTRSV_ERROR_NOT_SUPPORTED, "plan was analysed with host_only=1");
+  if (nrhs < 0) return fail(SPTRSV_ERROR_INVALID_VALUE, "nrhs < 0");
+  if (layout != SPTRSV_COL_MAJOR && layout != SPTRSV_ROW_MAJOR) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad layout");
+  if (nrhs > 0 && p.n > 0) {
+    if (!b || !x) return fail(SPTRSV_ERROR_INVALID_VALUE, "b or x is NULL");
+    int64_t need = layout == SPTRSV_COL_MAJOR ? p.n : nrhs;
+    if (layout == SPTRSV_COL_MAJOR && nrhs == 1) need = 1;  // a single column: ld unused
+    if (layout == SPTRSV_COL_MAJOR && nrhs > 1) need = p.n;
+    if (ldb < need || ldx < need) return fail(SPTRSV_ERROR_INVALID_VALUE, "leading dimension too small");
+  }
+  Error e = sptrsv::solve(p, b, ldb, x, ldx, nrhs, layout, stream);
+  if (e.status) return fail(e);
+  return SPTRSV_SUCCESS;
+}
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_free(sptrsv_plan_t plan) {
+  if (!plan) return SPTRSV_SUCCESS;
+  release(plan->p);
+  delete plan;
+  return SPTRSV_SUCCESS;
+}
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_info(sptrsv_plan_t plan, sptrsv_plan_info_t* out) {
+  if (!plan || !out) return fail(SPTRSV_ERROR_INVALID_VALUE, "NULL argument");
+  const Plan& p = plan->p;
+  std::memset(out, 0, sizeof(*out));
+  out->n = p.n;
+  out->depth = p.depth;
+  out->nseg = (int32_t)p.segs.size();
+  out->variant = p.opts.variant;
+  out->dtype = p.dtype;
+  out->fill = p.fill;
+  out->reorder = p.opts.reorder;
+  out->selector = p.opts.selector;
+  out->nnz = p.nnz;
+  out->min_block_rows = p.min_block_rows;
+  out->sm_count = p.sm_count;
+  out->launches_per_solve = p.launches_per_solve;
+  out->analyse_ms = p.analyse_ms;
+  out->device_bytes = (int64_t)p.arena_bytes;
+  return SPTRSV_SUCCESS;
+}
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_segments(sptrsv_plan_t plan, sptrsv_seg_info_t* out, int32_t cap,
+                                                   int32_t* count) {
+  if (!plan || (cap > 0 && !out)) return fail(SPTRSV_ERROR_INVALID_VALUE, "NULL argument");
+  const Plan& p = plan->p;
+  for (int32_t i = 0; i < cap && i < (int32_t)p.segs.size(); ++i) out[i] = p.segs[i].info;
+  if (count) *count = (int32_t)p.segs.size();
+  return SPTRSV_SUCCESS;
+}
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_perm(sptrsv_plan_t plan, int32_t* host_new_to_old) {
+  if (!plan || (!host_new_to_old && plan->p.n)) return fail(SPTRSV_ERROR_INVALID_VALUE, "NULL argument");
+  std::memcpy(host_new_to_old, plan->p.perm.data(), plan->p.perm.size() * 4);
+  return SPTRSV_SUCCESS;
+}
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_levels(sptrsv_plan_t plan, int32_t* host_leaf_level) {
+  if (!plan || (!host_leaf_level && plan->p.n)) return fail(SPTRSV_ERROR_INVALID_VALUE, "NULL argument");
+  std::memcpy(host_leaf_level, plan->p.leaf_level.data(), plan->p.leaf_level.size() * 4);
+  return SPTRSV_SUCCESS;
+}
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_seg_array(sptrsv_plan_t plan, int32_t seg, int32_t which,
+                                                    int32_t* host_out, int64_t cap, int64_t* count) {
+  if (!plan) return fail(SPTRSV_ERROR_INVALID_VALUE, "plan is NULL");
+  const Plan& p = plan->p;
+  if (seg < 0 || seg >= (int32_t)p.segs.size()) return fail(SPTRSV_ERROR_INVALID_VALUE, "segment out of range");
+  const Segment& S = p.segs[seg];
+  std::vector<int32_t> tmp;
+  const std::vector<int32_t>* src = nullptr;
+  if (which == SPTRSV_ARRAY_IN_DEGREE && S.info.kind == 0) {
+    src = &S.in_degree;
+  } else if (which == SPTRSV_ARRAY_LEVEL_PTR && S.info.kind == 0) {
+    src = &S.level_ptr;
+  } else if (which == SPTRSV_ARRAY_DCSR_ROWS && S.info.kind == 1) {
+    // nonempty local rows, whatever the storage format
+    for (int32_t k = 0; k < (int32_t)S.rp.size() - 1 && S.info.format == SPTRSV_FMT_CSR; ++k)
+      if (S.rp[k + 1] > S.rp[k]) tmp.push_back(k);
+    if (S.info.format == SPTRSV_FMT_DCSR)
+      for (int32_t r : S.rows) tmp.push_back(r - S.info.row0);
+    src = &tmp;
+  } else {
+    return fail(SPTRSV_ERROR_INVALID_VALUE, "array not defined for this segment kind");
+  }
+  int64_t sz = (int64_t)src->size();
+  if (host_out && cap > 0) std::memcpy(host_out, src->data(), (size_t)std::min(cap, sz) * 4);
+  if (count) *count = sz;
+  return SPTRSV_SUCCESS;
+}
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_matrix(sptrsv_plan_t plan, int64_t* row_ptr, int32_t* col_idx,
+                                                 void* val) {
+  if (!plan) return fail(SPTRSV_ERROR_INVALID_VALUE, "plan is NULL");
+  const Plan& p = plan->p;
+  if (row_ptr) std::memcpy(row_ptr, p.p_rp.data(), p.p_rp.size() * 8);
+  if (col_idx) std::memcpy(col_idx, p.p_ci.data(), p.p_ci.size() * 4);
+  if (val) std::memcpy(val, p.p_val.data(), p.p_val.size());
+  return SPTRSV_SUCCESS;
+}
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_set_profiling(sptrsv_plan_t plan, int32_t on) {
+  if (!plan) return fail(SPTRSV_ERROR_INVALID_VALUE, "plan is NULL");
+  plan->p.profiling = on != 0;
+  plan->p.last_nseg_timed = -1;
+  return SPTRSV_SUCCESS;
+}
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_seg_times(sptrsv_plan_t plan, float* ms, int32_t cap, int32_t* count) {
+  if (!plan || (cap > 0 && !ms)) return fail(SPTRSV_ERROR_INVALID_VALUE, "NULL argument");
+  Error e = seg_times(plan->p, ms, cap, count);
+  if (e.status) return fail(e);
+  return SPTRSV_SUCCESS;
+}
+
+SPTRSV_EXPORT const char* sptrsv_status_string(sptrsv_status_t s) {
+  switch (s) {
+    case SPTRSV_SUCCESS: return "SPTRSV_SUCCESS";
+    case SPTRSV_ERROR_INVALID_VALUE: return "SPTRSV_ERROR_INVALID_VALUE";
+    case SPTRSV_ERROR_NOT_TRIANGULAR: return "SPTRSV_ERROR_NOT_TRIANGULAR";
+    case SPTRSV_ERROR_UNSORTED: return "SPTRSV_ERROR_UNSORTED";
+    case SPTRSV_ERROR_ZERO_PIVOT: return "SPTRSV_ERROR_ZERO_PIVOT";
+    case SPTRSV_ERROR_NOT_SUPPORTED: return "SPTRSV_ERROR_NOT_SUPPORTED";
+    case SPTRSV_ERROR_ALLOC: return "SPTRSV_ERROR_ALLOC";
+    case SPTRSV_ERROR_CUDA: return "SPTRSV_ERROR_CUDA";
+    case SPTRSV_ERROR_DEADLOCK: return "SPTRSV_ERROR_DEADLOCK";
+  }
+  return "SPTRSV_UNKNOWN_STATUS";
+}
+
+SPTRSV_EXPORT const char* sptrsv_last_error(void) { return g_last_error.c_str(); }
+
+SPTRSV_EXPORT const char* sptrsv_version(void) { return "sptrsv-b200 0.1 (sm_100a)"; }

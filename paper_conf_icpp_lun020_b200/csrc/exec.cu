@@ -1,0 +1,414 @@
+// Device side: plan upload, the Alg 7 segment loop (IMPROVED-RECURSIVE-BLOCK-
+// ALGORITHM) and kernel dispatch.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <string>
+
+#include "internal.h"
+#include "kernels.cuh"
+
+namespace sptrsv {
+
+#define CUDA_TRY(x)                                                                  \
+  do {                                                                               \
+    cudaError_t e_ = (x);                                                            \
+    if (e_ != cudaSuccess)                                                           \
+      return Error{SPTRSV_ERROR_CUDA, std::string(#x) + ": " + cudaGetErrorString(e_)}; \
+  } while (0)
+
+namespace {
+
+size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+template <typename F>
+void dispatch_multi(int nrhs, F&& f) {
+  if (nrhs <= 8)
+    f(std::integral_constant<int, 8>(), std::integral_constant<int, 1>());
+  else if (nrhs <= 32)
+    f(std::integral_constant<int, 32>(), std::integral_constant<int, 1>());
+  else if (nrhs <= 64)
+    f(std::integral_constant<int, 32>(), std::integral_constant<int, 2>());
+  else if (nrhs <= 128)
+    f(std::integral_constant<int, 32>(), std::integral_constant<int, 4>());
+  else if (nrhs <= 256)
+    f(std::integral_constant<int, 32>(), std::integral_constant<int, 8>());
+  else
+    f(std::integral_constant<int, 32>(), std::integral_constant<int, 16>());
+}
+
+inline unsigned cdiv(int64_t a, int64_t b) { return (unsigned)((a + b - 1) / b); }
+
+// long rows -> a warp per component (L247 "a thread or a 32-thread warp")
+inline bool tri_use_warp(const Segment& S) { return S.info.nnz_per_row > 8; }
+
+template <typename T>
+Error run_segments(Plan& p, T* w, int nrhs, cudaStream_t s, k::SolveState st, cudaEvent_t* ev) {
+  const T* diag = (const T*)p.d_diag;
+  for (size_t si = 0; si < p.segs.size(); ++si) {
+    Segment& S = p.segs[si];
+    const auto& I = S.info;
+    const int m = I.row1 - I.row0;
+    const T* val = (const T*)S.d_val;
+    if (I.kind == 1) {  // square: b -= A x
+      if (S.nzr > 0 && I.nnz > 0) {
+        bool dcsr = I.format == SPTRSV_FMT_DCSR;
+        if (nrhs == 1) {
+          if (I.impl == SPTRSV_IMPL_SQ_VECTOR) {
+            unsigned g = cdiv((int64_t)S.nzr * 32, 256);
+            if (dcsr)
+              k::sq_vector_1<T, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w);
+            else
+              k::sq_vector_1<T, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w);
+          } else {
+            unsigned g = cdiv(S.nzr, 256);
+            if (dcsr)
+              k::sq_scalar_1<T, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w);
+            else
+              k::sq_scalar_1<T, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w);
+          }
+        } else {
+          dispatch_multi(nrhs, [&](auto G, auto R) {
+            unsigned g = cdiv((int64_t)S.nzr * G, 256);
+            if (dcsr)
+              k::sq_multi<T, G, R, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w, nrhs);
+            else
+              k::sq_multi<T, G, R, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w, nrhs);
+          });
+        }
+      }
+    } else if (m > 0) {  // triangle: x_seg = L_seg^{-1} b_seg
+      switch (I.impl) {
+        case SPTRSV_IMPL_TRI_DIAG:
+          k::tri_diag<T><<<cdiv((int64_t)m * nrhs, 256), 256, 0, s>>>(I.row0, m, nrhs, diag, w);
+          break;
+        case SPTRSV_IMPL_TRI_LEVELSET: {
+          const bool warp = tri_use_warp(S);
+          for (int l = 0; l < I.nlevels; ++l) {
+            int ra = I.row0 + S.level_ptr[l], rb = I.row0 + S.level_ptr[l + 1];
+            if (rb <= ra) continue;
+            if (nrhs == 1) {
+              if (warp)
+                k::tri_level_1<T, true><<<cdiv((int64_t)(rb - ra) * 32, 256), 256, 0, s>>>(
+                    ra, rb, I.row0, S.d_rp, S.d_ci, val, diag, w);
+              else
+                k::tri_level_1<T, false><<<cdiv(rb - ra, 256), 256, 0, s>>>(ra, rb, I.row0, S.d_rp, S.d_ci, val,
+                                                                          diag, w);
+            } else {
+              dispatch_multi(nrhs, [&](auto G, auto R) {
+                k::tri_level_multi<T, G, R><<<cdiv((int64_t)(rb - ra) * G, 256), 256, 0, s>>>(
+                    ra, rb, I.row0, S.d_rp, S.d_ci, val, diag, w, nrhs);
+              });
+            }
+          }
+          break;
+        }
+        case SPTRSV_IMPL_TRI_CHAIN: {
+          if (nrhs == 1) {
+            if (tri_use_warp(S))
+              k::tri_chain_1<T, true><<<1, 1024, 0, s>>>(I.row0, I.nlevels, S.d_level_ptr, S.d_rp, S.d_ci, val,
+                                                        diag, w);
+            else
+              k::tri_chain_1<T, false><<<1, 1024, 0, s>>>(I.row0, I.nlevels, S.d_level_ptr, S.d_rp, S.d_ci, val,
+                                                         diag, w);
+          } else {
+            dispatch_multi(nrhs, [&](auto G, auto R) {
+              k::tri_chain_multi<T, G, R><<<1, 1024, 0, s>>>(I.row0, I.nlevels, S.d_level_ptr, S.d_rp, S.d_ci,
+                                                            val, diag, w, nrhs);
+            });
+          }
+          break;
+        }
+        default: {  // SPTRSV_IMPL_TRI_SYNCFREE
+          const int cap = p.sm_count * 8;  // 8 CTAs x 8 warps per SM
+          if (nrhs == 1) {
+            if (tri_use_warp(S))
+              k::tri_syncfree_warp<T><<<std::min<unsigned>(cdiv(m, 8), cap), 256, 0, s>>>(
+                  I.row0, m, S.d_rp, S.d_ci, val, diag, w, p.d_flags, st, S.ticket_slot);
+            else
+              k::tri_syncfree_thread<T><<<std::min<unsigned>(cdiv(m, 256), cap), 256, 0, s>>>(
+                  I.row0, m, S.d_rp, S.d_ci, val, diag, w, p.d_flags, st, S.ticket_slot);
+          } else {
+            dispatch_multi(nrhs, [&](auto G, auto R) {
+              k::tri_syncfree_multi<T, G, R><<<std::min<unsigned>(cdiv((int64_t)m * G, 256), cap), 256, 0, s>>>(
+                  I.row0, m, S.d_rp, S.d_ci, val, diag, w, p.d_flags, st, S.ticket_slot, nrhs);
+            });
+          }
+          break;
+        }
+      }
+    }
+    if (ev) CUDA_TRY(cudaEventRecord(ev[2 + si], s));
+  }
+  return {SPTRSV_SUCCESS, ""};
+}
+
+int count_launches(const Plan& p) {
+  int c = 2;  // permute in / out
+  for (auto& S : p.segs) {
+    if (S.info.kind == 1) {
+      c += (S.nzr > 0 && S.info.nnz > 0);
+    } else if (S.info.row1 > S.info.row0) {
+      if (S.info.impl == SPTRSV_IMPL_TRI_LEVELSET) {
+        for (int l = 0; l < S.info.nlevels; ++l) c += S.level_ptr[l + 1] > S.level_ptr[l];
+      } else {
+        c += 1;
+      }
+    }
+  }
+  return c;
+}
+
+template <typename T>
+Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs, sptrsv_layout_t layout,
+                   cudaStream_t s) {
+  const int n = p.n;
+  size_t need = (size_t)n * nrhs * sizeof(T);
+  if (need > p.ws.w_bytes) {
+    if (p.ws.w) cudaFree(p.ws.w);
+    p.ws.w = nullptr;
+    p.ws.w_bytes = 0;
+    if (cudaMalloc(&p.ws.w, std::max<size_t>(need, 256)) != cudaSuccess) {
+      cudaGetLastError();
+      return {SPTRSV_ERROR_ALLOC, "workspace allocation failed"};
+    }
+    p.ws.w_bytes = need;
+  }
+  T* w = (T*)p.ws.w;
+  k::SolveState st{&p.d_state->epoch, p.d_state->tickets, p.nticket, p.d_error};
+  cudaEvent_t* ev = nullptr;
+  if (p.profiling) {
+    size_t need_ev = p.segs.size() + 3;
+    while (p.events.size() < need_ev) {
+      cudaEvent_t e;
+      CUDA_TRY(cudaEventCreate(&e));
+      p.events.push_back((void*)e);
+    }
+    ev = (cudaEvent_t*)p.events.data();
+    CUDA_TRY(cudaEventRecord(ev[0], s));
+  }
+  const int* iperm = p.d_perm + n;  // old -> new, stored right after perm
+  if (nrhs == 1) {
+    int64_t stride = layout == SPTRSV_ROW_MAJOR ? ldb : 1;
+    k::perm_in_1<T><<<std::max(1u, cdiv(n, 256)), 256, 0, s>>>(n, p.d_perm, b, stride, w, st);
+  } else if (layout == SPTRSV_COL_MAJOR) {
+    dim3 g(std::max(1u, cdiv(n, 32)), cdiv(nrhs, 32));
+    k::perm_in_cm<T><<<g, dim3(32, 8), 0, s>>>(n, nrhs, iperm, b, ldb, w, st);
+  } else {
+    k::perm_in_rm<T><<<std::max(1u, cdiv((int64_t)n * nrhs, 256)), 256, 0, s>>>(n, nrhs, p.d_perm, b, ldb, w, st);
+  }
+  CUDA_TRY(cudaGetLastError());
+  if (ev) CUDA_TRY(cudaEventRecord(ev[1], s));
+  Error e = run_segments<T>(p, w, nrhs, s, st, ev);
+  if (e.status) return e;
+  CUDA_TRY(cudaGetLastError());
+  if (nrhs == 1) {
+    int64_t stride = layout == SPTRSV_ROW_MAJOR ? ldx : 1;
+    k::perm_out_1<T><<<std::max(1u, cdiv(n, 256)), 256, 0, s>>>(n, p.d_perm, w, x, stride);
+  } else if (layout == SPTRSV_COL_MAJOR) {
+    dim3 g(std::max(1u, cdiv(n, 32)), cdiv(nrhs, 32));
+    k::perm_out_cm<T><<<g, dim3(32, 8), 0, s>>>(n, nrhs, iperm, w, x, ldx);
+  } else {
+    k::perm_out_rm<T><<<std::max(1u, cdiv((int64_t)n * nrhs, 256)), 256, 0, s>>>(n, nrhs, p.d_perm, w, x, ldx);
+  }
+  CUDA_TRY(cudaGetLastError());
+  if (ev) {
+    CUDA_TRY(cudaEventRecord(ev[2 + p.segs.size()], s));
+    p.last_nseg_timed = (int)p.segs.size();
+  }
+  return {SPTRSV_SUCCESS, ""};
+}
+
+bool is_device_ptr(const void* ptr) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, ptr) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+}  // namespace
+
+Error upload(Plan& p, void* stream_v) {
+  cudaStream_t s = (cudaStream_t)stream_v;
+  const size_t vb = p.vbytes;
+  const int n = p.n;
+  // ---- arena layout (one allocation, segments in execution order, L229) ----
+  size_t off = 0;
+  auto take = [&](size_t bytes) {
+    size_t o = off;
+    off = align_up(off + bytes, 256);
+    return o;
+  };
+  size_t o_perm = take((size_t)2 * n * 4);  // perm (new->old) then iperm (old->new)
+  size_t o_diag = take((size_t)n * vb);
+  struct Offs { size_t rp, ci, val, rows, lp; };
+  std::vector<Offs> so(p.segs.size());
+  for (size_t i = 0; i < p.segs.size(); ++i) {
+    Segment& S = p.segs[i];
+    so[i].rp = take(S.rp.size() * 4);
+    so[i].ci = take(S.ci.size() * 4);
+    so[i].val = take(S.val.size());
+    so[i].rows = take(S.rows.size() * 4);
+    so[i].lp = take(S.level_ptr.size() * 4);
+  }
+  // sync-free tickets for every triangle (any may be forced later)
+  p.nticket = 0;
+  for (auto& S : p.segs)
+    if (S.info.kind == 0) S.ticket_slot = p.nticket++;
+  size_t o_flags = take((size_t)n * 4);
+  size_t o_state = take(sizeof(DevState) + (size_t)std::max(1, p.nticket) * 4);
+  p.arena_bytes = off;
+
+  int dev;
+  CUDA_TRY(cudaGetDevice(&dev));
+  p.device = dev;
+  if (cudaMalloc(&p.arena, std::max<size_t>(off, 256)) != cudaSuccess) {
+    cudaGetLastError();
+    return {SPTRSV_ERROR_ALLOC, "plan arena allocation failed (" + std::to_string(off) + " bytes)"};
+  }
+  // host staging of the whole arena, then one copy
+  std::vector<char> h(off, 0);
+  std::vector<int32_t> iperm(n);
+  // p.perm is already in ORIGINAL indexing (UPPER: composed with J), so the
+  // kernels gather b[perm[k]] / scatter x[perm[k]] directly.
+  for (int k2 = 0; k2 < n; ++k2) iperm[p.perm[k2]] = k2;
+  std::memcpy(&h[o_perm], p.perm.data(), (size_t)n * 4);
+  std::memcpy(&h[o_perm + (size_t)n * 4], iperm.data(), (size_t)n * 4);
+  std::memcpy(&h[o_diag], p.diag_new.data(), (size_t)n * vb);
+  char* A = (char*)p.arena;
+  for (size_t i = 0; i < p.segs.size(); ++i) {
+    Segment& S = p.segs[i];
+    std::memcpy(&h[so[i].rp], S.rp.data(), S.rp.size() * 4);
+    std::memcpy(&h[so[i].ci], S.ci.data(), S.ci.size() * 4);
+    std::memcpy(&h[so[i].val], S.val.data(), S.val.size());
+    std::memcpy(&h[so[i].rows], S.rows.data(), S.rows.size() * 4);
+    std::memcpy(&h[so[i].lp], S.level_ptr.data(), S.level_ptr.size() * 4);
+    S.d_rp = (const int32_t*)(A + so[i].rp);
+    S.d_ci = (const int32_t*)(A + so[i].ci);
+    S.d_val = (const void*)(A + so[i].val);
+    S.d_rows = (const int32_t*)(A + so[i].rows);
+    S.d_level_ptr = (const int32_t*)(A + so[i].lp);
+  }
+  p.d_perm = (const int32_t*)(A + o_perm);
+  p.d_diag = (const void*)(A + o_diag);
+  p.d_flags = (int32_t*)(A + o_flags);
+  p.d_state = (DevState*)(A + o_state);
+  CUDA_TRY(cudaMemcpyAsync(p.arena, h.data(), off, cudaMemcpyHostToDevice, s));
+  // mapped host word for the spin-wait watchdog
+  if (cudaHostAlloc((void**)&p.h_error, sizeof(int32_t), cudaHostAllocMapped) == cudaSuccess) {
+    *p.h_error = 0;
+    CUDA_TRY(cudaHostGetDevicePointer((void**)&p.d_error, p.h_error, 0));
+  } else {
+    cudaGetLastError();
+    p.h_error = nullptr;
+    p.d_error = nullptr;
+  }
+  CUDA_TRY(cudaStreamSynchronize(s));
+  p.launches_per_solve = count_launches(p);
+  return {SPTRSV_SUCCESS, ""};
+}
+
+Error solve(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t nrhs, sptrsv_layout_t layout,
+            void* stream_v) {
+  cudaStream_t s = (cudaStream_t)stream_v;
+  if (p.h_error && *(volatile int32_t*)p.h_error) {
+    *(volatile int32_t*)p.h_error = 0;
+    return {SPTRSV_ERROR_DEADLOCK, "a spin-wait watchdog tripped during an earlier solve on this plan"};
+  }
+  if (nrhs == 0 || p.n == 0) return {SPTRSV_SUCCESS, ""};
+  // the plan is bound to its device (our runtime's current device is not
+  // torch's: make it explicit on every call)
+  int cur = -1;
+  if (cudaGetDevice(&cur) != cudaSuccess || cur != p.device) CUDA_TRY(cudaSetDevice(p.device));
+  bool bd = is_device_ptr(b), xd = is_device_ptr(x);
+  if (bd != xd) return {SPTRSV_ERROR_INVALID_VALUE, "b and x must both be device or both be host pointers"};
+  const size_t vb = p.vbytes;
+  if (bd) {
+    if (p.dtype == SPTRSV_R64F)
+      return solve_device<double>(p, (const double*)b, ldb, (double*)x, ldx, nrhs, layout, s);
+    return solve_device<float>(p, (const float*)b, ldb, (float*)x, ldx, nrhs, layout, s);
+  }
+  // host buffers: stage through the device (end-to-end path), then sync
+  size_t need = (size_t)p.n * nrhs * vb;
+  if (need > p.ws.stage_bytes) {
+    if (p.ws.stage_b) cudaFree(p.ws.stage_b);
+    if (p.ws.stage_x) cudaFree(p.ws.stage_x);
+    p.ws.stage_b = p.ws.stage_x = nullptr;
+    p.ws.stage_bytes = 0;
+    if (cudaMalloc(&p.ws.stage_b, need) != cudaSuccess || cudaMalloc(&p.ws.stage_x, need) != cudaSuccess) {
+      cudaGetLastError();
+      return {SPTRSV_ERROR_ALLOC, "staging allocation failed"};
+    }
+    p.ws.stage_bytes = need;
+  }
+  // compact copies: col-major n x nrhs (ld n) or row-major n x nrhs (ld nrhs)
+  size_t width, height;
+  int64_t dld;
+  if (layout == SPTRSV_COL_MAJOR) {
+    width = (size_t)p.n * vb;
+    height = nrhs;
+    dld = p.n;
+  } else {
+    width = (size_t)nrhs * vb;
+    height = p.n;
+    dld = nrhs;
+  }
+  CUDA_TRY(cudaMemcpy2DAsync(p.ws.stage_b, width, b, (size_t)ldb * vb, width, height, cudaMemcpyHostToDevice, s));
+  Error e = p.dtype == SPTRSV_R64F
+                ? solve_device<double>(p, (const double*)p.ws.stage_b, dld, (double*)p.ws.stage_x, dld, nrhs, layout, s)
+                : solve_device<float>(p, (const float*)p.ws.stage_b, dld, (float*)p.ws.stage_x, dld, nrhs, layout, s);
+  if (e.status) return e;
+  CUDA_TRY(cudaMemcpy2DAsync(x, (size_t)ldx * vb, p.ws.stage_x, width, width, height, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  if (p.h_error && *(volatile int32_t*)p.h_error) {
+    *(volatile int32_t*)p.h_error = 0;
+    return {SPTRSV_ERROR_DEADLOCK, "spin-wait watchdog tripped"};
+  }
+  return {SPTRSV_SUCCESS, ""};
+}
+
+void release(Plan& p) {
+  if (p.device >= 0) cudaDeviceSynchronize();
+  if (p.arena) cudaFree(p.arena);
+  if (p.ws.w) cudaFree(p.ws.w);
+  if (p.ws.stage_b) cudaFree(p.ws.stage_b);
+  if (p.ws.stage_x) cudaFree(p.ws.stage_x);
+  if (p.h_error) cudaFreeHost(p.h_error);
+  for (void* e : p.events) cudaEventDestroy((cudaEvent_t)e);
+  p.arena = nullptr;
+  p.ws = Workspace{};
+  p.h_error = nullptr;
+  p.events.clear();
+}
+
+// seg times helper used by the C ABI
+Error seg_times(Plan& p, float* ms, int32_t cap, int32_t* count) {
+  if (!p.profiling || p.events.size() < p.segs.size() + 3 || p.last_nseg_timed != (int)p.segs.size())
+    return {SPTRSV_ERROR_INVALID_VALUE, "profiling is off or no solve was timed"};
+  cudaEvent_t* ev = (cudaEvent_t*)p.events.data();
+  int total = (int)p.segs.size() + 2;
+  CUDA_TRY(cudaEventSynchronize(ev[p.segs.size() + 2]));
+  for (int i = 0; i < total && i < cap; ++i) {
+    float t = 0.f;
+    CUDA_TRY(cudaEventElapsedTime(&t, ev[i], ev[i + 1]));
+    ms[i] = t;
+  }
+  if (count) *count = total;
+  return {SPTRSV_SUCCESS, ""};
+}
+
+Error device_info(int* sm_count, int* major, int* minor) {
+  int dev;
+  CUDA_TRY(cudaGetDevice(&dev));
+  cudaDeviceProp pr;
+  CUDA_TRY(cudaGetDeviceProperties(&pr, dev));
+  *sm_count = pr.multiProcessorCount;
+  *major = pr.major;
+  *minor = pr.minor;
+  return {SPTRSV_SUCCESS, ""};
+}
+
+}  // namespace sptrsv

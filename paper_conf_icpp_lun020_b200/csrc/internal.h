@@ -1,0 +1,115 @@
+// Internal plan representation of the B200 recursive-block SpTRSV library.
+// Not part of the ABI; see include/sptrsv.h.
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "sptrsv.h"
+
+namespace sptrsv {
+
+// Status carrier used inside the library (never crosses the ABI as C++).
+struct Error {
+  sptrsv_status_t status;
+  std::string msg;
+};
+
+void set_last_error(const std::string& msg);
+
+// One block of the reordered matrix P L P^T in execution order (Fig. 3(d),
+// PAPER.md:L229/L235): a triangle (solved) or a rectangle (b -= A x).
+struct Segment {
+  sptrsv_seg_info_t info{};
+  // ----- host copies (introspection + upload) -----
+  // TRI: off-diagonal entries only (the diagonal lives in Plan::diag_new).
+  // SQ : entries inside rows [row0,row1) x cols [col0,col1).
+  // CSR rows are local (0..m-1 for CSR, 0..nzr-1 for DCSR); columns are GLOBAL
+  // permuted indices so kernels index the permuted vector directly.
+  std::vector<int32_t> rp;         // CSR/DCSR row pointer (local offsets)
+  std::vector<int32_t> ci;         // global permuted column index
+  std::vector<char> val;           // dtype values
+  std::vector<int32_t> rows;       // DCSR: global permuted row of every stored row
+  std::vector<int32_t> level_ptr;  // TRI: nlevels+1 local row offsets
+  std::vector<int32_t> in_degree;  // TRI: off-diagonal count per local row
+  int32_t nzr = 0;                 // SQ: stored rows (== m for CSR)
+  // ----- device -----
+  const int32_t* d_rp = nullptr;
+  const int32_t* d_ci = nullptr;
+  const void* d_val = nullptr;
+  const int32_t* d_rows = nullptr;
+  const int32_t* d_level_ptr = nullptr;  // device copy (chain / level-set kernels)
+  int32_t ticket_slot = -1;              // sync-free: index into the device ticket array
+};
+
+// Mutable per-solve device state (one per plan).
+struct DevState {
+  uint32_t epoch;      // incremented by permute-in; ready flag == epoch means solved
+  uint32_t pad[3];
+  uint32_t tickets[1]; // [nticket] row-claim counters, zeroed by permute-in
+};
+
+struct Workspace {
+  void* w = nullptr;        // permuted solution/rhs, n x nrhs row-major
+  size_t w_bytes = 0;
+  void* stage_b = nullptr;  // host-pointer path staging (col-major n x nrhs)
+  void* stage_x = nullptr;
+  size_t stage_bytes = 0;
+};
+
+struct Plan {
+  sptrsv_opts_t opts{};
+  int32_t n = 0;
+  int64_t nnz = 0;
+  int32_t depth = 0;
+  sptrsv_dtype_t dtype = SPTRSV_R64F;
+  sptrsv_fill_t fill = SPTRSV_LOWER;
+  int32_t sm_count = 148;
+  int64_t min_block_rows = 0;
+  double analyse_ms = 0.0;
+  size_t vbytes = 8;
+
+  std::vector<Segment> segs;
+  std::vector<int32_t> perm;        // new -> old (original indexing; UPPER composed with J)
+  std::vector<int32_t> leaf_level;  // level of every new row inside its leaf
+  std::vector<char> diag_new;       // diagonal in new order (dtype)
+  // P L P^T kept on the host for introspection (sptrsv_plan_matrix)
+  std::vector<int64_t> p_rp;
+  std::vector<int32_t> p_ci;
+  std::vector<char> p_val;
+
+  // ----- device -----
+  int device = -1;
+  void* arena = nullptr;
+  size_t arena_bytes = 0;
+  const int32_t* d_perm = nullptr;
+  const void* d_diag = nullptr;
+  int32_t* d_flags = nullptr;  // per-row ready flags (sync-free)
+  DevState* d_state = nullptr;
+  int32_t nticket = 0;
+  int32_t* h_error = nullptr;  // mapped pinned host word set by the watchdog
+  int32_t* d_error = nullptr;  // its device alias
+  Workspace ws;
+  int launches_per_solve = 0;
+
+  // profiling
+  bool profiling = false;
+  std::vector<void*> events;  // cudaEvent_t
+  int last_nseg_timed = 0;
+};
+
+// analysis (host, deterministic); fills everything but the device fields
+Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx,
+                   const void* val);
+
+// kernel implementation choice per segment (selector / forced)
+void choose_impls(Plan& p);
+
+// device side (exec.cu)
+Error upload(Plan& p, void* stream);
+Error solve(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t nrhs,
+            sptrsv_layout_t layout, void* stream);
+void release(Plan& p);
+
+}  // namespace sptrsv

@@ -1,0 +1,170 @@
+"""CPU tests of the C-ABI library: it loads, exports every symbol that
+include/sptrsv.h declares, validates its input, and its host analysis is
+bit-exact against the structural oracle (levels, permutation, block
+partition, features, Alg 7 labels, formats, the permuted matrix).
+
+No compute call is made here (host_only plans: no device is touched)."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_icpp_lun020_b200 as sp
+from paper_conf_icpp_lun020_b200 import _capi as C
+from oracle import structure as st
+from workloads import generators as g
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+B200_T = 20 * 148 * 128
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _built():
+    from paper_conf_icpp_lun020_b200 import build
+    build.build()
+
+
+def test_exports_every_declared_symbol():
+    hdr = open(os.path.join(ROOT, "include", "sptrsv.h")).read()
+    hdr = re.sub(r"/\*.*?\*/", "", hdr, flags=re.S)  # drop comments
+    declared = set(re.findall(r"\b(sptrsv_[a-z_]+)\s*\(", hdr))
+    assert {"sptrsv_analyse", "sptrsv_solve", "sptrsv_free"} <= declared
+    L = C.lib()
+    for name in declared:
+        assert hasattr(L, name), name
+    assert declared == set(C.EXPORTS)
+    assert "sm_100a" in sp.version()
+
+
+def _analyse(M, **kw):
+    kw.setdefault("host_only", True)
+    kw.setdefault("min_block_rows", B200_T)
+    return sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, fill=M.uplo, **kw)
+
+
+def _compare(M, plan, A):
+    info = plan.info()
+    assert info["n"] == M.n and info["nnz"] == M.nnz and info["depth"] == A.depth
+    assert np.array_equal(plan.perm(), A.perm)
+    assert np.array_equal(plan.levels(), A.leaf_level)
+    segs = plan.segments()
+    assert len(segs) == len(A.segs)
+    for i, (s, o) in enumerate(zip(segs, A.segs)):
+        got = (s["kind"], s["row0"], s["row1"], s["col0"], s["col1"], s["nnz"], s["nlevels"],
+               s["nnz_per_row"], s["empty_rows"], s["kernel"], s["format"])
+        want = (o.kind, o.row0, o.row1, o.col0, o.col1, o.nnz, o.nlevels, o.nnz_per_row, o.empty_rows,
+                o.kernel, o.format)
+        assert got == want, (i, got, want)
+        arrs = A.seg_arrays[i]
+        if o.kind == "TRI":
+            assert np.array_equal(plan.seg_array(i, C.ARRAY_IN_DEGREE), arrs["IN_DEGREE"])
+            assert np.array_equal(plan.seg_array(i, C.ARRAY_LEVEL_PTR), arrs["LEVEL_PTR"])
+        else:
+            assert np.array_equal(plan.seg_array(i, C.ARRAY_DCSR_ROWS), arrs["DCSR_ROWS"])
+    rp, ci, va = plan.matrix()
+    assert np.array_equal(rp, A.p_row_ptr)
+    assert np.array_equal(ci, A.p_col_idx)
+    assert np.array_equal(va.view(np.uint8), np.asarray(A.p_val, dtype=va.dtype).view(np.uint8))
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C3", "C4", "C5"])
+@pytest.mark.parametrize("variant", ["REC", "COL", "ROW"])
+@pytest.mark.parametrize("depth", [0, 2, 3])
+def test_structure_parity_small_configs(name, variant, depth):
+    M, _ = g.gen_config(name, small=True)
+    plan = _analyse(M, variant=variant, depth=depth)
+    A = st.analyse(M, depth=depth, variant=variant)
+    _compare(M, plan, A)
+
+
+@pytest.mark.parametrize("name", ["C1", "C3", "C5"])
+def test_structure_parity_upper(name):
+    M, _ = g.gen_config(name, small=True)
+    U = g.to_upper(M)
+    plan = _analyse(U, depth=2)
+    _compare(U, plan, st.analyse(U, depth=2))
+
+
+@pytest.mark.parametrize("name", ["C3", "C4"])
+def test_structure_parity_no_reorder(name):
+    M, _ = g.gen_config(name, small=True)
+    plan = _analyse(M, depth=2, reorder=False)
+    _compare(M, plan, st.analyse(M, depth=2, reorder=False))
+
+
+def test_structure_parity_paper_rule_and_threshold():
+    M, _ = g.gen_config("C3", small=True)
+    for T in (5000, 7000, 20000, 10 ** 9):
+        plan = _analyse(M, min_block_rows=T)
+        _compare(M, plan, st.analyse(M, min_block_rows=T))
+
+
+def test_structure_parity_c2_full_size():
+    M, _ = g.gen_config("C2")
+    plan = _analyse(M)
+    A = st.analyse(M, min_block_rows=B200_T)
+    _compare(M, plan, A)
+    assert plan.info()["depth"] == 1
+
+
+@pytest.mark.parametrize("shape", ["diag", "chain", "dense", "arrow", "fig1", "n1", "n2", "empty"])
+def test_structure_parity_adversarial(shape):
+    M = {"diag": lambda: g.shape_diagonal(1000), "chain": lambda: g.shape_bidiagonal(3000),
+         "dense": lambda: g.shape_dense_lower(150), "arrow": lambda: g.shape_arrow(999),
+         "fig1": g.shape_paper_fig1, "n1": lambda: g.shape_diagonal(1),
+         "n2": lambda: g.shape_bidiagonal(2), "empty": lambda: g.shape_diagonal(0)}[shape]()
+    for depth in (0, 1, 4):
+        plan = _analyse(M, depth=depth)
+        _compare(M, plan, st.analyse(M, depth=depth))
+
+
+def test_deterministic_across_thread_counts():
+    M, _ = g.gen_config("C5", small=True)
+    a = _analyse(M, depth=3, threads=1)
+    b = _analyse(M, depth=3, threads=7)
+    assert np.array_equal(a.perm(), b.perm())
+    assert a.segments() == b.segments()
+    for x, y in zip(a.matrix(), b.matrix()):
+        assert np.array_equal(x, y)
+
+
+# ------------------------------------------------------------ validation
+def _expect(status, rp, ci, val, fill="L", **kw):
+    with pytest.raises(sp.SptrsvError) as e:
+        sp.sptrsv_analyse(np.array(rp), np.array(ci), np.array(val, dtype=np.float64), fill=fill,
+                          host_only=True, **kw)
+    assert e.value.status_name == status, str(e.value)
+
+
+def test_validation_errors():
+    _expect("UNSORTED", [0, 1, 3], [0, 1, 0], [1.0, 1.0, 1.0])          # row 1 cols 1,0
+    _expect("UNSORTED", [0, 1, 3], [0, 0, 0], [1.0, 1.0, 1.0])          # duplicate
+    _expect("NOT_TRIANGULAR", [0, 2, 3], [0, 1, 1], [1.0, 2.0, 1.0])    # (0,1) above diag
+    _expect("ZERO_PIVOT", [0, 1, 2], [0, 0], [1.0, 2.0])                # row 1 has no diagonal
+    _expect("ZERO_PIVOT", [0, 1, 3], [0, 0, 1], [1.0, 2.0, 0.0])        # zero diagonal
+    _expect("NOT_TRIANGULAR", [0, 1, 3], [0, 0, 1], [1.0, 2.0, 1.0], fill="U")  # (1,0) below diag
+    _expect("INVALID_VALUE", [0, 1, 3], [0, 0, 5], [1.0, 2.0, 1.0])     # column out of range
+    _expect("INVALID_VALUE", [1, 1, 3], [0, 0, 1], [1.0, 2.0, 1.0])     # row_ptr[0] != 0
+
+
+def test_validation_error_names_row():
+    with pytest.raises(sp.SptrsvError) as e:
+        sp.sptrsv_analyse(np.array([0, 1, 2, 4]), np.array([0, 1, 0, 1]), np.ones(4), host_only=True)
+    assert "row 2" in str(e.value)
+
+
+def test_float32_plan_structure_matches_float64():
+    M, _ = g.gen_config("C4", small=True)
+    a = _analyse(M, depth=2)
+    b = _analyse(M.astype(np.float32), depth=2)
+    assert np.array_equal(a.perm(), b.perm())
+    assert a.segments() == b.segments()
+
+
+def test_host_only_plan_refuses_solve():
+    M = g.shape_diagonal(4)
+    plan = _analyse(M)
+    with pytest.raises(sp.SptrsvError) as e:
+        plan.solve(np.ones(4))
+    assert e.value.status_name == "NOT_SUPPORTED"

@@ -1,0 +1,210 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bars (BASELINE.json north_star): fp64 rel_err <= 1e-10,
+fp32 rel_err <= 1e-4 against the fp64 oracle on the fp64 data; every fp64
+result also satisfies the componentwise backward-error bound of substitution
+(oracle.numeric.residual_bound_ok), which holds for any summation order.
+"""
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_icpp_lun020_b200 as sp
+from oracle import numeric as on
+from oracle import structure as st
+from workloads import generators as g
+
+pytestmark = pytest.mark.gpu
+TOL64, TOL32 = 1e-10, 1e-4
+B200_T = 20 * 148 * 128
+
+
+def _solve(M, b, dtype=torch.float64, layout="col", **kw):
+    """b: numpy (nrhs, n).  Returns x numpy (nrhs, n) float64."""
+    val = M.val if dtype == torch.float64 else M.val.astype(np.float32)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, val, fill=M.uplo, **kw)
+    bt = torch.from_numpy(b).to("cuda", dtype)
+    if layout == "col":
+        B = bt.T  # (n, nrhs) column-major
+    else:
+        B = bt.T.contiguous()  # (n, nrhs) row-major
+    if b.shape[0] == 1:
+        B = bt[0].contiguous()
+    X = sp.sptrsv_solve(plan, B)
+    torch.cuda.synchronize()
+    x = X.double().cpu().numpy()
+    x = x[None] if x.ndim == 1 else x.T
+    return x, plan
+
+
+def _check64(M, b, x):
+    ref = on.solve(M, b)
+    err = on.rel_err(x, ref)
+    assert err <= TOL64, err
+    ok, worst = on.residual_bound_ok(M, x, b)
+    assert ok, worst
+    return err
+
+
+CONFIGS = ["C1", "C2", "C3", "C4", "C5"]
+
+
+@pytest.mark.parametrize("name", CONFIGS)
+@pytest.mark.parametrize("selector", ["PAPER", "B200"])
+def test_small_configs_default(gpu, name, selector):
+    M, b = g.gen_config(name, small=True, nrhs=1)
+    x, _ = _solve(M, b, selector=selector, min_block_rows=max(2, M.n // 9))
+    _check64(M, b, x)
+
+
+@pytest.mark.parametrize("name", CONFIGS)
+@pytest.mark.parametrize("tri", ["TRI_LEVELSET", "TRI_SYNCFREE", "TRI_CHAIN"])
+@pytest.mark.parametrize("sq", ["SQ_SCALAR", "SQ_VECTOR"])
+def test_forced_kernels(gpu, name, tri, sq):
+    M, b = g.gen_config(name, small=True, nrhs=1)
+    if tri == "TRI_LEVELSET" and name in ("C2",):
+        pytest.skip("thousands of per-level launches; covered by C1/C3-C5")
+    x, plan = _solve(M, b, depth=2, force_tri_impl=tri, force_sq_impl=sq)
+    assert all(s["impl"] == tri for s in plan.segments() if s["kind"] == "TRI" and s["nlevels"] > 1)
+    _check64(M, b, x)
+
+
+@pytest.mark.parametrize("name", CONFIGS)
+@pytest.mark.parametrize("variant", ["REC", "COL", "ROW"])
+def test_variants(gpu, name, variant):
+    M, b = g.gen_config(name, small=True, nrhs=1)
+    x, _ = _solve(M, b, depth=3, variant=variant)
+    _check64(M, b, x)
+
+
+@pytest.mark.parametrize("name", CONFIGS)
+@pytest.mark.parametrize("nrhs", [2, 7, 33, 70])
+@pytest.mark.parametrize("tri", ["TRI_LEVELSET", "TRI_SYNCFREE", "TRI_CHAIN"])
+def test_multi_rhs(gpu, name, nrhs, tri):
+    if tri == "TRI_LEVELSET" and name == "C2":
+        pytest.skip("per-level launches")
+    M, b = g.gen_config(name, small=True, nrhs=nrhs)
+    x, _ = _solve(M, b, depth=2, force_tri_impl=tri)
+    _check64(M, b, x)
+
+
+@pytest.mark.parametrize("layout", ["col", "row"])
+def test_layouts(gpu, layout):
+    M, b = g.gen_config("C5", small=True, nrhs=9)
+    x, _ = _solve(M, b, layout=layout, depth=2)
+    _check64(M, b, x)
+
+
+@pytest.mark.parametrize("name", CONFIGS)
+def test_fp32(gpu, name):
+    M, b = g.gen_config(name, small=True, nrhs=1)
+    x, _ = _solve(M, b, dtype=torch.float32, depth=2)
+    assert on.rel_err(x, on.solve(M, b)) <= TOL32
+
+
+@pytest.mark.parametrize("name", ["C1", "C3", "C5"])
+def test_upper(gpu, name):
+    M, b = g.gen_config(name, small=True, nrhs=2)
+    U = g.to_upper(M)
+    x, _ = _solve(U, b, depth=2)
+    _check64(U, b, x)
+
+
+def test_repeated_solves_epoch(gpu):
+    M, b = g.gen_config("C3", small=True, nrhs=1)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, depth=2, force_tri_impl="TRI_SYNCFREE")
+    B = torch.from_numpy(b[0]).cuda()
+    ref = on.solve(M, b)
+    for _ in range(20):
+        X = plan.solve(B)
+    torch.cuda.synchronize()
+    assert on.rel_err(X.cpu().numpy()[None], ref) <= TOL64
+
+
+def test_in_place(gpu):
+    M, b = g.gen_config("C5", small=True, nrhs=4)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, depth=2)
+    B = torch.from_numpy(b).cuda().T
+    sp.sptrsv_solve(plan, B, x=B)
+    torch.cuda.synchronize()
+    _check64(M, b, B.T.cpu().numpy())
+
+
+def test_host_pointers(gpu):
+    M, b = g.gen_config("C2", small=True, nrhs=3)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val)
+    Bh = np.ascontiguousarray(b.T)  # (n, 3) row-major host
+    X = sp.sptrsv_solve(plan, Bh)
+    _check64(M, b, X.T)
+    Bp = torch.from_numpy(b).pin_memory().T  # pinned host, column-major
+    Xp = sp.sptrsv_solve(plan, Bp)
+    _check64(M, b, Xp.T.numpy())
+
+
+@pytest.mark.parametrize("shape", ["diag", "chain", "dense", "arrow", "n1", "fig1"])
+def test_adversarial(gpu, shape):
+    M = {"diag": lambda: g.shape_diagonal(10000), "chain": lambda: g.shape_bidiagonal(100_000),
+         "dense": lambda: g.shape_dense_lower(300), "arrow": lambda: g.shape_arrow(5000),
+         "n1": lambda: g.shape_diagonal(1), "fig1": g.shape_paper_fig1}[shape]()
+    b = g.gen_rhs(M.n, 1, seed=5)
+    for tri in (None, "TRI_SYNCFREE", "TRI_CHAIN"):
+        x, _ = _solve(M, b, depth=1 if M.n > 1 else 0, force_tri_impl=tri)
+        _check64(M, b, x)
+
+
+def test_long_chain_near_serial(gpu):
+    # nlevels > 20000 -> NEAR_SERIAL label (Alg 7), single-CTA chain kernel
+    M = g.shape_bidiagonal(300_000)
+    b = g.gen_rhs(M.n, 1, seed=6)
+    x, plan = _solve(M, b, selector="PAPER")
+    segs = plan.segments()
+    assert segs[0]["kernel"] == "NEAR_SERIAL" and segs[0]["impl"] == "TRI_CHAIN"
+    _check64(M, b, x)
+
+
+def test_zero_rhs_and_empty(gpu):
+    M = g.shape_diagonal(10)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val)
+    B = torch.zeros(10, 0, dtype=torch.float64, device="cuda")
+    sp.sptrsv_solve(plan, B)
+    E = g.shape_diagonal(0)
+    pe = sp.sptrsv_analyse(E.row_ptr, E.col_idx, E.val)
+    sp.sptrsv_solve(pe, torch.zeros(0, dtype=torch.float64, device="cuda"))
+
+
+def test_mixed_pointers_rejected(gpu):
+    M = g.shape_diagonal(10)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val)
+    with pytest.raises(sp.SptrsvError):
+        sp.sptrsv_solve(plan, torch.ones(10, dtype=torch.float64, device="cuda"), x=np.zeros(10))
+
+
+# ------------------------------------------------------------- full sizes
+@pytest.mark.parametrize("name", ["C1", "C2", "C3", "C4"])
+def test_full_size_configs(gpu, name):
+    """BASELINE.json sizes, default options (what bench.py times)."""
+    M, b = g.gen_config(name, nrhs=1)
+    x, plan = _solve(M, b)
+    err = _check64(M, b, x)
+    # the plan's structure at full size is the oracle's
+    A = st.analyse(M, min_block_rows=B200_T)
+    segs = plan.segments()
+    assert [(s["row0"], s["row1"], s["col0"], s["col1"], s["nnz"], s["nlevels"], s["kernel"])
+            for s in segs] == [(o.row0, o.row1, o.col0, o.col1, o.nnz, o.nlevels, o.kernel) for o in A.segs]
+    assert np.array_equal(plan.perm(), A.perm)
+    print(name, "rel_err", err)
+
+
+def test_full_size_c5_multi_rhs_sampled(gpu):
+    """C5: n=2M, 512 RHS in one solve; 6 sampled columns against the oracle."""
+    M, b = g.gen_config("C5", nrhs=512)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val)
+    B = torch.from_numpy(b).cuda().T
+    X = sp.sptrsv_solve(plan, B)
+    torch.cuda.synchronize()
+    cols = [0, 1, 77, 255, 256, 511]
+    xs = X[:, cols].T.cpu().numpy()
+    ref = on.solve(M, b[cols], threads=6)
+    assert on.rel_err(xs, ref) <= TOL64
+    ok, worst = on.residual_bound_ok(M, xs, b[cols])
+    assert ok, worst
