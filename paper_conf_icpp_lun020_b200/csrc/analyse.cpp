@@ -265,8 +265,17 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
     }
   });
   p.diag_new.resize((size_t)n * vb);
-  for (int32_t r = 0; r < n; ++r)
+  p.rdiag_new.resize((size_t)n * vb);
+  for (int32_t r = 0; r < n; ++r) {
     std::memcpy(&p.diag_new[(size_t)r * vb], &p.p_val[(size_t)(p.p_rp[r + 1] - 1) * vb], vb);
+    if (vb == 8) {
+      double v = 1.0 / *(const double*)&p.diag_new[(size_t)r * 8];
+      std::memcpy(&p.rdiag_new[(size_t)r * 8], &v, 8);
+    } else {
+      float v = (float)(1.0 / (double)*(const float*)&p.diag_new[(size_t)r * 4]);
+      std::memcpy(&p.rdiag_new[(size_t)r * 4], &v, 4);
+    }
+  }
 
   p.perm.resize(n);
   for (int32_t k = 0; k < n; ++k) p.perm[k] = p.fill == SPTRSV_LOWER ? R.perm[k] : n - 1 - R.perm[k];
@@ -379,7 +388,25 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
         S.rows[jr] = g.r0 + k;
       }
       std::memcpy(&S.ci[o], &p.p_ci[a], (size_t)(b - a) * 4);
-      std::memcpy(&S.val[(size_t)o * vb], &p.p_val[(size_t)a * vb], (size_t)(b - a) * vb);
+      {
+        // every stored row is scaled by 1/d_i (triangles: l_ij/d_i, squares:
+        // a_ij/d_i; permute-in scales b the same way), so the solve evaluates
+        // x_i = b_i/d_i - sum_j (l_ij/d_i) x_j with no division on the chain
+        const int32_t r = g.r0 + k;
+        if (vb == 8) {
+          double d = *(const double*)&p.diag_new[(size_t)r * 8];
+          for (int64_t q = a; q < b; ++q) {
+            double v = *(const double*)&p.p_val[(size_t)q * 8] / d;
+            std::memcpy(&S.val[(size_t)(o + q - a) * 8], &v, 8);
+          }
+        } else {
+          double d = (double)*(const float*)&p.diag_new[(size_t)r * 4];
+          for (int64_t q = a; q < b; ++q) {
+            float v = (float)((double)*(const float*)&p.p_val[(size_t)q * 4] / d);
+            std::memcpy(&S.val[(size_t)(o + q - a) * 4], &v, 4);
+          }
+        }
+      }
       o += b - a;
       if (dcsr)
         S.rp[++jr] = (int32_t)o;

@@ -3,6 +3,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -43,9 +45,78 @@ inline unsigned cdiv(int64_t a, int64_t b) { return (unsigned)((a + b - 1) / b);
 // long rows -> a warp per component (L247 "a thread or a 32-thread warp")
 inline bool tri_use_warp(const Segment& S) { return S.info.nnz_per_row > 8; }
 
+// Shared-memory geometry of the TMA-staged chain kernel (227 KB per CTA).
+// Overridable for tuning with SPTRSV_CHAIN_GEOM="NST,RMAX,EMAX,XW,LMAX".
+k::ChainGeom chain_geometry(const Plan& p) {
+  int NST, RMAX, EMAX, XW, LMAX;
+  if (p.vbytes == 8) {
+    NST = 4; RMAX = 1024; EMAX = 2048; XW = 4096; LMAX = 256;
+  } else {
+    NST = 4; RMAX = 2048; EMAX = 4096; XW = 4096; LMAX = 256;
+  }
+  if (const char* e = std::getenv("SPTRSV_CHAIN_GEOM")) {
+    int a, b, c, d, f;
+    if (std::sscanf(e, "%d,%d,%d,%d,%d", &a, &b, &c, &d, &f) == 5 && a >= 2 && b >= 1 && c >= 1 && d >= 1 &&
+        (d & (d - 1)) == 0 && f >= 1) {
+      NST = a; RMAX = b; EMAX = c; XW = d; LMAX = f;
+    }
+  }
+  return p.vbytes == 8 ? k::chain_geom<double>(NST, RMAX, EMAX, XW, LMAX)
+                       : k::chain_geom<float>(NST, RMAX, EMAX, XW, LMAX);
+}
+
+// Cut a chain triangle into stages of whole levels (rows <= RMAX, entries <=
+// EMAX, levels <= LMAX); a level that does not fit is split by rows.  Leaves
+// chain_recs empty when one row has more than EMAX entries (the unstaged
+// chain kernel runs instead).
+void build_chain_stages(Segment& S, const k::ChainGeom& g) {
+  S.chain_recs.clear();
+  const auto& I = S.info;
+  if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_CHAIN) return;
+  const int m = I.row1 - I.row0;
+  for (int r = 0; r < m; ++r)
+    if (S.rp[r + 1] - S.rp[r] > g.EMAX) return;
+  std::vector<int32_t> st = {0};
+  int cur_r = 0, cur_e = 0, cur_l = 0;
+  auto close = [&](int at) {
+    if (at > st.back()) st.push_back(at);
+    cur_r = cur_e = cur_l = 0;
+  };
+  for (int l = 0; l < I.nlevels; ++l) {
+    int la = S.level_ptr[l], lb = S.level_ptr[l + 1];
+    int lr = lb - la, le = S.rp[lb] - S.rp[la];
+    if (cur_r + lr <= g.RMAX && cur_e + le <= g.EMAX && cur_l + 1 <= g.LMAX) {
+      cur_r += lr; cur_e += le; cur_l += 1;
+      continue;
+    }
+    close(la);
+    if (lr <= g.RMAX && le <= g.EMAX) {
+      cur_r = lr; cur_e = le; cur_l = 1;
+      continue;
+    }
+    for (int r = la; r < lb; ++r) {  // split a wide level by rows
+      int re = S.rp[r + 1] - S.rp[r];
+      if (cur_r + 1 > g.RMAX || cur_e + re > g.EMAX) close(r);
+      cur_r += 1; cur_e += re; cur_l = 1;
+    }
+  }
+  close(m);
+  // records {sa, sb, e0, e1, l0, nl, 0, 0}
+  const int ns = (int)st.size() - 1;
+  S.chain_recs.assign((size_t)ns * 8, 0);
+  int l = 0;
+  for (int s = 0; s < ns; ++s) {
+    int sa = st[s], sb = st[s + 1];
+    while (S.level_ptr[l + 1] <= sa) ++l;  // level containing sa
+    int l_last = l;
+    while (S.level_ptr[l_last + 1] < sb) ++l_last;  // level containing sb-1
+    int32_t* R = &S.chain_recs[(size_t)s * 8];
+    R[0] = sa; R[1] = sb; R[2] = S.rp[sa]; R[3] = S.rp[sb]; R[4] = l; R[5] = l_last - l + 2;
+  }
+}
+
 template <typename T>
-Error run_segments(Plan& p, T* w, int nrhs, cudaStream_t s, k::SolveState st, cudaEvent_t* ev) {
-  const T* diag = (const T*)p.d_diag;
+Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveState st, cudaEvent_t* ev) {
   for (size_t si = 0; si < p.segs.size(); ++si) {
     Segment& S = p.segs[si];
     const auto& I = S.info;
@@ -58,30 +129,32 @@ Error run_segments(Plan& p, T* w, int nrhs, cudaStream_t s, k::SolveState st, cu
           if (I.impl == SPTRSV_IMPL_SQ_VECTOR) {
             unsigned g = cdiv((int64_t)S.nzr * 32, 256);
             if (dcsr)
-              k::sq_vector_1<T, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w);
+              k::sq_vector_1<T, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
             else
-              k::sq_vector_1<T, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w);
+              k::sq_vector_1<T, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
           } else {
             unsigned g = cdiv(S.nzr, 256);
             if (dcsr)
-              k::sq_scalar_1<T, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w);
+              k::sq_scalar_1<T, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
             else
-              k::sq_scalar_1<T, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w);
+              k::sq_scalar_1<T, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
           }
         } else {
           dispatch_multi(nrhs, [&](auto G, auto R) {
             unsigned g = cdiv((int64_t)S.nzr * G, 256);
             if (dcsr)
-              k::sq_multi<T, G, R, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w, nrhs);
+              k::sq_multi<T, G, R, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw,
+                                                           nrhs);
             else
-              k::sq_multi<T, G, R, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, w, nrhs);
+              k::sq_multi<T, G, R, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw,
+                                                            nrhs);
           });
         }
       }
     } else if (m > 0) {  // triangle: x_seg = L_seg^{-1} b_seg
       switch (I.impl) {
         case SPTRSV_IMPL_TRI_DIAG:
-          k::tri_diag<T><<<cdiv((int64_t)m * nrhs, 256), 256, 0, s>>>(I.row0, m, nrhs, diag, w);
+          k::tri_diag<T><<<cdiv((int64_t)m * nrhs, 256), 256, 0, s>>>(I.row0, m, nrhs, bw, xs);
           break;
         case SPTRSV_IMPL_TRI_LEVELSET: {
           const bool warp = tri_use_warp(S);
@@ -91,31 +164,43 @@ Error run_segments(Plan& p, T* w, int nrhs, cudaStream_t s, k::SolveState st, cu
             if (nrhs == 1) {
               if (warp)
                 k::tri_level_1<T, true><<<cdiv((int64_t)(rb - ra) * 32, 256), 256, 0, s>>>(
-                    ra, rb, I.row0, S.d_rp, S.d_ci, val, diag, w);
+                    ra, rb, I.row0, S.d_rp, S.d_ci, val, bw, xs);
               else
                 k::tri_level_1<T, false><<<cdiv(rb - ra, 256), 256, 0, s>>>(ra, rb, I.row0, S.d_rp, S.d_ci, val,
-                                                                          diag, w);
+                                                                          bw, xs);
             } else {
               dispatch_multi(nrhs, [&](auto G, auto R) {
                 k::tri_level_multi<T, G, R><<<cdiv((int64_t)(rb - ra) * G, 256), 256, 0, s>>>(
-                    ra, rb, I.row0, S.d_rp, S.d_ci, val, diag, w, nrhs);
+                    ra, rb, I.row0, S.d_rp, S.d_ci, val, bw, xs, nrhs);
               });
             }
           }
           break;
         }
         case SPTRSV_IMPL_TRI_CHAIN: {
-          if (nrhs == 1) {
+          if (nrhs == 1 && !S.chain_recs.empty()) {
+            const k::ChainGeom cg = chain_geometry(p);
+            const uint32_t smem = k::chain_smem_bytes<T>(cg);
+            static uint32_t attr_bytes = 0;  // per template instance
+            if (smem > attr_bytes) {
+              CUDA_TRY(cudaFuncSetAttribute(k::tri_chain_tma<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                            (int)smem));
+              attr_bytes = smem;
+            }
+            k::tri_chain_tma<T><<<1, 1024, smem, s>>>(I.row0, (int)(S.chain_recs.size() / 8),
+                                                      (const k::StageRec*)S.d_chain_recs, S.d_level_ptr, S.d_rp,
+                                                      S.d_ci, val, bw, xs, cg);
+          } else if (nrhs == 1) {
             if (tri_use_warp(S))
               k::tri_chain_1<T, true><<<1, 1024, 0, s>>>(I.row0, I.nlevels, S.d_level_ptr, S.d_rp, S.d_ci, val,
-                                                        diag, w);
+                                                        bw, xs);
             else
               k::tri_chain_1<T, false><<<1, 1024, 0, s>>>(I.row0, I.nlevels, S.d_level_ptr, S.d_rp, S.d_ci, val,
-                                                         diag, w);
+                                                         bw, xs);
           } else {
             dispatch_multi(nrhs, [&](auto G, auto R) {
               k::tri_chain_multi<T, G, R><<<1, 1024, 0, s>>>(I.row0, I.nlevels, S.d_level_ptr, S.d_rp, S.d_ci,
-                                                            val, diag, w, nrhs);
+                                                            val, bw, xs, nrhs);
             });
           }
           break;
@@ -124,15 +209,15 @@ Error run_segments(Plan& p, T* w, int nrhs, cudaStream_t s, k::SolveState st, cu
           const int cap = p.sm_count * 8;  // 8 CTAs x 8 warps per SM
           if (nrhs == 1) {
             if (tri_use_warp(S))
-              k::tri_syncfree_warp<T><<<std::min<unsigned>(cdiv(m, 8), cap), 256, 0, s>>>(
-                  I.row0, m, S.d_rp, S.d_ci, val, diag, w, p.d_flags, st, S.ticket_slot);
+              k::tri_syncfree_warp<T, 4><<<std::min<unsigned>(cdiv(m, 8), cap), 256, 0, s>>>(
+                  I.row0, m, S.d_rp, S.d_ci, val, bw, xs, st, S.ticket_slot);
             else
-              k::tri_syncfree_thread<T><<<std::min<unsigned>(cdiv(m, 256), cap), 256, 0, s>>>(
-                  I.row0, m, S.d_rp, S.d_ci, val, diag, w, p.d_flags, st, S.ticket_slot);
+              k::tri_syncfree_thread<T, 4><<<std::min<unsigned>(cdiv(m, 256), cap), 256, 0, s>>>(
+                  I.row0, m, S.d_rp, S.d_ci, val, bw, xs, st, S.ticket_slot);
           } else {
             dispatch_multi(nrhs, [&](auto G, auto R) {
               k::tri_syncfree_multi<T, G, R><<<std::min<unsigned>(cdiv((int64_t)m * G, 256), cap), 256, 0, s>>>(
-                  I.row0, m, S.d_rp, S.d_ci, val, diag, w, p.d_flags, st, S.ticket_slot, nrhs);
+                  I.row0, m, S.d_rp, S.d_ci, val, bw, xs, st, S.ticket_slot, nrhs);
             });
           }
           break;
@@ -166,17 +251,23 @@ Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs
   const int n = p.n;
   size_t need = (size_t)n * nrhs * sizeof(T);
   if (need > p.ws.w_bytes) {
-    if (p.ws.w) cudaFree(p.ws.w);
-    p.ws.w = nullptr;
+    if (p.ws.bw) cudaFree(p.ws.bw);
+    if (p.ws.xs) cudaFree(p.ws.xs);
+    p.ws.bw = p.ws.xs = nullptr;
     p.ws.w_bytes = 0;
-    if (cudaMalloc(&p.ws.w, std::max<size_t>(need, 256)) != cudaSuccess) {
+    // +256 B: the staged chain kernel's 16-byte-aligned TMA windows may read
+    // up to 15 bytes past the last row
+    if (cudaMalloc(&p.ws.bw, need + 256) != cudaSuccess || cudaMalloc(&p.ws.xs, need + 256) != cudaSuccess) {
       cudaGetLastError();
       return {SPTRSV_ERROR_ALLOC, "workspace allocation failed"};
     }
     p.ws.w_bytes = need;
   }
-  T* w = (T*)p.ws.w;
-  k::SolveState st{&p.d_state->epoch, p.d_state->tickets, p.nticket, p.d_error};
+  T* bw = (T*)p.ws.bw;
+  T* xs = (T*)p.ws.xs;
+  const T* rd = (const T*)p.d_rdiag;
+  const int fill = p.needs_sentinel ? 1 : 0;
+  k::SolveState st{p.d_tickets, p.nticket, p.d_error};
   cudaEvent_t* ev = nullptr;
   if (p.profiling) {
     size_t need_ev = p.segs.size() + 3;
@@ -191,26 +282,27 @@ Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs
   const int* iperm = p.d_perm + n;  // old -> new, stored right after perm
   if (nrhs == 1) {
     int64_t stride = layout == SPTRSV_ROW_MAJOR ? ldb : 1;
-    k::perm_in_1<T><<<std::max(1u, cdiv(n, 256)), 256, 0, s>>>(n, p.d_perm, b, stride, w, st);
+    k::perm_in_1<T><<<std::max(1u, cdiv(n, 256)), 256, 0, s>>>(n, p.d_perm, rd, b, stride, bw, xs, fill, st);
   } else if (layout == SPTRSV_COL_MAJOR) {
     dim3 g(std::max(1u, cdiv(n, 32)), cdiv(nrhs, 32));
-    k::perm_in_cm<T><<<g, dim3(32, 8), 0, s>>>(n, nrhs, iperm, b, ldb, w, st);
+    k::perm_in_cm<T><<<g, dim3(32, 8), 0, s>>>(n, nrhs, iperm, rd, b, ldb, bw, xs, fill, st);
   } else {
-    k::perm_in_rm<T><<<std::max(1u, cdiv((int64_t)n * nrhs, 256)), 256, 0, s>>>(n, nrhs, p.d_perm, b, ldb, w, st);
+    k::perm_in_rm<T><<<std::max(1u, cdiv((int64_t)n * nrhs, 256)), 256, 0, s>>>(n, nrhs, p.d_perm, rd, b, ldb, bw,
+                                                                                 xs, fill, st);
   }
   CUDA_TRY(cudaGetLastError());
   if (ev) CUDA_TRY(cudaEventRecord(ev[1], s));
-  Error e = run_segments<T>(p, w, nrhs, s, st, ev);
+  Error e = run_segments<T>(p, bw, xs, nrhs, s, st, ev);
   if (e.status) return e;
   CUDA_TRY(cudaGetLastError());
   if (nrhs == 1) {
     int64_t stride = layout == SPTRSV_ROW_MAJOR ? ldx : 1;
-    k::perm_out_1<T><<<std::max(1u, cdiv(n, 256)), 256, 0, s>>>(n, p.d_perm, w, x, stride);
+    k::perm_out_1<T><<<std::max(1u, cdiv(n, 256)), 256, 0, s>>>(n, p.d_perm, xs, x, stride);
   } else if (layout == SPTRSV_COL_MAJOR) {
     dim3 g(std::max(1u, cdiv(n, 32)), cdiv(nrhs, 32));
-    k::perm_out_cm<T><<<g, dim3(32, 8), 0, s>>>(n, nrhs, iperm, w, x, ldx);
+    k::perm_out_cm<T><<<g, dim3(32, 8), 0, s>>>(n, nrhs, iperm, xs, x, ldx);
   } else {
-    k::perm_out_rm<T><<<std::max(1u, cdiv((int64_t)n * nrhs, 256)), 256, 0, s>>>(n, nrhs, p.d_perm, w, x, ldx);
+    k::perm_out_rm<T><<<std::max(1u, cdiv((int64_t)n * nrhs, 256)), 256, 0, s>>>(n, nrhs, p.d_perm, xs, x, ldx);
   }
   CUDA_TRY(cudaGetLastError());
   if (ev) {
@@ -243,23 +335,25 @@ Error upload(Plan& p, void* stream_v) {
     return o;
   };
   size_t o_perm = take((size_t)2 * n * 4);  // perm (new->old) then iperm (old->new)
-  size_t o_diag = take((size_t)n * vb);
-  struct Offs { size_t rp, ci, val, rows, lp; };
+  size_t o_rdiag = take((size_t)n * vb);
+  struct Offs { size_t rp, ci, val, rows, lp, st; };
   std::vector<Offs> so(p.segs.size());
+  const k::ChainGeom cg = chain_geometry(p);
+  p.nticket = 0;
+  p.needs_sentinel = false;
   for (size_t i = 0; i < p.segs.size(); ++i) {
     Segment& S = p.segs[i];
+    build_chain_stages(S, cg);
     so[i].rp = take(S.rp.size() * 4);
     so[i].ci = take(S.ci.size() * 4);
     so[i].val = take(S.val.size());
     so[i].rows = take(S.rows.size() * 4);
     so[i].lp = take(S.level_ptr.size() * 4);
-  }
-  // sync-free tickets for every triangle (any may be forced later)
-  p.nticket = 0;
-  for (auto& S : p.segs)
+    so[i].st = take(S.chain_recs.size() * 4);
     if (S.info.kind == 0) S.ticket_slot = p.nticket++;
-  size_t o_flags = take((size_t)n * 4);
-  size_t o_state = take(sizeof(DevState) + (size_t)std::max(1, p.nticket) * 4);
+    if (S.info.kind == 0 && S.info.impl == SPTRSV_IMPL_TRI_SYNCFREE) p.needs_sentinel = true;
+  }
+  size_t o_tickets = take((size_t)std::max(1, p.nticket) * 4);
   p.arena_bytes = off;
 
   int dev;
@@ -277,7 +371,7 @@ Error upload(Plan& p, void* stream_v) {
   for (int k2 = 0; k2 < n; ++k2) iperm[p.perm[k2]] = k2;
   std::memcpy(&h[o_perm], p.perm.data(), (size_t)n * 4);
   std::memcpy(&h[o_perm + (size_t)n * 4], iperm.data(), (size_t)n * 4);
-  std::memcpy(&h[o_diag], p.diag_new.data(), (size_t)n * vb);
+  std::memcpy(&h[o_rdiag], p.rdiag_new.data(), (size_t)n * vb);
   char* A = (char*)p.arena;
   for (size_t i = 0; i < p.segs.size(); ++i) {
     Segment& S = p.segs[i];
@@ -286,16 +380,17 @@ Error upload(Plan& p, void* stream_v) {
     std::memcpy(&h[so[i].val], S.val.data(), S.val.size());
     std::memcpy(&h[so[i].rows], S.rows.data(), S.rows.size() * 4);
     std::memcpy(&h[so[i].lp], S.level_ptr.data(), S.level_ptr.size() * 4);
+    std::memcpy(&h[so[i].st], S.chain_recs.data(), S.chain_recs.size() * 4);
     S.d_rp = (const int32_t*)(A + so[i].rp);
     S.d_ci = (const int32_t*)(A + so[i].ci);
     S.d_val = (const void*)(A + so[i].val);
     S.d_rows = (const int32_t*)(A + so[i].rows);
     S.d_level_ptr = (const int32_t*)(A + so[i].lp);
+    S.d_chain_recs = (const int32_t*)(A + so[i].st);
   }
   p.d_perm = (const int32_t*)(A + o_perm);
-  p.d_diag = (const void*)(A + o_diag);
-  p.d_flags = (int32_t*)(A + o_flags);
-  p.d_state = (DevState*)(A + o_state);
+  p.d_rdiag = (const void*)(A + o_rdiag);
+  p.d_tickets = (uint32_t*)(A + o_tickets);
   CUDA_TRY(cudaMemcpyAsync(p.arena, h.data(), off, cudaMemcpyHostToDevice, s));
   // mapped host word for the spin-wait watchdog
   if (cudaHostAlloc((void**)&p.h_error, sizeof(int32_t), cudaHostAllocMapped) == cudaSuccess) {
@@ -373,7 +468,8 @@ Error solve(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t n
 void release(Plan& p) {
   if (p.device >= 0) cudaDeviceSynchronize();
   if (p.arena) cudaFree(p.arena);
-  if (p.ws.w) cudaFree(p.ws.w);
+  if (p.ws.bw) cudaFree(p.ws.bw);
+  if (p.ws.xs) cudaFree(p.ws.xs);
   if (p.ws.stage_b) cudaFree(p.ws.stage_b);
   if (p.ws.stage_x) cudaFree(p.ws.stage_x);
   if (p.h_error) cudaFreeHost(p.h_error);

@@ -41,17 +41,15 @@ struct Segment {
   const int32_t* d_rows = nullptr;
   const int32_t* d_level_ptr = nullptr;  // device copy (chain / level-set kernels)
   int32_t ticket_slot = -1;              // sync-free: index into the device ticket array
-};
-
-// Mutable per-solve device state (one per plan).
-struct DevState {
-  uint32_t epoch;      // incremented by permute-in; ready flag == epoch means solved
-  uint32_t pad[3];
-  uint32_t tickets[1]; // [nticket] row-claim counters, zeroed by permute-in
+  // TMA-staged chain kernel (nrhs == 1): 8-int stage records (k::StageRec),
+  // empty = not staged
+  std::vector<int32_t> chain_recs;
+  const int32_t* d_chain_recs = nullptr;
 };
 
 struct Workspace {
-  void* w = nullptr;        // permuted solution/rhs, n x nrhs row-major
+  void* bw = nullptr;       // permuted right-hand side being updated, n x nrhs row-major
+  void* xs = nullptr;       // permuted solution, n x nrhs row-major
   size_t w_bytes = 0;
   void* stage_b = nullptr;  // host-pointer path staging (col-major n x nrhs)
   void* stage_x = nullptr;
@@ -74,6 +72,7 @@ struct Plan {
   std::vector<int32_t> perm;        // new -> old (original indexing; UPPER composed with J)
   std::vector<int32_t> leaf_level;  // level of every new row inside its leaf
   std::vector<char> diag_new;       // diagonal in new order (dtype)
+  std::vector<char> rdiag_new;      // 1 / diagonal in new order (dtype), what kernels read
   // P L P^T kept on the host for introspection (sptrsv_plan_matrix)
   std::vector<int64_t> p_rp;
   std::vector<int32_t> p_ci;
@@ -84,10 +83,10 @@ struct Plan {
   void* arena = nullptr;
   size_t arena_bytes = 0;
   const int32_t* d_perm = nullptr;
-  const void* d_diag = nullptr;
-  int32_t* d_flags = nullptr;  // per-row ready flags (sync-free)
-  DevState* d_state = nullptr;
+  const void* d_rdiag = nullptr;  // 1/d in new order (permute-in scaling)
+  uint32_t* d_tickets = nullptr;  // [nticket] sync-free row-claim counters
   int32_t nticket = 0;
+  bool needs_sentinel = false;    // a sync-free triangle polls xs
   int32_t* h_error = nullptr;  // mapped pinned host word set by the watchdog
   int32_t* d_error = nullptr;  // its device alias
   Workspace ws;
