@@ -65,6 +65,12 @@ k::ChainGeom chain_geometry(const Plan& p) {
                        : k::chain_geom<float>(NST, RMAX, EMAX, XW, LMAX);
 }
 
+k::ChainGeom frozen_geometry(const Plan& p) {
+  const int* g = p.chain_geom;
+  return p.vbytes == 8 ? k::chain_geom<double>(g[0], g[1], g[2], g[3], g[4])
+                       : k::chain_geom<float>(g[0], g[1], g[2], g[3], g[4]);
+}
+
 // Cut a chain triangle into stages of whole levels (rows <= RMAX, entries <=
 // EMAX, levels <= LMAX); a level that does not fit is split by rows.  Leaves
 // chain_recs empty when one row has more than EMAX entries (the unstaged
@@ -101,18 +107,150 @@ void build_chain_stages(Segment& S, const k::ChainGeom& g) {
     }
   }
   close(m);
-  // records {sa, sb, e0, e1, l0, nl, 0, 0}
+  // records {sa, sb, e0, e1, l0, nl, 0, 0}, each followed by the record of
+  // stage s + NST (the one the producer issues when stage s is done)
   const int ns = (int)st.size() - 1;
-  S.chain_recs.assign((size_t)ns * 8, 0);
+  S.chain_recs.assign((size_t)ns * 16, 0);
   int l = 0;
   for (int s = 0; s < ns; ++s) {
     int sa = st[s], sb = st[s + 1];
     while (S.level_ptr[l + 1] <= sa) ++l;  // level containing sa
     int l_last = l;
     while (S.level_ptr[l_last + 1] < sb) ++l_last;  // level containing sb-1
-    int32_t* R = &S.chain_recs[(size_t)s * 8];
+    int32_t* R = &S.chain_recs[(size_t)s * 16];
     R[0] = sa; R[1] = sb; R[2] = S.rp[sa]; R[3] = S.rp[sb]; R[4] = l; R[5] = l_last - l + 2;
   }
+  for (int s = 0; s + g.NST < ns; ++s)
+    std::memcpy(&S.chain_recs[(size_t)s * 16 + 8], &S.chain_recs[(size_t)(s + g.NST) * 16], 32);
+}
+
+// ELL-staged chain (see k::tri_chain_ell): eligible when every row has <= 4
+// dependencies, all inside the x window of their level.  Geometry: RMAX rows
+// per stage, as many stages as fit in 227 KB next to the window.
+void build_chain_ell(Segment& S, size_t vb) {
+  S.ell_K = 0;
+  S.ell_recs.clear();
+  S.ell_data.clear();
+  const auto& I = S.info;
+  if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_CHAIN || I.nlevels < 2) return;
+  if (const char* e = std::getenv("SPTRSV_ELL"))
+    if (e[0] == '0') return;
+  const int m = I.row1 - I.row0;
+  int K = 0;
+  for (int r = 0; r < m; ++r) K = std::max(K, S.rp[r + 1] - S.rp[r]);
+  if (K < 1 || K > 4) return;
+  int RMAX = 2048, XW = 4096, NSTMAX = 4;
+  if (const char* e = std::getenv("SPTRSV_ELL_GEOM")) {
+    int a, b, c;
+    if (std::sscanf(e, "%d,%d,%d", &a, &b, &c) == 3 && a >= 1 && b >= 2 && (b & (b - 1)) == 0 && c >= 2) {
+      RMAX = a; XW = b; NSTMAX = c;
+    }
+  }
+  // every dependency of a row in level l must satisfy j >= end(l) - XW
+  for (int l = 0; l < I.nlevels; ++l) {
+    const int L1 = S.level_ptr[l + 1];
+    for (int r = S.level_ptr[l]; r < L1; ++r)
+      for (int q = S.rp[r]; q < S.rp[r + 1]; ++q)
+        if (S.ci[q] - I.row0 < L1 - XW) return;
+  }
+  const uint32_t sb_bytes = vb == 8 ? k::ell_stage_bytes<double>(K, RMAX) : k::ell_stage_bytes<float>(K, RMAX);
+  const uint32_t fixed = k::al16((XW + 2) * (uint32_t)vb) + 256;
+  const int NST = std::min<int>(NSTMAX, (int)((232448 - fixed) / (sb_bytes + 16)));
+  if (NST < 2) return;
+  // stage boundaries: whole levels where possible (<= RMAX rows, <= 256 levels)
+  std::vector<int32_t> st = {0};
+  int cur_r = 0, cur_l = 0;
+  for (int l = 0; l < I.nlevels; ++l) {
+    const int la = S.level_ptr[l], lb = S.level_ptr[l + 1], lr = lb - la;
+    if (cur_r + lr <= RMAX && cur_l + 1 <= 256) {
+      cur_r += lr;
+      cur_l += 1;
+      continue;
+    }
+    if (la > st.back()) st.push_back(la);
+    cur_r = cur_l = 0;
+    if (lr <= RMAX) {
+      cur_r = lr;
+      cur_l = 1;
+      continue;
+    }
+    for (int r = la + RMAX; r < lb; r += RMAX) st.push_back(r);  // split a wide level
+    cur_r = lb - st.back();
+    cur_l = 1;
+  }
+  if (m > st.back()) st.push_back(m);
+  const int ns = (int)st.size() - 1;
+  S.ell_recs.assign((size_t)ns * 16, 0);
+  size_t off = 0;
+  std::vector<size_t> offs(ns);
+  for (int q = 0; q < ns; ++q) {
+    const int n = st[q + 1] - st[q], npad = (n + 3) & ~3;
+    offs[q] = off;
+    off += k::al16(K * npad * 4) + k::al16(K * npad * (uint32_t)vb);
+  }
+  S.ell_data.assign(off, 0);
+  int l = 0;
+  for (int q = 0; q < ns; ++q) {
+    const int sa = st[q], sb = st[q + 1], n = sb - sa, npad = (n + 3) & ~3;
+    while (S.level_ptr[l + 1] <= sa) ++l;
+    int l_last = l;
+    while (S.level_ptr[l_last + 1] < sb) ++l_last;
+    int32_t* R = &S.ell_recs[(size_t)q * 16];
+    R[0] = sa; R[1] = sb; R[2] = l; R[3] = l_last - l + 2; R[4] = (int32_t)(offs[q] / 16); R[5] = npad;
+    int32_t* slots = (int32_t*)&S.ell_data[offs[q]];
+    char* vals = &S.ell_data[offs[q] + k::al16(K * npad * 4)];
+    for (int kk = 0; kk < K; ++kk)
+      for (int i = 0; i < npad; ++i) slots[kk * npad + i] = XW;  // the zero slot
+    for (int i = 0; i < n; ++i) {
+      const int r = sa + i;
+      int kk = 0;
+      for (int qq = S.rp[r]; qq < S.rp[r + 1]; ++qq, ++kk) {
+        slots[kk * npad + i] = (S.ci[qq] - I.row0) & (XW - 1);
+        std::memcpy(vals + ((size_t)kk * npad + i) * vb, &S.val[(size_t)qq * vb], vb);
+      }
+    }
+  }
+  for (int q = 0; q + NST < ns; ++q)
+    std::memcpy(&S.ell_recs[(size_t)q * 16 + 8], &S.ell_recs[(size_t)(q + NST) * 16], 32);
+  // consumer warps: cover the 90th-percentile level width with 2 rows/thread
+  std::vector<int> widths(I.nlevels);
+  for (int q = 0; q < I.nlevels; ++q) widths[q] = S.level_ptr[q + 1] - S.level_ptr[q];
+  std::nth_element(widths.begin(), widths.begin() + (I.nlevels * 9) / 10, widths.end());
+  int w90 = widths[(I.nlevels * 9) / 10];
+  // measured on B200 (C2): per-level cost is issue-bound and grows ~13
+  // cycles per extra warp, so 8..12 warps x 2 rows beat 31 warps x 1 row
+  int warps = std::max(4, std::min(12, (w90 + 2 * 32 - 1) / (2 * 32)));
+  if (const char* e = std::getenv("SPTRSV_ELL_WARPS")) warps = std::atoi(e);
+  S.ell_warps = std::max(1, std::min(31, warps));
+  S.ell_K = K;
+  S.ell_NST = NST;
+  S.ell_RMAX = RMAX;
+  S.ell_XW = XW;
+}
+
+template <typename T, int K>
+Error launch_chain_ell(Plan& p, Segment& S, const T* bw, T* xs, cudaStream_t s) {
+  const int NST = S.ell_NST, RMAX = S.ell_RMAX, XW = S.ell_XW;
+  const uint32_t smem = NST * k::ell_stage_bytes<T>(K, RMAX) + k::al16((XW + 2) * (uint32_t)sizeof(T)) + NST * 16;
+  constexpr int RPT = 2;
+  static uint32_t attr_bytes = 0;  // per template instance
+  if (smem > attr_bytes) {
+    CUDA_TRY(cudaFuncSetAttribute(k::tri_chain_ell<T, K, RPT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)smem));
+    attr_bytes = smem;
+  }
+  // consumer warps: enough that NC * RPT covers a typical level, at most 31
+  int nc_warps = S.ell_warps;
+  const int nst = (int)(S.ell_recs.size() / 16);
+  long long* tr = nullptr;
+  if (p.trace) {
+    if (S.h_trace.size() < (size_t)nst * 3) S.h_trace.assign((size_t)nst * 3, 0);
+    if (!S.d_trace) CUDA_TRY(cudaMalloc(&S.d_trace, (size_t)nst * 3 * 8));
+    tr = (long long*)S.d_trace;
+  }
+  k::tri_chain_ell<T, K, RPT><<<1, 32 * (nc_warps + 1), smem, s>>>(
+      S.info.row0, nst, (const k::EllRec*)S.d_ell_recs, S.d_level_ptr, S.d_ell_data, bw, xs, NST, RMAX, XW, tr);
+  return {SPTRSV_SUCCESS, ""};
 }
 
 template <typename T>
@@ -178,8 +316,17 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
           break;
         }
         case SPTRSV_IMPL_TRI_CHAIN: {
-          if (nrhs == 1 && !S.chain_recs.empty()) {
-            const k::ChainGeom cg = chain_geometry(p);
+          if (nrhs == 1 && S.ell_K > 0) {
+            Error e;
+            switch (S.ell_K) {
+              case 1: e = launch_chain_ell<T, 1>(p, S, bw, xs, s); break;
+              case 2: e = launch_chain_ell<T, 2>(p, S, bw, xs, s); break;
+              case 3: e = launch_chain_ell<T, 3>(p, S, bw, xs, s); break;
+              default: e = launch_chain_ell<T, 4>(p, S, bw, xs, s); break;
+            }
+            if (e.status) return e;
+          } else if (nrhs == 1 && !S.chain_recs.empty()) {
+            const k::ChainGeom cg = frozen_geometry(p);
             const uint32_t smem = k::chain_smem_bytes<T>(cg);
             static uint32_t attr_bytes = 0;  // per template instance
             if (smem > attr_bytes) {
@@ -187,9 +334,15 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
                                             (int)smem));
               attr_bytes = smem;
             }
-            k::tri_chain_tma<T><<<1, 1024, smem, s>>>(I.row0, (int)(S.chain_recs.size() / 8),
-                                                      (const k::StageRec*)S.d_chain_recs, S.d_level_ptr, S.d_rp,
-                                                      S.d_ci, val, bw, xs, cg);
+            const int nst = (int)(S.chain_recs.size() / 16);
+            long long* tr = nullptr;
+            if (p.trace) {  // debug: SPTRSV_TRACE=1, per-stage clock64 stamps
+              if (S.h_trace.size() < (size_t)nst * 3) S.h_trace.assign((size_t)nst * 3, 0);
+              if (!S.d_trace) CUDA_TRY(cudaMalloc(&S.d_trace, (size_t)nst * 3 * 8));
+              tr = (long long*)S.d_trace;
+            }
+            k::tri_chain_tma<T><<<1, 1024, smem, s>>>(I.row0, nst, (const k::StageRec*)S.d_chain_recs,
+                                                      S.d_level_ptr, S.d_rp, S.d_ci, val, bw, xs, cg, tr);
           } else if (nrhs == 1) {
             if (tri_use_warp(S))
               k::tri_chain_1<T, true><<<1, 1024, 0, s>>>(I.row0, I.nlevels, S.d_level_ptr, S.d_rp, S.d_ci, val,
@@ -243,6 +396,30 @@ int count_launches(const Plan& p) {
     }
   }
   return c;
+}
+
+// Debug (SPTRSV_TRACE=1): per-stage cycle breakdown of the staged chain
+// kernel -- time spent waiting for the TMA stage vs walking its levels.
+void dump_trace(Plan& p, cudaStream_t s) {
+  cudaStreamSynchronize(s);
+  for (size_t si = 0; si < p.segs.size(); ++si) {
+    Segment& S = p.segs[si];
+    if (!S.d_trace) continue;
+    const int nst = S.ell_K ? (int)(S.ell_recs.size() / 16) : (int)(S.chain_recs.size() / 16);
+    cudaMemcpy(S.h_trace.data(), S.d_trace, (size_t)nst * 24, cudaMemcpyDeviceToHost);
+    long long wait = 0, work = 0, gap = 0;
+    for (int k2 = 0; k2 < nst; ++k2) {
+      wait += S.h_trace[3 * k2 + 1] - S.h_trace[3 * k2];
+      work += S.h_trace[3 * k2 + 2] - S.h_trace[3 * k2 + 1];
+      if (k2) gap += S.h_trace[3 * k2] - S.h_trace[3 * k2 - 1];
+    }
+    long long tot = S.h_trace[3 * nst - 1] - S.h_trace[0];
+    std::fprintf(stderr,
+                 "[sptrsv trace] seg %zu: %d stages, %d levels, %lld cycles: tma-wait %.1f%%, walk %.1f%%, "
+                 "issue %.1f%%; per stage %.0f cycles, per level %.0f cycles\n",
+                 si, nst, S.info.nlevels, tot, 100.0 * wait / tot, 100.0 * work / tot, 100.0 * gap / tot,
+                 (double)tot / nst, (double)tot / S.info.nlevels);
+  }
 }
 
 template <typename T>
@@ -309,6 +486,7 @@ Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs
     CUDA_TRY(cudaEventRecord(ev[2 + p.segs.size()], s));
     p.last_nseg_timed = (int)p.segs.size();
   }
+  if (p.trace) dump_trace(p, s);
   return {SPTRSV_SUCCESS, ""};
 }
 
@@ -336,14 +514,20 @@ Error upload(Plan& p, void* stream_v) {
   };
   size_t o_perm = take((size_t)2 * n * 4);  // perm (new->old) then iperm (old->new)
   size_t o_rdiag = take((size_t)n * vb);
-  struct Offs { size_t rp, ci, val, rows, lp, st; };
+  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed; };
   std::vector<Offs> so(p.segs.size());
+  p.trace = std::getenv("SPTRSV_TRACE") != nullptr;
   const k::ChainGeom cg = chain_geometry(p);
+  p.chain_geom[0] = cg.NST; p.chain_geom[1] = cg.RMAX; p.chain_geom[2] = cg.EMAX;
+  p.chain_geom[3] = cg.XW; p.chain_geom[4] = cg.LMAX;
   p.nticket = 0;
   p.needs_sentinel = false;
   for (size_t i = 0; i < p.segs.size(); ++i) {
     Segment& S = p.segs[i];
     build_chain_stages(S, cg);
+    build_chain_ell(S, vb);
+    so[i].er = take(S.ell_recs.size() * 4);
+    so[i].ed = take(S.ell_data.size());
     so[i].rp = take(S.rp.size() * 4);
     so[i].ci = take(S.ci.size() * 4);
     so[i].val = take(S.val.size());
@@ -387,6 +571,10 @@ Error upload(Plan& p, void* stream_v) {
     S.d_rows = (const int32_t*)(A + so[i].rows);
     S.d_level_ptr = (const int32_t*)(A + so[i].lp);
     S.d_chain_recs = (const int32_t*)(A + so[i].st);
+    std::memcpy(&h[so[i].er], S.ell_recs.data(), S.ell_recs.size() * 4);
+    std::memcpy(&h[so[i].ed], S.ell_data.data(), S.ell_data.size());
+    S.d_ell_recs = (const int32_t*)(A + so[i].er);
+    S.d_ell_data = (const char*)(A + so[i].ed);
   }
   p.d_perm = (const int32_t*)(A + o_perm);
   p.d_rdiag = (const void*)(A + o_rdiag);
@@ -473,6 +661,8 @@ void release(Plan& p) {
   if (p.ws.stage_b) cudaFree(p.ws.stage_b);
   if (p.ws.stage_x) cudaFree(p.ws.stage_x);
   if (p.h_error) cudaFreeHost(p.h_error);
+  for (auto& S : p.segs)
+    if (S.d_trace) cudaFree(S.d_trace);
   for (void* e : p.events) cudaEventDestroy((cudaEvent_t)e);
   p.arena = nullptr;
   p.ws = Workspace{};

@@ -45,6 +45,14 @@ struct Segment {
   // empty = not staged
   std::vector<int32_t> chain_recs;
   const int32_t* d_chain_recs = nullptr;
+  // ELL-staged chain kernel (nrhs == 1, rows with <= 4 window-resident deps)
+  int ell_K = 0, ell_NST = 0, ell_RMAX = 0, ell_XW = 0, ell_warps = 8;  // ell_K == 0: not used
+  std::vector<int32_t> ell_recs;   // 16 ints per stage (k::EllRec + the record of stage s + NST)
+  std::vector<char> ell_data;      // per-stage blocks: slots[K][npad] int32, values[K][npad]
+  const int32_t* d_ell_recs = nullptr;
+  const char* d_ell_data = nullptr;
+  void* d_trace = nullptr;          // debug trace (SPTRSV_TRACE)
+  std::vector<long long> h_trace;
 };
 
 struct Workspace {
@@ -87,6 +95,8 @@ struct Plan {
   uint32_t* d_tickets = nullptr;  // [nticket] sync-free row-claim counters
   int32_t nticket = 0;
   bool needs_sentinel = false;    // a sync-free triangle polls xs
+  int chain_geom[5] = {0, 0, 0, 0, 0};  // NST, RMAX, EMAX, XW, LMAX frozen at upload
+  bool trace = false;                   // SPTRSV_TRACE debug stamps
   int32_t* h_error = nullptr;  // mapped pinned host word set by the watchdog
   int32_t* d_error = nullptr;  // its device alias
   Workspace ws;

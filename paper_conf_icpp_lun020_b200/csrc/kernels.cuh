@@ -529,9 +529,9 @@ __global__ void __launch_bounds__(256) tri_syncfree_multi(int r0, int m, const i
 //
 // Stage s (a record computed by the analysis) covers local rows [sa, sb) --
 // whole levels where possible -- with their entries [e0, e1) and level
-// pointers lp[l0 .. l0+nl-1].  The record itself travels in the stage buffer,
-// so consumers never touch global memory for control; thread 0 keeps the
-// records of the stages it will issue next in registers.
+// pointers lp[l0 .. l0+nl-1].  recs[2s] is stage s's record and recs[2s+1]
+// the record of stage s+NST; both travel in stage s's buffer, so neither the
+// consumers nor the producer (thread 0) touch global memory for control.
 struct StageRec {
   int sa, sb, e0, e1, l0, nl, pad0, pad1;
 };
@@ -583,12 +583,12 @@ __host__ __device__ inline ChainGeom chain_geom(int NST, int RMAX, int EMAX, int
   g.cap_val = al16((EMAX + 4) * (uint32_t)sizeof(T));
   g.cap_v = al16((RMAX + 4) * (uint32_t)sizeof(T));
   g.cap_lp = al16((LMAX + 8) * 4);
-  g.stage_bytes = 32 + g.cap_rp + g.cap_ci + g.cap_val + g.cap_v + g.cap_lp;
+  g.stage_bytes = 64 + g.cap_rp + g.cap_ci + g.cap_val + g.cap_v + g.cap_lp;
   return g;
 }
 template <typename T>
 __host__ __device__ inline uint32_t chain_smem_bytes(const ChainGeom& g) {
-  return g.NST * g.stage_bytes + g.XW * (uint32_t)sizeof(T) + g.NST * 8;
+  return g.NST * g.stage_bytes + g.XW * (uint32_t)sizeof(T) + g.NST * 16;  // + full/empty mbarriers
 }
 
 // 16-byte aligned window around element range [first, first+count)
@@ -612,14 +612,22 @@ template <typename T>
 __global__ void __launch_bounds__(1024, 1)
     tri_chain_tma(int r0, int nstage, const StageRec* __restrict__ recs, const int* __restrict__ lp,
                   const int* __restrict__ rp, const int* __restrict__ ci, const T* __restrict__ val,
-                  const T* __restrict__ bw, T* __restrict__ xs, ChainGeom g) {
+                  const T* __restrict__ bw, T* __restrict__ xs, ChainGeom g, long long* __restrict__ trace) {
+  // Warp-specialised: the last warp is the TMA producer, the other warps
+  // (NC threads) walk the levels and synchronise on named barrier 1, so the
+  // copy issue never sits on the dependency chain.
   extern __shared__ __align__(128) unsigned char smem[];
-  const int tid = threadIdx.x, nt = blockDim.x;
+  const int tid = threadIdx.x;
+  const int NC = blockDim.x - 32;
   const int xmask = g.XW - 1;  // XW is a power of two
   T* xw = (T*)(smem + g.NST * g.stage_bytes);
-  uint64_t* bars = (uint64_t*)(smem + g.NST * g.stage_bytes + g.XW * sizeof(T));
+  uint64_t* full = (uint64_t*)(smem + g.NST * g.stage_bytes + g.XW * sizeof(T));
+  uint64_t* empty = full + g.NST;
   if (tid == 0) {
-    for (int b = 0; b < g.NST; ++b) mbar_init(&bars[b], 1);
+    for (int b = 0; b < g.NST; ++b) {
+      mbar_init(&full[b], 1);
+      mbar_init(&empty[b], 1);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
@@ -636,78 +644,268 @@ __global__ void __launch_bounds__(1024, 1)
     unsigned char* base = smem + (size_t)b * g.stage_bytes;
     Bufs B;
     B.rec = (StageRec*)base;
-    B.rp = (int*)(base + 32);
-    B.ci = (int*)(base + 32 + g.cap_rp);
-    B.val = (T*)(base + 32 + g.cap_rp + g.cap_ci);
-    B.b = (T*)(base + 32 + g.cap_rp + g.cap_ci + g.cap_val);
-    B.lp = (int*)(base + 32 + g.cap_rp + g.cap_ci + g.cap_val + g.cap_v);
+    B.rp = (int*)(base + 64);
+    B.ci = (int*)(base + 64 + g.cap_rp);
+    B.val = (T*)(base + 64 + g.cap_rp + g.cap_ci);
+    B.b = (T*)(base + 64 + g.cap_rp + g.cap_ci + g.cap_val);
+    B.lp = (int*)(base + 64 + g.cap_rp + g.cap_ci + g.cap_val + g.cap_v);
     return B;
   };
-  auto issue = [&](int s, const StageRec& R) {
-    const int b = s % g.NST;
-    Bufs B = bufs(b);
-    Win wr = win(rp, R.sa, R.sb - R.sa + 1);
-    Win wc = win(ci, R.e0, R.e1 - R.e0);
-    Win wv = win(val, R.e0, R.e1 - R.e0);
-    Win wb = win(bw, (int64_t)r0 + R.sa, R.sb - R.sa);
-    Win wl = win(lp, R.l0, R.nl);
-    const bool ents = R.e1 > R.e0;
-    uint32_t tot = 32 + wr.bytes + wb.bytes + wl.bytes + (ents ? wc.bytes + wv.bytes : 0u);
-    mbar_expect_tx(&bars[b], tot);
-    tma_bulk_g2s(B.rec, recs + s, 32, &bars[b]);
-    tma_bulk_g2s(B.rp, wr.src, wr.bytes, &bars[b]);
-    if (ents) {
-      tma_bulk_g2s(B.ci, wc.src, wc.bytes, &bars[b]);
-      tma_bulk_g2s(B.val, wv.src, wv.bytes, &bars[b]);
+
+  if (tid >= NC) {  // ---------------- producer warp
+    if (tid == NC) {
+      int b = 0;
+      uint32_t ph = 0;
+      for (int s = 0; s < nstage; ++s) {
+        Bufs B = bufs(b);
+        StageRec R;
+        if (s < g.NST) {
+          R = recs[2 * s];
+        } else {
+          mbar_wait(&empty[b], ph ^ 1u);  // consumers released stage s - NST
+          R = B.rec[1];                   // stage s's record rode in with stage s - NST
+        }
+        Win wr = win(rp, R.sa, R.sb - R.sa + 1);
+        Win wc = win(ci, R.e0, R.e1 - R.e0);
+        Win wv = win(val, R.e0, R.e1 - R.e0);
+        Win wb = win(bw, (int64_t)r0 + R.sa, R.sb - R.sa);
+        Win wl = win(lp, R.l0, R.nl);
+        const bool ents = R.e1 > R.e0;
+        uint32_t tot = 64 + wr.bytes + wb.bytes + wl.bytes + (ents ? wc.bytes + wv.bytes : 0u);
+        mbar_expect_tx(&full[b], tot);
+        tma_bulk_g2s(B.rec, recs + 2 * s, 64, &full[b]);
+        tma_bulk_g2s(B.rp, wr.src, wr.bytes, &full[b]);
+        if (ents) {
+          tma_bulk_g2s(B.ci, wc.src, wc.bytes, &full[b]);
+          tma_bulk_g2s(B.val, wv.src, wv.bytes, &full[b]);
+        }
+        tma_bulk_g2s(B.b, wb.src, wb.bytes, &full[b]);
+        tma_bulk_g2s(B.lp, wl.src, wl.bytes, &full[b]);
+        if (++b == g.NST) {
+          b = 0;
+          ph ^= 1u;
+        }
+      }
     }
-    tma_bulk_g2s(B.b, wb.src, wb.bytes, &bars[b]);
-    tma_bulk_g2s(B.lp, wl.src, wl.bytes, &bars[b]);
-  };
-  StageRec nxt{};
-  if (tid == 0) {
-    for (int s = 0; s < g.NST && s < nstage; ++s) issue(s, recs[s]);
-    if (g.NST < nstage) nxt = recs[g.NST];
+    return;
   }
 
+  // ---------------- consumer warps
+  int b = 0;
+  uint32_t ph = 0;
   for (int s = 0; s < nstage; ++s) {
-    const int b = s % g.NST;
-    mbar_wait(&bars[b], (uint32_t)((s / g.NST) & 1));
+    long long t0 = 0;
+    if (trace && tid == 0) t0 = clock64();
+    mbar_wait(&full[b], ph);
+    if (trace && tid == 0) {
+      trace[3 * s] = t0;
+      trace[3 * s + 1] = clock64();
+    }
     const Bufs B = bufs(b);
-    const StageRec R = *B.rec;
-    StageRec nxt2{};
-    if (tid == 0 && s + g.NST + 1 < nstage) nxt2 = recs[s + g.NST + 1];  // lands during this stage
+    const StageRec R = B.rec[0];
     const int* s_rp = B.rp + shift_of(rp, R.sa);
     const int* s_ci = B.ci + shift_of(ci, R.e0);
     const T* s_val = B.val + shift_of(val, R.e0);
     const T* s_b = B.b + shift_of(bw, (int64_t)r0 + R.sa);
     const int* s_lp = B.lp + shift_of(lp, R.l0);
-    bool synced = false;
     for (int li = 0; li + 1 < R.nl; ++li) {
       const int L0 = s_lp[li], L1 = s_lp[li + 1];
       const int la = max(L0, R.sa), lb = min(L1, R.sb);
       const int xlo = L1 - g.XW;  // deps >= xlo are in the window
-      for (int r = la + tid; r < lb; r += nt) {
+      for (int r = la + tid; r < lb; r += NC) {
         const int i = r - R.sa;
         const int p0 = s_rp[i] - R.e0, p1 = s_rp[i + 1] - R.e0;
         T acc = s_b[i];
-        for (int p = p0; p < p1; ++p) {
-          const int j = s_ci[p] - r0;
-          const T xj = j >= xlo ? xw[j & xmask] : xs[r0 + j];
-          acc -= s_val[p] * xj;
+        int p = p0;
+        for (; p + 1 < p1; p += 2) {  // two independent dependency loads in flight
+          const int j0 = s_ci[p] - r0, j1 = s_ci[p + 1] - r0;
+          const T v0 = s_val[p], v1 = s_val[p + 1];
+          const T x0 = j0 >= xlo ? xw[j0 & xmask] : xs[r0 + j0];
+          const T x1 = j1 >= xlo ? xw[j1 & xmask] : xs[r0 + j1];
+          acc -= v0 * x0;
+          acc -= v1 * x1;
+        }
+        if (p < p1) {
+          const int j0 = s_ci[p] - r0;
+          const T x0 = j0 >= xlo ? xw[j0 & xmask] : xs[r0 + j0];
+          acc -= s_val[p] * x0;
         }
         xw[r & xmask] = acc;
         xs[r0 + r] = acc;
       }
-      synced = false;
-      if (L1 <= R.sb) {
-        __syncthreads();  // level barrier (Alg 2 L96)
-        synced = true;
+      // level barrier (Alg 2 L96) -- also at a stage end that splits a
+      // level, so the buffer can be released below
+      asm volatile("bar.sync 1, %0;" ::"r"(NC) : "memory");
+    }
+    if (trace && tid == 0) trace[3 * s + 2] = clock64();
+    if (tid == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(&empty[b])) : "memory");
+    if (++b == g.NST) {
+      b = 0;
+      ph ^= 1u;
+    }
+  }
+}
+
+// ------------------------- K4 (staged, ELL): narrow rows, window-resident deps
+// When every row of a chain triangle has at most K dependencies and every
+// dependency lies inside the x window of its level (both checked by the
+// analysis), each stage ships an ELL block instead of CSR: for slot k and
+// stage row i, the dependency's WINDOW SLOT (j mod XW; XW = a zero slot for
+// padding) and its value, column-major so lanes read consecutive words.  A
+// row is then K x {LDS slot, LDS value, LDS x, DFMA}: no row pointers, no
+// branches, no modulo on the dependency chain.
+struct EllRec {
+  int sa, sb, l0, nl, off16, npad, pad0, pad1;  // off16: stage block offset in 16-byte units
+};
+
+template <typename T>
+__host__ __device__ inline uint32_t ell_stage_bytes(int K, int RMAX) {
+  const int npad = (RMAX + 3) & ~3;
+  return 64 + al16(K * npad * 4) + al16(K * npad * (uint32_t)sizeof(T)) + al16((RMAX + 4) * (uint32_t)sizeof(T)) +
+         al16((RMAX + 8) * 4);
+}
+
+template <typename T, int K, int RPT>
+__global__ void __launch_bounds__(1024, 1)
+    tri_chain_ell(int r0, int nstage, const EllRec* __restrict__ recs, const int* __restrict__ lp,
+                  const char* __restrict__ ell, const T* __restrict__ bw, T* __restrict__ xs, int NST, int RMAX,
+                  int XW, long long* __restrict__ trace) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  const int tid = threadIdx.x;
+  const int NC = blockDim.x - 32;
+  const int xmask = XW - 1;
+  const int npad_max = (RMAX + 3) & ~3;
+  const uint32_t cap_idx = al16(K * npad_max * 4), cap_val = al16(K * npad_max * (uint32_t)sizeof(T));
+  const uint32_t cap_b = al16((RMAX + 4) * (uint32_t)sizeof(T));
+  const uint32_t sbytes = ell_stage_bytes<T>(K, RMAX);
+  T* xw = (T*)(smem + NST * sbytes);  // XW slots + one zero slot
+  uint64_t* full = (uint64_t*)(smem + NST * sbytes + al16((XW + 2) * (uint32_t)sizeof(T)));
+  uint64_t* empty = full + NST;
+  if (tid == 0) {
+    for (int b = 0; b < NST; ++b) {
+      mbar_init(&full[b], 1);
+      mbar_init(&empty[b], 1);
+    }
+    xw[XW] = T(0);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  auto base_of = [&](int b) { return smem + (size_t)b * sbytes; };
+
+  if (tid >= NC) {  // ---------------- producer warp
+    if (tid == NC) {
+      int b = 0;
+      uint32_t ph = 0;
+      for (int s = 0; s < nstage; ++s) {
+        unsigned char* B = base_of(b);
+        EllRec R;
+        if (s < NST) {
+          R = recs[2 * s];
+        } else {
+          mbar_wait(&empty[b], ph ^ 1u);
+          R = ((const EllRec*)B)[1];
+        }
+        const int n = R.sb - R.sa;
+        const uint32_t blk_idx = al16(K * R.npad * 4), blk_val = al16(K * R.npad * (uint32_t)sizeof(T));
+        Win wb = win(bw, (int64_t)r0 + R.sa, n);
+        Win wl = win(lp, R.l0, R.nl);
+        uint32_t tot = 64 + blk_idx + blk_val + wb.bytes + wl.bytes;
+        mbar_expect_tx(&full[b], tot);
+        tma_bulk_g2s(B, recs + 2 * s, 64, &full[b]);
+        const char* src = ell + (size_t)R.off16 * 16;
+        tma_bulk_g2s(B + 64, src, blk_idx, &full[b]);
+        tma_bulk_g2s(B + 64 + cap_idx, src + blk_idx, blk_val, &full[b]);
+        tma_bulk_g2s(B + 64 + cap_idx + cap_val, wb.src, wb.bytes, &full[b]);
+        tma_bulk_g2s(B + 64 + cap_idx + cap_val + cap_b, wl.src, wl.bytes, &full[b]);
+        if (++b == NST) {
+          b = 0;
+          ph ^= 1u;
+        }
       }
     }
-    if (!synced) __syncthreads();  // every thread is done with buffer b
-    if (tid == 0 && s + g.NST < nstage) {
-      issue(s + g.NST, nxt);
-      nxt = nxt2;
+    return;
+  }
+
+  int b = 0;
+  uint32_t ph = 0;
+  for (int s = 0; s < nstage; ++s) {
+    long long t0 = 0;
+    if (trace && tid == 0) t0 = clock64();
+    mbar_wait(&full[b], ph);
+    if (trace && tid == 0) {
+      trace[3 * s] = t0;
+      trace[3 * s + 1] = clock64();
+    }
+    unsigned char* B = base_of(b);
+    const EllRec R = ((const EllRec*)B)[0];
+    const int npad = R.npad;
+    const int* s_idx = (const int*)(B + 64);
+    const T* s_val = (const T*)(B + 64 + cap_idx);
+    const T* s_b = (const T*)(B + 64 + cap_idx + cap_val) + shift_of(bw, (int64_t)r0 + R.sa);
+    const int* s_lp = (const int*)(B + 64 + cap_idx + cap_val + cap_b) + shift_of(lp, R.l0);
+    // Software pipeline across levels: this thread's rows of level li+1
+    // (rows la + tid + q*NC, q < RPT) -- their b, slots and values, none of
+    // which depend on x -- are loaded before the barrier that ends level li,
+    // so after it only ld.shared x -> DFMA -> store remains on the dependency
+    // chain.  Branch-free: a row slot past the level end loads row 0 of the
+    // stage and is neutralised (slot = the zero slot, value 0, b 0); only the
+    // stores are predicated.
+    const int nrow = R.sb - R.sa;
+    int la = max(s_lp[0], R.sa) - R.sa, lb = min(s_lp[1], R.sb) - R.sa;  // stage-local
+    T pb[RPT], pv[RPT][K];
+    int ps[RPT][K];
+    auto prefetch = [&](int la_, int lb_) {
+#pragma unroll
+      for (int q = 0; q < RPT; ++q) {
+        const int i = la_ + tid + q * NC;
+        const bool ok = i < lb_;
+        const int ic = ok ? i : 0;
+        pb[q] = ok ? s_b[ic] : T(0);
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+          const int sl = s_idx[k * npad + ic];
+          const T v = s_val[k * npad + ic];
+          ps[q][k] = ok ? sl : XW;
+          pv[q][k] = ok ? v : T(0);
+        }
+      }
+    };
+    prefetch(la, lb);
+    T* const xs_stage = xs + r0 + R.sa;
+    const int sa_mask = R.sa;  // row r = sa + i; window slot (sa + i) & xmask
+    for (int li = 0; li + 1 < R.nl; ++li) {
+#pragma unroll
+      for (int q = 0; q < RPT; ++q) {  // operands already in registers
+        T acc = pb[q];
+#pragma unroll
+        for (int k = 0; k < K; ++k) acc -= pv[q][k] * xw[ps[q][k]];
+        const int i = la + tid + q * NC;
+        if (i < lb) {
+          xw[(sa_mask + i) & xmask] = acc;
+          xs_stage[i] = acc;
+        }
+      }
+      if (lb - la > RPT * NC) {  // warp-uniform: a level wider than NC * RPT rows
+        for (int i = la + tid + RPT * NC; i < lb; i += NC) {
+          T a2 = s_b[i];
+#pragma unroll
+          for (int k = 0; k < K; ++k) a2 -= s_val[k * npad + i] * xw[s_idx[k * npad + i]];
+          xw[(sa_mask + i) & xmask] = a2;
+          xs_stage[i] = a2;
+        }
+      }
+      if (li + 2 < R.nl) {
+        la = max(s_lp[li + 1] - R.sa, 0);
+        lb = min(s_lp[li + 2] - R.sa, nrow);
+        prefetch(la, lb);
+      }
+      asm volatile("bar.sync 1, %0;" ::"r"(NC) : "memory");  // level barrier (Alg 2 L96)
+    }
+    if (trace && tid == 0) trace[3 * s + 2] = clock64();
+    if (tid == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(&empty[b])) : "memory");
+    if (++b == NST) {
+      b = 0;
+      ph ^= 1u;
     }
   }
 }
