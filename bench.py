@@ -55,6 +55,8 @@ def parse():
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0, help="oracle baseline budget")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--dist", action="store_true",
+                    help="run the NCCL sharded multi-RHS path even at world size 1 (tests the code path)")
     return ap.parse_args()
 
 
@@ -140,8 +142,8 @@ def load_peaks():
 
 
 def load_traffic(kernel_impl: str):
-    """dram bytes per launch of the dominant kernel from the committed ncu
-    summary (profiles/ncu_summary.json), else None."""
+    """dram bytes per launch of the dominant kernel ("<config>:<impl>") from
+    the committed ncu summary (profiles/ncu_summary.json), else None."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
         d = json.load(open(p))
@@ -184,10 +186,10 @@ def run_reference(args):
     from workloads import generators as g
     from oracle import numeric as on
     nrhs = args.nrhs or DEFAULT_NRHS[args.config]
-    M, b = g.gen_config(args.config, nrhs=nrhs)
+    M = g.gen_matrix(args.config)
     threads = 1 if nrhs == 1 else min(nrhs, len(os.sched_getaffinity(0)))
     cols = nrhs if nrhs == 1 else min(nrhs, threads * 2)
-    bs = np.ascontiguousarray(b[:cols])
+    bs = g.gen_rhs_cols(M.n, 0, cols, seed=g.config_seed(args.config))  # a bounded sample of the columns
     for _ in range(args.warmup):
         on.solve_timed(M, bs, threads=threads)
     ts = []
@@ -199,11 +201,21 @@ def run_reference(args):
     line = {"metric": METRIC, "value": val, "unit": "GFLOPS", "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
-            "config": {"workload": WORKLOAD[args.config], "n": M.n, "nnz": M.nnz, "nrhs_timed": cols},
+            "config": {"workload": WORKLOAD[args.config], "n": M.n, "nnz": M.nnz, "nrhs": nrhs, "nrhs_timed": cols},
             "cpu_baseline": {"value": val, "unit": "GFLOPS", "cores": used, "kind": "oracle",
                              "sample": f"{args.steps} full solves x {cols} RHS column(s)"},
             "e2e": {"value": val, "unit": "GFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def load_tlvl():
+    """Measured per-level synchronisation latencies (scripts/microbench/t_lvl.cu,
+    summarised in profiles/t_lvl.json), or None."""
+    p = os.path.join(ROOT, "profiles", "t_lvl.json")
+    try:
+        return json.load(open(p))
+    except Exception:
+        return None
 
 
 def main():
@@ -215,20 +227,35 @@ def main():
     import torch.distributed as dist
 
     ws, rank, local = dist_env()
-    if ws > 1:
-        dist.init_process_group("nccl")
+    use_dist = ws > 1 or args.dist
+    if use_dist:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29517")
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local), rank=rank, world_size=ws)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
 
     import paper_conf_icpp_lun020_b200 as sp
+    from paper_conf_icpp_lun020_b200.dist import check_replicated, dist_solve, shard_bounds
     from workloads import generators as g
 
-    nrhs = args.nrhs or DEFAULT_NRHS[args.config]
+    cfg = args.config
+    nrhs_total = args.nrhs or DEFAULT_NRHS[cfg]
+    # C5 (multi-RHS) shards its RHS columns over the ranks (strong scaling);
+    # every other config runs one independent replica per rank (weak scaling,
+    # a single solve does not shard)
+    sharded = nrhs_total > 1 and use_dist
+    if sharded:
+        c0, c1 = shard_bounds(nrhs_total, ws, rank)
+    else:
+        c0, c1 = 0, nrhs_total
+    nrhs = c1 - c0
     tdt = torch.float64 if args.dtype == "f64" else torch.float32
+    npdt = np.float64 if args.dtype == "f64" else np.float32
     vb = 8 if args.dtype == "f64" else 4
-    M, b_np = g.gen_config(args.config, nrhs=nrhs)
-    if rank:
-        b_np = g.gen_rhs(M.n, nrhs, seed=g.SEED_BASE + int(args.config[1:]) + 1000 + rank)
+    M = g.gen_matrix(cfg)
+    seed = g.config_seed(cfg) if (sharded or rank == 0) else g.config_seed(cfg) + 7919 * rank
+    b_np = g.gen_rhs_cols(M.n, c0, c1, seed=seed)  # (nrhs, n): this rank's columns
     val = M.val if args.dtype == "f64" else M.val.astype(np.float32)
 
     # preprocess (analysis + upload): one warm-up, median of 3
@@ -244,6 +271,8 @@ def main():
     preprocess_ms = float(np.median(pre))
     info = plan.info()
     segs = plan.segments()
+    if use_dist:
+        check_replicated(plan)
 
     B = torch.from_numpy(b_np).to(dev, tdt).T  # (n, nrhs) column-major
     if nrhs == 1:
@@ -290,8 +319,9 @@ def main():
         t_max = t_local
     plan.set_profiling(False)
 
-    flops_step = 2.0 * M.nnz * nrhs
-    value = ws * flops_step * args.steps / t_max / 1e9
+    # whole-job work per step: all RHS columns (sharded) or one replica per rank
+    flops_job = 2.0 * M.nnz * (nrhs_total if sharded else nrhs * ws)
+    value = flops_job * args.steps / t_max / 1e9
     ms_per_step = t_max / args.steps * 1e3
 
     # ---------------- roofline of the dominant kernel
@@ -299,45 +329,86 @@ def main():
     seg_mean = seg_acc / args.steps  # [perm-in, seg..., perm-out]
     names = ["permute_in"] + [f"seg{i}:{s['impl']}" for i, s in enumerate(segs)] + ["permute_out"]
     dom = int(np.argmax(seg_mean))
+    dep = None
     if 1 <= dom <= len(segs):
         dseg = segs[dom - 1]
         dbytes = seg_alg_bytes(dseg, nrhs, vb)
         dimpl = dseg["impl"]
+        if dseg["kind"] == "TRI" and dseg["nlevels"] > 1:
+            ns_lvl = seg_mean[dom] * 1e6 / dseg["nlevels"]
+            dep = {"nlevels": dseg["nlevels"], "ns_per_level": ns_lvl}
+            tl = load_tlvl()
+            if tl:
+                dep["t_lvl_floor_ns"] = tl.get("smem_chain_bar_ns")
+                dep["t_lvl_source"] = "profiles/t_lvl.json (bar.sync + ld.shared/DFMA/st.shared chain, 1 SM)"
     else:
         dbytes = M.n * 4 + 2 * M.n * nrhs * vb
         dimpl = "PERMUTE"
     achieved = dbytes / (seg_mean[dom] / 1e3) / 1e9
-    tr = load_traffic(dimpl)
+    tr = load_traffic(f"{cfg}:{dimpl}")
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": tr, "kernel": names[dom], "share_of_step": float(seg_mean[dom] / seg_mean.sum()),
+                "alg_bytes_per_launch": dbytes,
                 "peak_source": f"{peak_kind} copy bandwidth (MEASURED_PEAKS.json hbm_gbs)"}
+    if dep:
+        roofline["dependency"] = dep
     whole_bytes = algorithmic_bytes(M.n, M.nnz, nrhs, vb)
-    whole = {"achieved_gbs": whole_bytes / (ms_per_step / 1e3) / 1e9, "frac": whole_bytes / (ms_per_step / 1e3) / 1e9 / peak,
-             "alg_bytes": whole_bytes}
+    whole = {"achieved_gbs": whole_bytes / (ms_per_step / 1e3) / 1e9,
+             "frac": whole_bytes / (ms_per_step / 1e3) / 1e9 / peak, "alg_bytes": whole_bytes}
 
-    # ---------------- end to end through the C ABI with host buffers
-    Bh = torch.from_numpy(b_np.astype(np.float64 if vb == 8 else np.float32)).pin_memory().T
-    if nrhs == 1:
-        Bh = Bh[:, 0].contiguous().pin_memory()
-    Xh = torch.empty_like(Bh).pin_memory() if nrhs == 1 else torch.empty(nrhs, M.n, dtype=tdt).pin_memory().T
-    for _ in range(2):
-        sp.sptrsv_solve(plan, Bh, Xh, stream=stream)
-    e2e_ms = []
-    for _ in range(max(3, min(args.steps, 20))):
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        sp.sptrsv_solve(plan, Bh, Xh, stream=stream)  # H2D + solve + D2H (+ sync)
-        e1.record(stream)
-        e1.synchronize()
-        e2e_ms.append(e0.elapsed_time(e1))
+    # ---------------- end to end through the public API with host buffers
+    e2e_iters = max(3, min(args.steps, 20 if nrhs_total == 1 else 3))
+    if sharded:
+        # root: pinned host B (all columns) -> H2D -> dist_solve (NCCL scatter,
+        # per-rank solve, NCCL gather) -> D2H; max over ranks
+        if rank == 0:
+            b_all = g.gen_rhs(M.n, nrhs_total, seed=g.config_seed(cfg), dtype=npdt)
+            Bh = torch.from_numpy(b_all).pin_memory()  # (k, n) row-major == (n, k) column-major
+            Xh = torch.empty_like(Bh).pin_memory()
+            del b_all
+        e2e_ms = []
+        for it in range(e2e_iters + 1):
+            dist.barrier()
+            torch.cuda.synchronize()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            Bd = Bh.to(dev, non_blocking=True).T if rank == 0 else None
+            Xd = dist_solve(plan, Bd, nrhs=None if rank == 0 else nrhs_total)
+            if rank == 0:
+                Xh.copy_(Xd.T, non_blocking=True)
+            e1.record(stream)
+            e1.synchronize()
+            if it:
+                e2e_ms.append(e0.elapsed_time(e1))
+            del Bd, Xd
+        h2d = d2h = M.n * nrhs_total * vb
+    else:
+        Bh = torch.from_numpy(b_np.astype(npdt)).pin_memory().T
+        if nrhs == 1:
+            Bh = Bh[:, 0].contiguous().pin_memory()
+        Xh = torch.empty_like(Bh).pin_memory() if nrhs == 1 else torch.empty(nrhs, M.n, dtype=tdt).pin_memory().T
+        for _ in range(2):
+            sp.sptrsv_solve(plan, Bh, Xh, stream=stream)
+        e2e_ms = []
+        for _ in range(e2e_iters):
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            sp.sptrsv_solve(plan, Bh, Xh, stream=stream)  # H2D + solve + D2H (+ sync)
+            e1.record(stream)
+            e1.synchronize()
+            e2e_ms.append(e0.elapsed_time(e1))
+        h2d = d2h = M.n * nrhs * vb
     e2e_t = float(np.mean(e2e_ms)) / 1e3
     if ws > 1:
         tt = torch.tensor([e2e_t], dtype=torch.float64, device=dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         e2e_t = float(tt.item())
-    e2e = {"value": ws * flops_step / e2e_t / 1e9, "unit": "GFLOPS", "h2d_bytes_per_step": M.n * nrhs * vb,
-           "d2h_bytes_per_step": M.n * nrhs * vb, "ms_per_step": e2e_t * 1e3}
+    e2e = {"value": flops_job / e2e_t / 1e9, "unit": "GFLOPS", "h2d_bytes_per_step": h2d,
+           "d2h_bytes_per_step": d2h, "ms_per_step": e2e_t * 1e3,
+           "path": "dist_solve (NCCL scatter/gather) from pinned host B on rank 0" if sharded
+           else "sptrsv_solve with pinned host b/x (H2D + solve + D2H inside the call)"}
 
     # ---------------- parity of the timed result (sampled for multi-RHS)
     parity = None
@@ -357,12 +428,15 @@ def main():
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": "GFLOPS", "n_gpus": ws, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "strong" if sharded or (nrhs_total > 1 and ws == 1) else "weak",
             "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
-            "config": {"workload": WORKLOAD[args.config], "n": M.n, "nnz": M.nnz, "nrhs": nrhs,
-                       "selector": args.selector, "variant": args.variant, "depth": info["depth"],
-                       "segments": len(segs), "l2": "flushed (256 MB write) between timed solves"
-                       if not args.no_flush else "not flushed", "parallelism": f"rhs-replicas x{ws}"},
+            "config": {"workload": WORKLOAD[cfg], "n": M.n, "nnz": M.nnz, "nrhs": nrhs_total,
+                       "nrhs_per_rank": nrhs, "selector": args.selector, "variant": args.variant,
+                       "depth": info["depth"], "segments": len(segs),
+                       "l2": "flushed (256 MB write) between timed solves" if not args.no_flush else "not flushed",
+                       "parallelism": (f"rhs-columns sharded x{ws} (NCCL scatter/gather only in e2e)" if sharded
+                                       else f"rhs-replicas x{ws}")},
             "preprocess_ms": preprocess_ms,
             "hbm_whole_solve": whole,
             "roofline": roofline,
@@ -374,7 +448,7 @@ def main():
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
-    if ws > 1:
+    if use_dist:
         dist.destroy_process_group()
 
 

@@ -194,6 +194,14 @@ sptrsv_status_t sptrsv_plan_seg_array(sptrsv_plan_t plan, int32_t seg, int32_t w
  * col_idx[nnz], val[nnz] (dtype of the plan).  Any pointer may be NULL. */
 sptrsv_status_t sptrsv_plan_matrix(sptrsv_plan_t plan, int64_t* row_ptr, int32_t* col_idx, void* val);
 
+/* 64-bit FNV-1a digest of everything a solve depends on: n, nnz, dtype,
+ * fill, depth, the permutation, every segment descriptor and every stored
+ * array (row pointers, columns, values, DCSR rows, level pointers) and the
+ * scaled diagonal.  The analysis is bit-deterministic, so replicated plans
+ * on different ranks must agree (all_reduce MIN == MAX).
+ * Host-only computation; works for host_only plans. */
+sptrsv_status_t sptrsv_plan_hash(sptrsv_plan_t plan, uint64_t* out);
+
 /* Per-segment timing of later solves with CUDA events (diagnostics/bench).
  * When on, sptrsv_solve records an event around every segment on its stream;
  * sptrsv_seg_times synchronises and returns milliseconds of the LAST solve:

@@ -135,6 +135,12 @@ class Plan:
                 "sptrsv_plan_matrix")
         return rp, ci, va
 
+    def hash(self) -> int:
+        """64-bit digest of the plan (identical on every rank for the same input)."""
+        h = ctypes.c_uint64(0)
+        C.check(C.lib().sptrsv_plan_hash(self._h, ctypes.byref(h)), "sptrsv_plan_hash")
+        return int(h.value)
+
     def set_profiling(self, on: bool = True) -> None:
         C.check(C.lib().sptrsv_set_profiling(self._h, 1 if on else 0), "sptrsv_set_profiling")
 

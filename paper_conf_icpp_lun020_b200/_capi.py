@@ -28,7 +28,7 @@ ARRAY_IN_DEGREE, ARRAY_LEVEL_PTR, ARRAY_DCSR_ROWS = 0, 1, 2
 
 EXPORTS = ["sptrsv_opts_default", "sptrsv_analyse", "sptrsv_solve", "sptrsv_free", "sptrsv_plan_info",
            "sptrsv_plan_segments", "sptrsv_plan_perm", "sptrsv_plan_levels", "sptrsv_plan_seg_array",
-           "sptrsv_plan_matrix", "sptrsv_set_profiling", "sptrsv_seg_times", "sptrsv_status_string",
+           "sptrsv_plan_matrix", "sptrsv_plan_hash", "sptrsv_set_profiling", "sptrsv_seg_times", "sptrsv_status_string",
            "sptrsv_last_error", "sptrsv_version"]
 
 
@@ -90,6 +90,8 @@ def lib() -> ctypes.CDLL:
     L.sptrsv_plan_seg_array.argtypes = [vp, i32, i32, vp, i64, ctypes.POINTER(i64)]
     L.sptrsv_plan_matrix.restype = ctypes.c_int
     L.sptrsv_plan_matrix.argtypes = [vp, vp, vp, vp]
+    L.sptrsv_plan_hash.restype = ctypes.c_int
+    L.sptrsv_plan_hash.argtypes = [vp, ctypes.POINTER(ctypes.c_uint64)]
     L.sptrsv_set_profiling.restype = ctypes.c_int
     L.sptrsv_set_profiling.argtypes = [vp, i32]
     L.sptrsv_seg_times.restype = ctypes.c_int

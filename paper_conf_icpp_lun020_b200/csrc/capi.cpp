@@ -255,6 +255,42 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_matrix(sptrsv_plan_t plan, int64_t* ro
   return SPTRSV_SUCCESS;
 }
 
+namespace {
+struct Fnv {
+  uint64_t h = 1469598103934665603ull;
+  void add(const void* p, size_t bytes) {
+    const unsigned char* c = (const unsigned char*)p;
+    for (size_t i = 0; i < bytes; ++i) h = (h ^ c[i]) * 1099511628211ull;
+  }
+  template <typename V>
+  void vec(const std::vector<V>& v) {
+    uint64_t s = v.size();
+    add(&s, 8);
+    if (!v.empty()) add(v.data(), v.size() * sizeof(V));
+  }
+};
+}  // namespace
+
+SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_hash(sptrsv_plan_t plan, uint64_t* out) {
+  if (!plan || !out) return fail(SPTRSV_ERROR_INVALID_VALUE, "NULL argument");
+  const Plan& p = plan->p;
+  Fnv f;
+  int64_t hdr[6] = {p.n, p.nnz, (int64_t)p.dtype, (int64_t)p.fill, p.depth, (int64_t)p.segs.size()};
+  f.add(hdr, sizeof(hdr));
+  f.vec(p.perm);
+  f.vec(p.rdiag_new);
+  for (const auto& S : p.segs) {
+    f.add(&S.info, sizeof(S.info));
+    f.vec(S.rp);
+    f.vec(S.ci);
+    f.vec(S.val);
+    f.vec(S.rows);
+    f.vec(S.level_ptr);
+  }
+  *out = f.h;
+  return SPTRSV_SUCCESS;
+}
+
 SPTRSV_EXPORT sptrsv_status_t sptrsv_set_profiling(sptrsv_plan_t plan, int32_t on) {
   if (!plan) return fail(SPTRSV_ERROR_INVALID_VALUE, "plan is NULL");
   plan->p.profiling = on != 0;

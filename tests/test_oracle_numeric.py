@@ -146,3 +146,12 @@ def test_rel_err_definition():
     ref = np.array([[1.0, -2.0, 4.0]])
     x = np.array([[1.0, -2.0, 4.0 + 4e-10]])
     assert abs(on.rel_err(x, ref) - 1e-10) < 1e-15
+
+
+def test_rhs_column_shards_match_full_draw():
+    """bench.py / dist ranks draw only their RHS columns (PCG64 jump-ahead);
+    they must be byte-identical to the corresponding columns of gen_rhs."""
+    from workloads import generators as g
+    full = g.gen_rhs(997, 9, seed=123)
+    for c0, c1 in [(0, 9), (0, 1), (3, 7), (8, 9)]:
+        assert np.array_equal(g.gen_rhs_cols(997, c0, c1, seed=123), full[c0:c1])

@@ -13,6 +13,9 @@ from .generators import (  # noqa: F401
     Matrix,
     gen_config,
     gen_rhs,
+    gen_rhs_cols,
+    gen_matrix,
+    config_seed,
     c1_random,
     c2_laplacian_ic0,
     c3_powerlaw_layers,

@@ -266,6 +266,21 @@ def gen_rhs(n: int, nrhs: int = 1, seed: int = SEED_BASE + 1000, dtype=np.float6
     return (2.0 * rng.random((nrhs, n)) - 1.0).astype(dtype)
 
 
+def gen_rhs_cols(n: int, c0: int, c1: int, seed: int = SEED_BASE + 1000, dtype=np.float64) -> np.ndarray:
+    """Columns [c0, c1) of gen_rhs(n, nrhs, seed) without drawing the others
+    (PCG64 jump-ahead; one 64-bit draw per double), numpy shape (c1-c0, n).
+    Lets every rank of a sharded SpTRSM create only its own shard."""
+    bg = np.random.PCG64(seed)
+    bg.advance(int(c0) * int(n))
+    rng = np.random.Generator(bg)
+    return (2.0 * rng.random((c1 - c0, n)) - 1.0).astype(dtype)
+
+
+def config_seed(name: str) -> int:
+    """Seed of a config's right-hand sides (gen_config)."""
+    return SEED_BASE + int(name[1:]) + 1000
+
+
 # name -> (builder, default nrhs); full BASELINE.json sizes
 CONFIGS = {
     "C1": (lambda: c1_random(), 1),
@@ -294,8 +309,14 @@ def gen_config(name: str, small: bool = False, nrhs: int | None = None, dtype=np
     if dtype != np.float64:
         L = L.astype(dtype)
     nr = default_nrhs if nrhs is None else nrhs
-    b = gen_rhs(L.n, nr, seed=SEED_BASE + k + 1000, dtype=dtype)
+    b = gen_rhs(L.n, nr, seed=config_seed(name), dtype=dtype)
     return L, b
+
+
+def gen_matrix(name: str, small: bool = False, dtype=np.float64) -> Matrix:
+    """The matrix of a config only (no right-hand side)."""
+    L = (SMALL if small else CONFIGS)[name][0]()
+    return L.astype(dtype) if dtype != np.float64 else L
 
 
 # ---------------------------------------------------------------------------
