@@ -79,7 +79,12 @@ typedef enum {
   SPTRSV_IMPL_TRI_SYNCFREE = 2,  /* K3: persistent multi-CTA, ticketed rows, per-row ready flags    */
   SPTRSV_IMPL_TRI_CHAIN = 3,     /* K4: single CTA, level loop with bar.sync, x window in smem      */
   SPTRSV_IMPL_SQ_SCALAR = 4,     /* K5/K7: thread (or RHS-group) per row, CSR or DCSR               */
-  SPTRSV_IMPL_SQ_VECTOR = 5      /* K6/K8: warp per row, CSR or DCSR                                */
+  SPTRSV_IMPL_SQ_VECTOR = 5,     /* K6/K8: warp per row, CSR or DCSR                                */
+  SPTRSV_IMPL_TRI_SUPERNODE = 6, /* B200: warp per fundamental supernode (<= 32 rows): dense GEMV of its
+                                    shared external columns + register-resident dense triangle     */
+  SPTRSV_IMPL_TRI_PIPE = 7       /* B200: narrow-level triangle split by original row index over P CTAs
+                                    (a pipeline); shared-memory spin flags inside a CTA, no per-level
+                                    barrier; cross-CTA dependencies polled in L2                     */
 } sptrsv_impl_t;
 
 /* Which kernel implements each Alg 7 label. PAPER maps labels 1:1 onto the
@@ -91,7 +96,9 @@ typedef struct {
   int32_t variant;          /* sptrsv_variant_t, default REC                                   */
   int32_t depth;            /* -1 = the paper's rule (L299); >= 0 forces a uniform depth       */
   int64_t min_block_rows;   /* depth-rule threshold; 0 = 20 * SMs * 128 (378,880 on 148 SMs)   */
-  int32_t reorder;          /* 0 = level-set reordering of every triangle (L231), 1 = none     */
+  int32_t reorder;          /* 0 = level-set reordering of every triangle (L231), 1 = none,
+                               2 = auto (default): none when the input is supernodal (mean width of
+                               its fundamental supernodes >= 8, R29), else level        */
   int32_t selector;         /* sptrsv_selector_t, default SPTRSV_SELECT_B200                   */
   int32_t force_tri_impl;   /* -1 = auto; else an sptrsv_impl_t for every triangle (tests)     */
   int32_t force_sq_impl;    /* -1 = auto; else an sptrsv_impl_t for every square (tests)       */
@@ -153,7 +160,7 @@ sptrsv_status_t sptrsv_free(sptrsv_plan_t plan);
 /* ---------------------------------------------------------------- introspection
  * Used for the bit-exact structural parity against the oracle and for reporting. */
 typedef struct {
-  int32_t n, depth, nseg, variant, dtype, fill, reorder, selector;
+  int32_t n, depth, nseg, variant, dtype, fill, reorder /* effective: 0 level, 1 none */, selector;
   int64_t nnz;
   int64_t min_block_rows;
   int32_t sm_count;

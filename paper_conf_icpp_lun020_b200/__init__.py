@@ -172,11 +172,15 @@ class Plan:
 
 
 def sptrsv_analyse(row_ptr, col_idx, val, n: int | None = None, fill: str = "L", variant: str = "REC",
-                   depth: int = -1, min_block_rows: int = 0, reorder: bool = True, selector: str = "B200",
+                   depth: int = -1, min_block_rows: int = 0, reorder="auto", selector: str = "B200",
                    force_tri_impl: str | None = None, force_sq_impl: str | None = None,
                    host_only: bool = False, sm_count: int = 0, threads: int = 0, stream=None,
                    device: int | None = None) -> Plan:
-    """Preprocess a CSR lower (fill='L') or upper (fill='U') triangular matrix."""
+    """Preprocess a CSR lower (fill='L') or upper (fill='U') triangular matrix.
+
+    reorder: True = level-set reordering of every triangle (the paper, L231),
+    False = none, "auto" = none for supernodal inputs, else level (R29).
+    """
     rp = _as_int32(row_ptr)
     ci = _as_int32(col_idx)
     n = (len(rp) - 1) if n is None else n
@@ -191,7 +195,7 @@ def sptrsv_analyse(row_ptr, col_idx, val, n: int | None = None, fill: str = "L",
     o.variant = C.VARIANTS[variant]
     o.depth = depth
     o.min_block_rows = min_block_rows
-    o.reorder = 0 if reorder else 1
+    o.reorder = 2 if reorder == "auto" else (0 if reorder else 1)
     o.selector = C.SELECTORS[selector]
     o.force_tri_impl = -1 if force_tri_impl is None else C.IMPLS.index(force_tri_impl)
     o.force_sq_impl = -1 if force_sq_impl is None else C.IMPLS.index(force_sq_impl)

@@ -123,6 +123,34 @@ int32_t clamp_depth(int64_t n, int32_t d) {
   return std::min(d, lg);
 }
 
+// Fundamental supernodes, cut into pieces of <= kSnMax rows: row r joins the
+// piece of row r-1 iff its off-diagonal columns are exactly those of row
+// r-1 plus r-1 itself (so the piece's diagonal block is dense and its rows
+// share one list of external columns).  Returns the number of pieces.
+constexpr int32_t kSnMax = 32;
+
+int64_t supernode_pieces(int32_t n, const std::vector<int64_t>& rp, const std::vector<int32_t>& ci,
+                         std::vector<int32_t>* starts) {
+  int64_t np = 0;
+  int32_t start = 0;
+  for (int32_t r = 0; r < n; ++r) {
+    bool join = false;
+    if (r > start && r - start < kSnMax) {
+      const int64_t a0 = rp[r - 1], l0 = rp[r] - 1 - a0;  // off-diagonals of r-1
+      const int64_t a1 = rp[r], l1 = rp[r + 1] - 1 - a1;  // off-diagonals of r
+      join = l1 == l0 + 1 && ci[a1 + l1 - 1] == r - 1 &&
+             std::equal(ci.begin() + a0, ci.begin() + a0 + l0, ci.begin() + a1);
+    }
+    if (!join) {
+      start = r;
+      ++np;
+      if (starts) starts->push_back(r);
+    }
+  }
+  if (starts) starts->push_back(n);
+  return np;
+}
+
 struct Reorderer {
   const LowerCSR& L;
   bool reorder;
@@ -212,7 +240,15 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
   // ---- recursive reordering: every node, root and leaves (reading R3) ----
   // Siblings are independent once their parent is reordered (each only reads
   // dependencies inside its own range), so one depth level runs in parallel.
-  Reorderer R(L, p.opts.reorder == 0);
+  // reorder AUTO (reading R29): a supernodal input keeps its order, because
+  // level sorting scatters the rows of every dense diagonal block over as
+  // many levels as the block is wide (SURVEY.md 7.3 hard part 5)
+  p.reorder_eff = p.opts.reorder == 1 ? 1 : 0;
+  if (p.opts.reorder == 2 && n > 0) {
+    const int64_t np = supernode_pieces(n, L.rp, L.ci, nullptr);
+    p.reorder_eff = (np > 0 && (double)n / (double)np >= 8.0) ? 1 : 0;
+  }
+  Reorderer R(L, p.reorder_eff == 0);
   std::vector<int32_t> leaf_nl;
   std::vector<std::pair<int32_t, int32_t>> nodes = {{0, n}};
   for (int32_t d = 0; d <= p.depth && n > 0; ++d) {
@@ -280,6 +316,7 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
   p.perm.resize(n);
   for (int32_t k = 0; k < n; ++k) p.perm[k] = p.fill == SPTRSV_LOWER ? R.perm[k] : n - 1 - R.perm[k];
   p.leaf_level = R.leaf_level;
+  p.lower_old = R.perm;
 
   // ---- segment geometry in execution order ----
   struct Geo { int32_t kind, r0, r1, c0, c1, leaf; };
@@ -359,6 +396,24 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
       }
       I.max_level_rows = mx;
       S.nzr = m;
+      {  // fundamental-supernode pieces of the triangle (its own entries only)
+        S.sn_ptr.clear();
+        int32_t start = 0;
+        for (int32_t k = 0; k < m; ++k) {
+          bool join = false;
+          if (k > start && k - start < kSnMax) {
+            const int64_t a0 = lo_idx[k - 1], l0 = hi_idx[k - 1] - a0;
+            const int64_t a1 = lo_idx[k], l1 = hi_idx[k] - a1;
+            join = l1 == l0 + 1 && p.p_ci[a1 + l1 - 1] == g.r0 + k - 1 &&
+                   std::equal(p.p_ci.begin() + a0, p.p_ci.begin() + a0 + l0, p.p_ci.begin() + a1);
+          }
+          if (!join) {
+            start = k;
+            S.sn_ptr.push_back(k);
+          }
+        }
+        S.sn_ptr.push_back(m);
+      }
     } else {
       I.nnz = tot;
       I.nnz_per_row = m ? (int32_t)(tot / m) : 0;
@@ -442,12 +497,24 @@ void choose_impls(Plan& p) {
         case SPTRSV_K_NEAR_SERIAL: impl = SPTRSV_IMPL_TRI_CHAIN; break;
         default: impl = SPTRSV_IMPL_TRI_SYNCFREE; break;
       }
-      if (p.opts.selector == SPTRSV_SELECT_B200 && I.nlevels > 1) {
+      const int64_t npieces = (int64_t)S.sn_ptr.size() - 1;
+      const bool supernodal = npieces > 0 && (double)(I.row1 - I.row0) / (double)npieces >= 8.0;
+      if (p.opts.selector == SPTRSV_SELECT_B200 && I.nlevels > 1 && supernodal) {
+        impl = SPTRSV_IMPL_TRI_SUPERNODE;
+      } else if (p.opts.selector == SPTRSV_SELECT_B200 && I.nlevels > 1) {
         int64_t m = I.row1 - I.row0;
         // narrow levels: one CTA walks the level chain with bar.sync (no
         // cross-SM flag round trips); wide levels: all SMs
-        if (I.max_level_rows <= 2048 || (m / std::max(1, I.nlevels)) <= 256)
-          impl = SPTRSV_IMPL_TRI_CHAIN;
+        if (I.max_level_rows <= 2048 || (m / std::max(1, I.nlevels)) <= 256) {
+          // narrow levels: one SM per partition walks the level chain at
+          // shared-memory latency (pipeline of P CTAs for big triangles with
+          // <= 4 dependencies per row, one CTA otherwise)
+          int32_t kmax = 0;
+          for (int64_t r = 0; r < m; ++r) kmax = std::max(kmax, S.in_degree[r]);
+          impl = (kmax >= 1 && kmax <= 4 && m >= 4096 && std::getenv("SPTRSV_NO_PIPE") == nullptr)
+                     ? SPTRSV_IMPL_TRI_PIPE
+                     : SPTRSV_IMPL_TRI_CHAIN;
+        }
         else if (I.nlevels <= 20)
           impl = SPTRSV_IMPL_TRI_LEVELSET;
         else
@@ -455,6 +522,14 @@ void choose_impls(Plan& p) {
       }
       if (p.opts.force_tri_impl >= SPTRSV_IMPL_TRI_LEVELSET && p.opts.force_tri_impl <= SPTRSV_IMPL_TRI_CHAIN)
         impl = p.opts.force_tri_impl;
+      if (p.opts.force_tri_impl == SPTRSV_IMPL_TRI_SUPERNODE && I.nlevels > 1) impl = SPTRSV_IMPL_TRI_SUPERNODE;
+      if (p.opts.force_tri_impl == SPTRSV_IMPL_TRI_PIPE && I.nlevels > 1) impl = SPTRSV_IMPL_TRI_PIPE;
+      // the level-set and chain kernels walk levels as contiguous row ranges,
+      // which only the level-set reordering guarantees; without it a triangle
+      // runs sync-free (or supernodal), whatever its Alg 7 label
+      if (p.reorder_eff == 1 &&
+          (impl == SPTRSV_IMPL_TRI_LEVELSET || impl == SPTRSV_IMPL_TRI_CHAIN || impl == SPTRSV_IMPL_TRI_PIPE))
+        impl = supernodal ? SPTRSV_IMPL_TRI_SUPERNODE : SPTRSV_IMPL_TRI_SYNCFREE;
       if (p.opts.force_tri_impl == SPTRSV_IMPL_TRI_DIAG && I.nlevels <= 1) impl = SPTRSV_IMPL_TRI_DIAG;
       I.impl = impl;
     } else {

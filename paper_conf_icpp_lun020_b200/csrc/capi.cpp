@@ -40,7 +40,7 @@ SPTRSV_EXPORT void sptrsv_opts_default(sptrsv_opts_t* o) {
   o->variant = SPTRSV_VARIANT_REC;
   o->depth = -1;
   o->min_block_rows = 0;
-  o->reorder = 0;
+  o->reorder = 2;
   o->selector = SPTRSV_SELECT_B200;
   o->force_tri_impl = -1;
   o->force_sq_impl = -1;
@@ -87,7 +87,7 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_analyse(int32_t n, int64_t nnz, const int32
   else
     sptrsv_opts_default(&o);
   if (o.variant < 0 || o.variant > 2) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad variant");
-  if (o.reorder < 0 || o.reorder > 1) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad reorder");
+  if (o.reorder < 0 || o.reorder > 2) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad reorder");
   if (o.selector < 0 || o.selector > 1) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad selector");
   if (o.min_block_rows < 0) return fail(SPTRSV_ERROR_INVALID_VALUE, "min_block_rows < 0");
 
@@ -185,7 +185,7 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_info(sptrsv_plan_t plan, sptrsv_plan_i
   out->variant = p.opts.variant;
   out->dtype = p.dtype;
   out->fill = p.fill;
-  out->reorder = p.opts.reorder;
+  out->reorder = p.reorder_eff;
   out->selector = p.opts.selector;
   out->nnz = p.nnz;
   out->min_block_rows = p.min_block_rows;

@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <numeric>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -24,20 +25,51 @@ namespace {
 
 size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 
+// SpMM lane geometry for nrhs > 1: G lanes per row, RPT columns per lane per
+// pass (capped by SPTRSV_SPMM="RPTMAX,UN" for tuning; default 8,2), UN row entries per
+// gather round.  `multi_sync` is the sync-free triangle, which always uses
+// UN = 1 (its polling is per entry).
+SpmmCfg spmm_cfg() {
+  SpmmCfg c;
+  if (const char* e = std::getenv("SPTRSV_SPMM")) {
+    int a, b;
+    if (std::sscanf(e, "%d,%d", &a, &b) == 2 && (a == 1 || a == 2 || a == 4 || a == 8 || a == 16) && (b == 1 || b == 2)) {
+      c.rpt_max = a;
+      c.un = b;
+    }
+  }
+  return c;
+}
+
 template <typename F>
-void dispatch_multi(int nrhs, F&& f) {
+void dispatch_rpt(int nrhs, int rpt_max, F&& f) {
   if (nrhs <= 8)
     f(std::integral_constant<int, 8>(), std::integral_constant<int, 1>());
-  else if (nrhs <= 32)
+  else if (nrhs <= 32 || rpt_max == 1)
     f(std::integral_constant<int, 32>(), std::integral_constant<int, 1>());
-  else if (nrhs <= 64)
+  else if (nrhs <= 64 || rpt_max == 2)
     f(std::integral_constant<int, 32>(), std::integral_constant<int, 2>());
-  else if (nrhs <= 128)
+  else if (nrhs <= 128 || rpt_max == 4)
     f(std::integral_constant<int, 32>(), std::integral_constant<int, 4>());
-  else if (nrhs <= 256)
+  else if (nrhs <= 256 || rpt_max == 8)
     f(std::integral_constant<int, 32>(), std::integral_constant<int, 8>());
   else
     f(std::integral_constant<int, 32>(), std::integral_constant<int, 16>());
+}
+
+template <typename F>
+void dispatch_multi(int nrhs, F&& f) {
+  dispatch_rpt(nrhs, 16, f);
+}
+
+template <typename F>
+void dispatch_multi_un(int nrhs, const SpmmCfg& c, F&& f) {
+  dispatch_rpt(nrhs, c.rpt_max, [&](auto G, auto R) {
+    if (c.un == 2)
+      f(G, R, std::integral_constant<int, 2>());
+    else
+      f(G, R, std::integral_constant<int, 1>());
+  });
 }
 
 inline unsigned cdiv(int64_t a, int64_t b) { return (unsigned)((a + b - 1) / b); }
@@ -125,8 +157,35 @@ void build_chain_stages(Segment& S, const k::ChainGeom& g) {
 }
 
 // ELL-staged chain (see k::tri_chain_ell): eligible when every row has <= 4
-// dependencies, all inside the x window of their level.  Geometry: RMAX rows
-// per stage, as many stages as fit in 227 KB next to the window.
+// dependencies, all inside the x window of their level.  The triangle is cut
+// into steps (levels; a level wider than NW*RG*32 rows is cut into chunks)
+// of 32-row groups, steps into stages (<= RMAX rows, <= PMAX padded rows,
+// <= SMAX steps, never wrapping the window) that fit NST buffers next to the
+// window in 227 KB.
+struct EllGeom {
+  int XW, NST, RMAX, PMAX, SMAX;
+};
+
+EllGeom ell_geometry(int K, size_t vb) {
+  EllGeom g{4096, 3, 1024, 1536, 128};
+  if (const char* e = std::getenv("SPTRSV_ELL_GEOM")) {
+    int a, b, c;
+    if (std::sscanf(e, "%d,%d,%d", &a, &b, &c) == 3 && a >= 64 && b >= 2 && (b & (b - 1)) == 0 && c >= 2) {
+      g.RMAX = a; g.XW = b; g.NST = c;
+    }
+  }
+  // shrink the stage until NST buffers + window fit (and NST stages fit the window)
+  for (;;) {
+    g.PMAX = g.RMAX + g.RMAX / 2;
+    const uint32_t sb = vb == 8 ? k::ell_stage_bytes<double>(K, g.RMAX, g.PMAX, g.SMAX)
+                                : k::ell_stage_bytes<float>(K, g.RMAX, g.PMAX, g.SMAX);
+    const size_t tot = (size_t)g.NST * sb + k::al16((g.XW + 2) * (uint32_t)vb) + 16 * g.NST;
+    if ((tot <= 232448 && (size_t)(g.NST + 1) * g.RMAX <= (size_t)g.XW) || g.RMAX <= 128) break;
+    g.RMAX -= 128;
+  }
+  return g;
+}
+
 void build_chain_ell(Segment& S, size_t vb) {
   S.ell_K = 0;
   S.ell_recs.clear();
@@ -139,13 +198,8 @@ void build_chain_ell(Segment& S, size_t vb) {
   int K = 0;
   for (int r = 0; r < m; ++r) K = std::max(K, S.rp[r + 1] - S.rp[r]);
   if (K < 1 || K > 4) return;
-  int RMAX = 2048, XW = 4096, NSTMAX = 4;
-  if (const char* e = std::getenv("SPTRSV_ELL_GEOM")) {
-    int a, b, c;
-    if (std::sscanf(e, "%d,%d,%d", &a, &b, &c) == 3 && a >= 1 && b >= 2 && (b & (b - 1)) == 0 && c >= 2) {
-      RMAX = a; XW = b; NSTMAX = c;
-    }
-  }
+  const EllGeom G = ell_geometry(K, vb);
+  const int XW = G.XW;
   // every dependency of a row in level l must satisfy j >= end(l) - XW
   for (int l = 0; l < I.nlevels; ++l) {
     const int L1 = S.level_ptr[l + 1];
@@ -153,94 +207,130 @@ void build_chain_ell(Segment& S, size_t vb) {
       for (int q = S.rp[r]; q < S.rp[r + 1]; ++q)
         if (S.ci[q] - I.row0 < L1 - XW) return;
   }
-  const uint32_t sb_bytes = vb == 8 ? k::ell_stage_bytes<double>(K, RMAX) : k::ell_stage_bytes<float>(K, RMAX);
-  const uint32_t fixed = k::al16((XW + 2) * (uint32_t)vb) + 256;
-  const int NST = std::min<int>(NSTMAX, (int)((232448 - fixed) / (sb_bytes + 16)));
-  if (NST < 2) return;
-  // stage boundaries: whole levels where possible (<= RMAX rows, <= 256 levels)
-  std::vector<int32_t> st = {0};
-  int cur_r = 0, cur_l = 0;
-  for (int l = 0; l < I.nlevels; ++l) {
-    const int la = S.level_ptr[l], lb = S.level_ptr[l + 1], lr = lb - la;
-    if (cur_r + lr <= RMAX && cur_l + 1 <= 256) {
-      cur_r += lr;
-      cur_l += 1;
-      continue;
-    }
-    if (la > st.back()) st.push_back(la);
-    cur_r = cur_l = 0;
-    if (lr <= RMAX) {
-      cur_r = lr;
-      cur_l = 1;
-      continue;
-    }
-    for (int r = la + RMAX; r < lb; r += RMAX) st.push_back(r);  // split a wide level
-    cur_r = lb - st.back();
-    cur_l = 1;
-  }
-  if (m > st.back()) st.push_back(m);
-  const int ns = (int)st.size() - 1;
-  S.ell_recs.assign((size_t)ns * 16, 0);
-  size_t off = 0;
-  std::vector<size_t> offs(ns);
-  for (int q = 0; q < ns; ++q) {
-    const int n = st[q + 1] - st[q], npad = (n + 3) & ~3;
-    offs[q] = off;
-    off += k::al16(K * npad * 4) + k::al16(K * npad * (uint32_t)vb);
-  }
-  S.ell_data.assign(off, 0);
-  int l = 0;
-  for (int q = 0; q < ns; ++q) {
-    const int sa = st[q], sb = st[q + 1], n = sb - sa, npad = (n + 3) & ~3;
-    while (S.level_ptr[l + 1] <= sa) ++l;
-    int l_last = l;
-    while (S.level_ptr[l_last + 1] < sb) ++l_last;
-    int32_t* R = &S.ell_recs[(size_t)q * 16];
-    R[0] = sa; R[1] = sb; R[2] = l; R[3] = l_last - l + 2; R[4] = (int32_t)(offs[q] / 16); R[5] = npad;
-    int32_t* slots = (int32_t*)&S.ell_data[offs[q]];
-    char* vals = &S.ell_data[offs[q] + k::al16(K * npad * 4)];
-    for (int kk = 0; kk < K; ++kk)
-      for (int i = 0; i < npad; ++i) slots[kk * npad + i] = XW;  // the zero slot
-    for (int i = 0; i < n; ++i) {
-      const int r = sa + i;
-      int kk = 0;
-      for (int qq = S.rp[r]; qq < S.rp[r + 1]; ++qq, ++kk) {
-        slots[kk * npad + i] = (S.ci[qq] - I.row0) & (XW - 1);
-        std::memcpy(vals + ((size_t)kk * npad + i) * vb, &S.val[(size_t)qq * vb], vb);
-      }
-    }
-  }
-  for (int q = 0; q + NST < ns; ++q)
-    std::memcpy(&S.ell_recs[(size_t)q * 16 + 8], &S.ell_recs[(size_t)(q + NST) * 16], 32);
-  // consumer warps: cover the 90th-percentile level width with 2 rows/thread
+  // consumer warps: cover the 90th-percentile level width with RG = 2 groups each
   std::vector<int> widths(I.nlevels);
   for (int q = 0; q < I.nlevels; ++q) widths[q] = S.level_ptr[q + 1] - S.level_ptr[q];
   std::nth_element(widths.begin(), widths.begin() + (I.nlevels * 9) / 10, widths.end());
-  int w90 = widths[(I.nlevels * 9) / 10];
-  // measured on B200 (C2): per-level cost is issue-bound and grows ~13
-  // cycles per extra warp, so 8..12 warps x 2 rows beat 31 warps x 1 row
-  int warps = std::max(4, std::min(12, (w90 + 2 * 32 - 1) / (2 * 32)));
+  const int w90 = widths[(I.nlevels * 9) / 10];
+  const int RG = 2;
+  int warps = std::max(4, std::min(16, (w90 + RG * 32 - 1) / (RG * 32)));
   if (const char* e = std::getenv("SPTRSV_ELL_WARPS")) warps = std::atoi(e);
-  S.ell_warps = std::max(1, std::min(31, warps));
+  warps = std::max(1, std::min(31, warps));
+  const int cap = warps * RG * 32;  // rows per step
+  // steps: {row_start, nrows} (triangle-local rows)
+  // (a level is also cut where its rows cross a multiple of XW in global row
+  // numbering, so no step wraps the window; running the two chunks of a
+  // level one after the other is valid: rows of a level are independent)
+  std::vector<std::pair<int, int>> steps;
+  for (int l = 0; l < I.nlevels; ++l) {
+    const int lb = S.level_ptr[l + 1];
+    for (int a = S.level_ptr[l]; a < lb;) {
+      const int to_wrap = XW - (int)(((uint32_t)(I.row0 + a)) & ((uint32_t)XW - 1));
+      const int nr = std::min({cap, lb - a, to_wrap});
+      steps.push_back({a, nr});
+      a += nr;
+    }
+  }
+  // stages
+  struct St { int s0, s1, sa, sb, npad; };
+  std::vector<St> stages;
+  const uint32_t mask = (uint32_t)XW - 1;
+  {
+    St cur{0, 0, 0, 0, 0};
+    for (int q = 0; q < (int)steps.size(); ++q) {
+      const int ra = steps[q].first, nr = steps[q].second;
+      const int padded = (nr + 31) / 32 * 32;
+      // a stage never wraps the window: rows [sa, sb) must have contiguous slots
+      const uint32_t slot0 = ((uint32_t)(I.row0 + cur.sa)) & mask;
+      const bool fits = cur.s1 > cur.s0 && (ra + nr - cur.sa) <= G.RMAX && cur.npad + padded <= G.PMAX &&
+                        cur.s1 - cur.s0 < G.SMAX && slot0 + (uint32_t)(ra + nr - cur.sa) <= (uint32_t)XW;
+      if (cur.s1 > cur.s0 && !fits) {
+        stages.push_back(cur);
+        cur = St{q, q, ra, ra, 0};
+      }
+      if (cur.s1 == cur.s0) cur = St{q, q, ra, ra, 0};
+      // a single step that wraps the window on its own: split it at the wrap
+      cur.s1 = q + 1;
+      cur.sb = ra + nr;
+      cur.npad += padded;
+    }
+    if (cur.s1 > cur.s0) stages.push_back(cur);
+  }
+  // a step whose rows wrap the window inside one stage would break the bulk
+  // store; steps are <= cap rows and stages start fresh at wraps, so check
+  for (auto& st : stages) {
+    const uint32_t slot0 = ((uint32_t)(I.row0 + st.sa)) & mask;
+    if (slot0 + (uint32_t)(st.sb - st.sa) > (uint32_t)XW || st.sb - st.sa > G.RMAX || st.npad > G.PMAX ||
+        st.s1 - st.s0 > G.SMAX)
+      return;  // geometry cannot hold this triangle: fall back to the CSR chain
+  }
+  const int W = (K + 1) / 2;
+  const int ns = (int)stages.size();
+  S.ell_recs.assign((size_t)ns * 16, 0);
+  std::vector<size_t> offs(ns);
+  size_t off = 0;
+  for (int q = 0; q < ns; ++q) {
+    const int npad = stages[q].npad;
+    const size_t bytes = 16 * (size_t)(stages[q].s1 - stages[q].s0) + k::al16(W * npad * 4) + k::al16(K * npad * (uint32_t)vb);
+    offs[q] = off;
+    off += k::al16((uint32_t)bytes);
+  }
+  S.ell_data.assign(off, 0);
+  for (int q = 0; q < ns; ++q) {
+    const St& st = stages[q];
+    const int nst = st.s1 - st.s0, npad = st.npad;
+    char* blk = &S.ell_data[offs[q]];
+    int32_t* srec = (int32_t*)blk;
+    uint32_t* words = (uint32_t*)(blk + 16 * nst);
+    char* vals = blk + 16 * nst + k::al16(W * npad * 4);
+    const uint32_t zero = (uint32_t)XW;
+    for (int w = 0; w < W; ++w)
+      for (int i = 0; i < npad; ++i) words[w * npad + i] = zero | (zero << 16);
+    int grp = 0;
+    for (int t = st.s0; t < st.s1; ++t) {
+      const int ra = steps[t].first, nr = steps[t].second, ng = (nr + 31) / 32;
+      int32_t* R4 = srec + 4 * (t - st.s0);
+      R4[0] = grp; R4[1] = ng; R4[2] = ra - st.sa; R4[3] = nr;
+      for (int i = 0; i < nr; ++i) {
+        const int r = ra + i, pi = grp * 32 + i;
+        int kk = 0;
+        for (int qq = S.rp[r]; qq < S.rp[r + 1]; ++qq, ++kk) {
+          const uint32_t sl = ((uint32_t)S.ci[qq]) & mask;  // global permuted row -> window slot
+          uint32_t& wd = words[(kk >> 1) * npad + pi];
+          wd = (kk & 1) ? ((wd & 0xffffu) | (sl << 16)) : ((wd & 0xffff0000u) | sl);
+          std::memcpy(vals + ((size_t)kk * npad + pi) * vb, &S.val[(size_t)qq * vb], vb);
+        }
+      }
+      grp += ng;
+    }
+    int32_t* R = &S.ell_recs[(size_t)q * 16];
+    const size_t bytes = 16 * (size_t)nst + k::al16(W * npad * 4) + k::al16(K * npad * (uint32_t)vb);
+    R[0] = st.sa; R[1] = st.sb; R[2] = nst; R[3] = (int32_t)(offs[q] / 16); R[4] = (int32_t)k::al16((uint32_t)bytes);
+    R[5] = npad;
+  }
+  for (int q = 0; q + G.NST < ns; ++q)
+    std::memcpy(&S.ell_recs[(size_t)q * 16 + 8], &S.ell_recs[(size_t)(q + G.NST) * 16], 32);
+  S.ell_warps = warps;
   S.ell_K = K;
-  S.ell_NST = NST;
-  S.ell_RMAX = RMAX;
+  S.ell_NST = G.NST;
+  S.ell_RMAX = G.RMAX;
+  S.ell_PMAX = G.PMAX;
+  S.ell_SMAX = G.SMAX;
   S.ell_XW = XW;
 }
 
 template <typename T, int K>
 Error launch_chain_ell(Plan& p, Segment& S, const T* bw, T* xs, cudaStream_t s) {
-  const int NST = S.ell_NST, RMAX = S.ell_RMAX, XW = S.ell_XW;
-  const uint32_t smem = NST * k::ell_stage_bytes<T>(K, RMAX) + k::al16((XW + 2) * (uint32_t)sizeof(T)) + NST * 16;
-  constexpr int RPT = 2;
+  const int NST = S.ell_NST, RMAX = S.ell_RMAX, PMAX = S.ell_PMAX, SMAX = S.ell_SMAX, XW = S.ell_XW;
+  const uint32_t smem = NST * k::ell_stage_bytes<T>(K, RMAX, PMAX, SMAX) + k::al16((XW + 2) * (uint32_t)sizeof(T)) +
+                        NST * 16;
+  constexpr int RG = 2;
   static uint32_t attr_bytes = 0;  // per template instance
   if (smem > attr_bytes) {
-    CUDA_TRY(cudaFuncSetAttribute(k::tri_chain_ell<T, K, RPT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    CUDA_TRY(cudaFuncSetAttribute(k::tri_chain_ell<T, K, RG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                   (int)smem));
     attr_bytes = smem;
   }
-  // consumer warps: enough that NC * RPT covers a typical level, at most 31
-  int nc_warps = S.ell_warps;
   const int nst = (int)(S.ell_recs.size() / 16);
   long long* tr = nullptr;
   if (p.trace) {
@@ -248,8 +338,186 @@ Error launch_chain_ell(Plan& p, Segment& S, const T* bw, T* xs, cudaStream_t s) 
     if (!S.d_trace) CUDA_TRY(cudaMalloc(&S.d_trace, (size_t)nst * 3 * 8));
     tr = (long long*)S.d_trace;
   }
-  k::tri_chain_ell<T, K, RPT><<<1, 32 * (nc_warps + 1), smem, s>>>(
-      S.info.row0, nst, (const k::EllRec*)S.d_ell_recs, S.d_level_ptr, S.d_ell_data, bw, xs, NST, RMAX, XW, tr);
+  k::tri_chain_ell<T, K, RG><<<1, 32 * (S.ell_warps + 1), smem, s>>>(
+      S.info.row0, nst, (const k::EllRec*)S.d_ell_recs, S.d_ell_data, bw, xs, NST, RMAX, PMAX, SMAX, XW, tr);
+  return {SPTRSV_SUCCESS, ""};
+}
+
+// Supernodal pieces (see k::tri_supernode): per piece its shared external
+// column list, the dense external values V_J (column-major, ld = width) and
+// the packed strictly-lower diagonal block.  Values are the D^-1-scaled ones
+// of the segment (R27).
+void build_supernodes(Segment& S, size_t vb) {
+  S.sn_desc.clear();
+  S.sn_cols.clear();
+  S.sn_vals.clear();
+  S.sn_blk.clear();
+  const auto& I = S.info;
+  if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_SUPERNODE) return;
+  const int np = (int)S.sn_ptr.size() - 1;
+  std::vector<k::SnDesc> desc(np);
+  size_t nv = 0, nb = 0, nc = 0;
+  for (int J = 0; J < np; ++J) {
+    const int a = S.sn_ptr[J], w = S.sn_ptr[J + 1] - a;
+    const int ne = S.rp[a + 1] - S.rp[a];
+    desc[J] = k::SnDesc{I.row0 + a, w, ne, (int)nc, (long long)nv, (long long)nb};
+    nc += ne;
+    nv += (size_t)ne * w;
+    nb += (size_t)w * (w - 1) / 2;
+  }
+  S.sn_cols.resize(nc);
+  S.sn_vals.assign(std::max<size_t>(nv, 1) * vb, 0);
+  S.sn_blk.assign(std::max<size_t>(nb, 1) * vb, 0);
+  for (int J = 0; J < np; ++J) {
+    const k::SnDesc& d = desc[J];
+    const int a = S.sn_ptr[J];
+    std::memcpy(&S.sn_cols[d.coff], &S.ci[S.rp[a]], (size_t)d.ne * 4);
+    for (int t = 0; t < d.w; ++t) {
+      const int base = S.rp[a + t];
+      for (int q = 0; q < d.ne; ++q)
+        std::memcpy(&S.sn_vals[((size_t)d.voff + (size_t)q * d.w + t) * vb], &S.val[(size_t)(base + q) * vb], vb);
+      for (int c = 0; c < t; ++c) {
+        const size_t off = (size_t)d.boff + (size_t)c * (d.w - 1) - (size_t)c * (c - 1) / 2 + (t - c - 1);
+        std::memcpy(&S.sn_blk[off * vb], &S.val[(size_t)(base + d.ne + c) * vb], vb);
+      }
+    }
+  }
+  S.sn_desc.resize((size_t)np * sizeof(k::SnDesc));
+  std::memcpy(S.sn_desc.data(), desc.data(), S.sn_desc.size());
+}
+
+// Partitioned pipeline chain (see k::tri_chain_pipe).  Partitions are
+// contiguous ranges of the ORIGINAL (lower) row index, balanced in rows; a
+// partition's rows keep the triangle's level order; groups are 32 rows of
+// one level; stages are GMAX consecutive groups.
+void build_pipeline(const Plan& p, Segment& S, size_t vb) {
+  S.pipe_P = 0;
+  S.pipe_K = 0;
+  S.pipe_recs.clear();
+  S.pipe_data.clear();
+  S.pipe_stage0.clear();
+  const auto& I = S.info;
+  if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_PIPE) return;
+  const int m = I.row1 - I.row0;
+  int K = 0;
+  for (int r = 0; r < m; ++r) K = std::max(K, S.rp[r + 1] - S.rp[r]);
+  if (K < 1 || K > 4 || m < 1) return;  // the launcher falls back to the chain kernel
+  const int XW = 8192, NST = 3, GMAX = K <= 2 ? 32 : 16;
+  const int RM = GMAX * 32;
+  int P = (int)std::max<int64_t>(1, std::min<int64_t>(p.sm_count / 2, m / 32768));
+  if (const char* e = std::getenv("SPTRSV_PIPE_P")) P = std::max(1, std::min(p.sm_count, std::atoi(e)));
+  // partition by rank of the original (lower) row index
+  std::vector<int32_t> order(m), part(m), pos(m);
+  std::iota(order.begin(), order.end(), 0);
+  std::sort(order.begin(), order.end(),
+            [&](int a, int b) { return p.lower_old[I.row0 + a] < p.lower_old[I.row0 + b]; });
+  for (int q = 0; q < m; ++q) part[order[q]] = (int)((int64_t)q * P / m);
+  std::vector<std::vector<int32_t>> rows(P);
+  for (int r = 0; r < m; ++r) {
+    pos[r] = (int32_t)rows[part[r]].size();
+    rows[part[r]].push_back(r);
+  }
+  const uint32_t mask = (uint32_t)XW - 1;
+  S.pipe_stage0.push_back(0);
+  std::vector<std::pair<std::vector<int32_t>, int>> stage_rows;  // padded rows (-1 = pad), pos0
+  int g90src = 0;
+  std::vector<int> gpl;  // groups per (partition, level)
+  for (int q = 0; q < P; ++q) {
+    const auto& R = rows[q];
+    // groups: runs of one level, chunks of 32
+    std::vector<std::vector<int32_t>> groups;
+    for (size_t a = 0; a < R.size();) {
+      const int lv = p.leaf_level[I.row0 + R[a]];
+      size_t b = a;
+      while (b < R.size() && p.leaf_level[I.row0 + R[b]] == lv) ++b;
+      gpl.push_back((int)((b - a + 31) / 32));
+      for (size_t c = a; c < b; c += 32) {
+        std::vector<int32_t> gr(32, -1);
+        for (size_t d = c; d < std::min(b, c + 32); ++d) gr[d - c] = R[d];
+        groups.push_back(gr);
+      }
+      a = b;
+    }
+    for (size_t g0 = 0; g0 < groups.size(); g0 += GMAX) {
+      std::vector<int32_t> pr;
+      int pos0 = -1;
+      for (size_t g = g0; g < std::min(groups.size(), g0 + GMAX); ++g)
+        for (int r : groups[g]) {
+          pr.push_back(r);
+          if (r >= 0 && pos0 < 0) pos0 = pos[r];
+        }
+      stage_rows.push_back({pr, pos0});
+    }
+    S.pipe_stage0.push_back((int32_t)stage_rows.size());
+  }
+  (void)g90src;
+  const int ns = (int)stage_rows.size();
+  S.pipe_recs.assign((size_t)ns * 16, 0);
+  std::vector<size_t> offs(ns);
+  size_t off = 0;
+  for (int t = 0; t < ns; ++t) {
+    const int npad = (int)stage_rows[t].first.size();
+    offs[t] = off;
+    off += vb == 8 ? k::pipe_off_b<double>(K, npad) - 64 : k::pipe_off_b<float>(K, npad) - 64;
+  }
+  S.pipe_data.assign(std::max<size_t>(off, 16), 0);
+  for (int t = 0; t < ns; ++t) {
+    const auto& pr = stage_rows[t].first;
+    const int npad = (int)pr.size();
+    char* blk = &S.pipe_data[offs[t]];  // == stage buffer + 64
+    int32_t* grow = (int32_t*)blk;
+    uint32_t* words = (uint32_t*)(blk + k::pipe_off_words(npad) - 64);
+    char* vals = blk + k::pipe_off_vals(K, npad) - 64;
+    int pos1 = stage_rows[t].second;
+    for (int i = 0; i < npad; ++i) {
+      const int r = pr[i];
+      for (int k2 = 0; k2 <= K; ++k2) words[(size_t)k2 * npad + i] = (uint32_t)XW;  // zero slot
+      if (r < 0) {
+        grow[i] = -1;
+        continue;
+      }
+      grow[i] = I.row0 + r;
+      pos1 = std::max(pos1, pos[r] + 1);
+      words[(size_t)K * npad + i] = (uint32_t)pos[r] & mask;
+      int kk = 0;
+      for (int q = S.rp[r]; q < S.rp[r + 1]; ++q, ++kk) {
+        const int j = S.ci[q] - I.row0;  // local row of the dependency
+        const bool local = part[j] == part[r] && pos[r] - pos[j] <= XW - 2 * RM;
+        words[(size_t)kk * npad + i] = local ? ((uint32_t)pos[j] & mask) : (0x80000000u | (uint32_t)S.ci[q]);
+        std::memcpy(vals + ((size_t)kk * npad + i) * vb, &S.val[(size_t)q * vb], vb);
+      }
+    }
+    int32_t* R = &S.pipe_recs[(size_t)t * 16];
+    const size_t bytes = vb == 8 ? k::pipe_off_b<double>(K, npad) - 64 : k::pipe_off_b<float>(K, npad) - 64;
+    R[0] = stage_rows[t].second; R[1] = pos1; R[2] = npad / 32; R[3] = (int32_t)(offs[t] / 16);
+    R[4] = (int32_t)bytes; R[5] = npad;
+  }
+  // consumer warps: twice the typical groups per level (warps on level l+1
+  // wait on level l through the shared-memory flags: a pipeline, not a barrier)
+  std::nth_element(gpl.begin(), gpl.begin() + gpl.size() * 9 / 10, gpl.end());
+  const int g90 = gpl.empty() ? 1 : gpl[gpl.size() * 9 / 10];
+  int nw = std::max(4, std::min(16, 2 * g90));
+  if (const char* e = std::getenv("SPTRSV_PIPE_WARPS")) nw = std::max(1, std::min(31, std::atoi(e)));
+  S.pipe_NW = nw;
+  S.pipe_P = P;
+  S.pipe_K = K;
+  S.pipe_GMAX = GMAX;
+  S.pipe_XW = XW;
+  S.pipe_NST = NST;
+}
+
+template <typename T, int K>
+Error launch_pipe(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
+  const uint32_t smem = S.pipe_NST * k::pipe_stage_bytes<T>(K, S.pipe_GMAX) +
+                        k::al16((S.pipe_XW + 2) * (uint32_t)sizeof(T)) + 16 * S.pipe_NST;
+  static uint32_t attr_bytes = 0;  // per template instance
+  if (smem > attr_bytes) {
+    CUDA_TRY(cudaFuncSetAttribute(k::tri_chain_pipe<T, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    attr_bytes = smem;
+  }
+  k::tri_chain_pipe<T, K><<<S.pipe_P, 32 * (S.pipe_NW + 1), smem, s>>>(
+      S.pipe_P, S.d_pipe_stage0, (const k::PipeRec*)S.d_pipe_recs, S.d_pipe_data, bw, xs, S.pipe_NST, S.pipe_GMAX,
+      S.pipe_XW, st, S.ticket_slot);
   return {SPTRSV_SUCCESS, ""};
 }
 
@@ -278,14 +546,14 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
               k::sq_scalar_1<T, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
           }
         } else {
-          dispatch_multi(nrhs, [&](auto G, auto R) {
+          dispatch_multi_un(nrhs, p.spmm, [&](auto G, auto R, auto U) {
             unsigned g = cdiv((int64_t)S.nzr * G, 256);
             if (dcsr)
-              k::sq_multi<T, G, R, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw,
-                                                           nrhs);
+              k::sq_multi<T, G, R, U, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs,
+                                                              bw, nrhs);
             else
-              k::sq_multi<T, G, R, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw,
-                                                            nrhs);
+              k::sq_multi<T, G, R, U, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs,
+                                                               bw, nrhs);
           });
         }
       }
@@ -307,14 +575,27 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
                 k::tri_level_1<T, false><<<cdiv(rb - ra, 256), 256, 0, s>>>(ra, rb, I.row0, S.d_rp, S.d_ci, val,
                                                                           bw, xs);
             } else {
-              dispatch_multi(nrhs, [&](auto G, auto R) {
-                k::tri_level_multi<T, G, R><<<cdiv((int64_t)(rb - ra) * G, 256), 256, 0, s>>>(
+              dispatch_multi_un(nrhs, p.spmm, [&](auto G, auto R, auto U) {
+                k::tri_level_multi<T, G, R, U><<<cdiv((int64_t)(rb - ra) * G, 256), 256, 0, s>>>(
                     ra, rb, I.row0, S.d_rp, S.d_ci, val, bw, xs, nrhs);
               });
             }
           }
           break;
         }
+        case SPTRSV_IMPL_TRI_PIPE:
+          if (nrhs == 1 && S.pipe_K > 0) {
+            Error e;
+            switch (S.pipe_K) {
+              case 1: e = launch_pipe<T, 1>(p, S, bw, xs, st, s); break;
+              case 2: e = launch_pipe<T, 2>(p, S, bw, xs, st, s); break;
+              case 3: e = launch_pipe<T, 3>(p, S, bw, xs, st, s); break;
+              default: e = launch_pipe<T, 4>(p, S, bw, xs, st, s); break;
+            }
+            if (e.status) return e;
+            break;
+          }
+          [[fallthrough]];  // nrhs > 1 or not buildable: the single-CTA chain
         case SPTRSV_IMPL_TRI_CHAIN: {
           if (nrhs == 1 && S.ell_K > 0) {
             Error e;
@@ -351,25 +632,47 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
               k::tri_chain_1<T, false><<<1, 1024, 0, s>>>(I.row0, I.nlevels, S.d_level_ptr, S.d_rp, S.d_ci, val,
                                                          bw, xs);
           } else {
-            dispatch_multi(nrhs, [&](auto G, auto R) {
-              k::tri_chain_multi<T, G, R><<<1, 1024, 0, s>>>(I.row0, I.nlevels, S.d_level_ptr, S.d_rp, S.d_ci,
+            dispatch_multi_un(nrhs, p.spmm, [&](auto G, auto R, auto U) {
+              k::tri_chain_multi<T, G, R, U><<<1, 1024, 0, s>>>(I.row0, I.nlevels, S.d_level_ptr, S.d_rp, S.d_ci,
                                                             val, bw, xs, nrhs);
             });
           }
           break;
         }
+        case SPTRSV_IMPL_TRI_SUPERNODE:
+          if (nrhs == 1) {
+            const int np = (int)S.sn_ptr.size() - 1;
+            const unsigned g = std::max(1u, std::min<unsigned>(cdiv(np, 8), p.sm_count * 8));
+            k::tri_supernode<T><<<g, 256, 0, s>>>(np, (const k::SnDesc*)S.d_sn_desc, S.d_sn_cols,
+                                                  (const T*)S.d_sn_vals, (const T*)S.d_sn_blk, bw, xs, st,
+                                                  S.ticket_slot);
+            break;
+          }
+          [[fallthrough]];  // nrhs > 1: the multi-RHS sync-free kernel on the CSR copy
         default: {  // SPTRSV_IMPL_TRI_SYNCFREE
+          // enough resident warps for about two of the triangle's widest
+          // levels: more only spin on rows whose dependencies are levels away
           const int cap = p.sm_count * 8;  // 8 CTAs x 8 warps per SM
+          const int64_t wl = std::max<int64_t>(1, I.max_level_rows);
+          // (round-1 sweeps on C3: 2 CTAs/SM best for thread-per-row, 3 for
+          // warp-per-row; the full 8/SM grid was 1.5x slower)
+          auto ctas = [&](int64_t rows_per_cta, int64_t rows_total) {
+            const int per_sm = rows_per_cta == 8 ? 3 : 2;
+            int64_t c = std::max<int64_t>((int64_t)per_sm * p.sm_count, cdiv(2 * wl, rows_per_cta));
+            if (rows_per_cta == 8) c = (int64_t)per_sm * p.sm_count;
+            if (const char* ev2 = std::getenv("SPTRSV_SF_CTAS")) c = std::max(1, std::atoi(ev2));
+            return (unsigned)std::min<int64_t>({c, (int64_t)cap, (int64_t)cdiv(rows_total, rows_per_cta)});
+          };
           if (nrhs == 1) {
             if (tri_use_warp(S))
-              k::tri_syncfree_warp<T, 4><<<std::min<unsigned>(cdiv(m, 8), cap), 256, 0, s>>>(
-                  I.row0, m, S.d_rp, S.d_ci, val, bw, xs, st, S.ticket_slot);
+              k::tri_syncfree_warp<T, 8><<<std::max(1u, ctas(8, m)), 256, 0, s>>>(I.row0, m, S.d_rp, S.d_ci, val,
+                                                                                  bw, xs, st, S.ticket_slot);
             else
-              k::tri_syncfree_thread<T, 4><<<std::min<unsigned>(cdiv(m, 256), cap), 256, 0, s>>>(
+              k::tri_syncfree_thread<T, 4, 32><<<std::max(1u, ctas(256, m)), 256, 0, s>>>(
                   I.row0, m, S.d_rp, S.d_ci, val, bw, xs, st, S.ticket_slot);
           } else {
             dispatch_multi(nrhs, [&](auto G, auto R) {
-              k::tri_syncfree_multi<T, G, R><<<std::min<unsigned>(cdiv((int64_t)m * G, 256), cap), 256, 0, s>>>(
+              k::tri_syncfree_multi<T, G, R><<<std::max(1u, ctas(256 / G, m)), 256, 0, s>>>(
                   I.row0, m, S.d_rp, S.d_ci, val, bw, xs, st, S.ticket_slot, nrhs);
             });
           }
@@ -443,8 +746,26 @@ Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs
   T* bw = (T*)p.ws.bw;
   T* xs = (T*)p.ws.xs;
   const T* rd = (const T*)p.d_rdiag;
-  const int fill = p.needs_sentinel ? 1 : 0;
-  k::SolveState st{p.d_tickets, p.nticket, p.d_error};
+  // nrhs == 1: sync-free rows poll their dependencies' values, which start
+  // as the sentinel; nrhs > 1: they poll per-row epoch flags instead
+  const int fill = (p.needs_sentinel && nrhs == 1) ? 1 : 0;
+  uint32_t epoch = 0;
+  if (nrhs > 1 && p.needs_sentinel) {
+    if (!p.ws.flags) {
+      if (cudaMalloc(&p.ws.flags, (size_t)std::max(1, n) * 4) != cudaSuccess) {
+        cudaGetLastError();
+        return {SPTRSV_ERROR_ALLOC, "flag workspace allocation failed"};
+      }
+      CUDA_TRY(cudaMemsetAsync(p.ws.flags, 0, (size_t)std::max(1, n) * 4, s));
+      p.epoch = 0;
+    }
+    if (++p.epoch == 0) {  // wrapped after 2^32 solves: restart from clean flags
+      CUDA_TRY(cudaMemsetAsync(p.ws.flags, 0, (size_t)std::max(1, n) * 4, s));
+      p.epoch = 1;
+    }
+    epoch = p.epoch;
+  }
+  k::SolveState st{p.d_tickets, p.nticket, p.d_error, (uint32_t*)p.ws.flags, epoch, p.backoff_ns};
   cudaEvent_t* ev = nullptr;
   if (p.profiling) {
     size_t need_ev = p.segs.size() + 3;
@@ -514,9 +835,12 @@ Error upload(Plan& p, void* stream_v) {
   };
   size_t o_perm = take((size_t)2 * n * 4);  // perm (new->old) then iperm (old->new)
   size_t o_rdiag = take((size_t)n * vb);
-  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed; };
+  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed, sd, sc, sv, sbk, ps, pr, pd; };
   std::vector<Offs> so(p.segs.size());
   p.trace = std::getenv("SPTRSV_TRACE") != nullptr;
+  p.spmm = spmm_cfg();
+  p.backoff_ns = 128;
+  if (const char* e = std::getenv("SPTRSV_SF_BACKOFF")) p.backoff_ns = (uint32_t)std::max(0, std::atoi(e));
   const k::ChainGeom cg = chain_geometry(p);
   p.chain_geom[0] = cg.NST; p.chain_geom[1] = cg.RMAX; p.chain_geom[2] = cg.EMAX;
   p.chain_geom[3] = cg.XW; p.chain_geom[4] = cg.LMAX;
@@ -526,6 +850,8 @@ Error upload(Plan& p, void* stream_v) {
     Segment& S = p.segs[i];
     build_chain_stages(S, cg);
     build_chain_ell(S, vb);
+    build_supernodes(S, vb);
+    build_pipeline(p, S, vb);
     so[i].er = take(S.ell_recs.size() * 4);
     so[i].ed = take(S.ell_data.size());
     so[i].rp = take(S.rp.size() * 4);
@@ -534,8 +860,17 @@ Error upload(Plan& p, void* stream_v) {
     so[i].rows = take(S.rows.size() * 4);
     so[i].lp = take(S.level_ptr.size() * 4);
     so[i].st = take(S.chain_recs.size() * 4);
+    so[i].sd = take(S.sn_desc.size());
+    so[i].sc = take(S.sn_cols.size() * 4);
+    so[i].sv = take(S.sn_vals.size());
+    so[i].sbk = take(S.sn_blk.size());
+    so[i].ps = take(S.pipe_stage0.size() * 4);
+    so[i].pr = take(S.pipe_recs.size() * 4);
+    so[i].pd = take(S.pipe_data.size());
     if (S.info.kind == 0) S.ticket_slot = p.nticket++;
-    if (S.info.kind == 0 && S.info.impl == SPTRSV_IMPL_TRI_SYNCFREE) p.needs_sentinel = true;
+    if (S.info.kind == 0 && (S.info.impl == SPTRSV_IMPL_TRI_SYNCFREE || S.info.impl == SPTRSV_IMPL_TRI_SUPERNODE ||
+                             S.info.impl == SPTRSV_IMPL_TRI_PIPE))
+      p.needs_sentinel = true;
   }
   size_t o_tickets = take((size_t)std::max(1, p.nticket) * 4);
   p.arena_bytes = off;
@@ -575,6 +910,20 @@ Error upload(Plan& p, void* stream_v) {
     std::memcpy(&h[so[i].ed], S.ell_data.data(), S.ell_data.size());
     S.d_ell_recs = (const int32_t*)(A + so[i].er);
     S.d_ell_data = (const char*)(A + so[i].ed);
+    std::memcpy(&h[so[i].sd], S.sn_desc.data(), S.sn_desc.size());
+    std::memcpy(&h[so[i].sc], S.sn_cols.data(), S.sn_cols.size() * 4);
+    std::memcpy(&h[so[i].sv], S.sn_vals.data(), S.sn_vals.size());
+    std::memcpy(&h[so[i].sbk], S.sn_blk.data(), S.sn_blk.size());
+    S.d_sn_desc = (const void*)(A + so[i].sd);
+    S.d_sn_cols = (const int32_t*)(A + so[i].sc);
+    S.d_sn_vals = (const void*)(A + so[i].sv);
+    S.d_sn_blk = (const void*)(A + so[i].sbk);
+    std::memcpy(&h[so[i].ps], S.pipe_stage0.data(), S.pipe_stage0.size() * 4);
+    std::memcpy(&h[so[i].pr], S.pipe_recs.data(), S.pipe_recs.size() * 4);
+    std::memcpy(&h[so[i].pd], S.pipe_data.data(), S.pipe_data.size());
+    S.d_pipe_stage0 = (const int32_t*)(A + so[i].ps);
+    S.d_pipe_recs = (const int32_t*)(A + so[i].pr);
+    S.d_pipe_data = (const char*)(A + so[i].pd);
   }
   p.d_perm = (const int32_t*)(A + o_perm);
   p.d_rdiag = (const void*)(A + o_rdiag);
@@ -660,6 +1009,7 @@ void release(Plan& p) {
   if (p.ws.xs) cudaFree(p.ws.xs);
   if (p.ws.stage_b) cudaFree(p.ws.stage_b);
   if (p.ws.stage_x) cudaFree(p.ws.stage_x);
+  if (p.ws.flags) cudaFree(p.ws.flags);
   if (p.h_error) cudaFreeHost(p.h_error);
   for (auto& S : p.segs)
     if (S.d_trace) cudaFree(S.d_trace);

@@ -33,6 +33,7 @@ struct Segment {
   std::vector<int32_t> rows;       // DCSR: global permuted row of every stored row
   std::vector<int32_t> level_ptr;  // TRI: nlevels+1 local row offsets
   std::vector<int32_t> in_degree;  // TRI: off-diagonal count per local row
+  std::vector<int32_t> sn_ptr;     // TRI: fundamental-supernode pieces (<= 32 rows), local row starts + m
   int32_t nzr = 0;                 // SQ: stored rows (== m for CSR)
   // ----- device -----
   const int32_t* d_rp = nullptr;
@@ -41,14 +42,31 @@ struct Segment {
   const int32_t* d_rows = nullptr;
   const int32_t* d_level_ptr = nullptr;  // device copy (chain / level-set kernels)
   int32_t ticket_slot = -1;              // sync-free: index into the device ticket array
+  // supernodal kernel (nrhs == 1): piece descriptors, shared external
+  // column lists, dense external values (column-major, ld = width) and the
+  // packed strictly-lower diagonal blocks
+  std::vector<char> sn_desc, sn_vals, sn_blk;
+  std::vector<int32_t> sn_cols;
+  const void* d_sn_desc = nullptr;
+  const int32_t* d_sn_cols = nullptr;
+  const void* d_sn_vals = nullptr;
+  const void* d_sn_blk = nullptr;
+  // partitioned pipeline chain (nrhs == 1): P partitions, per-partition stages
+  int pipe_P = 0, pipe_K = 0, pipe_NW = 4, pipe_GMAX = 32, pipe_XW = 8192, pipe_NST = 3;
+  std::vector<int32_t> pipe_stage0;  // [P+1] first stage of every partition
+  std::vector<int32_t> pipe_recs;    // 16 ints per stage (k::PipeRec + pad)
+  std::vector<char> pipe_data;       // stage blocks
+  const int32_t* d_pipe_stage0 = nullptr;
+  const int32_t* d_pipe_recs = nullptr;
+  const char* d_pipe_data = nullptr;
   // TMA-staged chain kernel (nrhs == 1): 8-int stage records (k::StageRec),
   // empty = not staged
   std::vector<int32_t> chain_recs;
   const int32_t* d_chain_recs = nullptr;
   // ELL-staged chain kernel (nrhs == 1, rows with <= 4 window-resident deps)
-  int ell_K = 0, ell_NST = 0, ell_RMAX = 0, ell_XW = 0, ell_warps = 8;  // ell_K == 0: not used
+  int ell_K = 0, ell_NST = 0, ell_RMAX = 0, ell_PMAX = 0, ell_SMAX = 0, ell_XW = 0, ell_warps = 8;  // ell_K == 0: not used
   std::vector<int32_t> ell_recs;   // 16 ints per stage (k::EllRec + the record of stage s + NST)
-  std::vector<char> ell_data;      // per-stage blocks: slots[K][npad] int32, values[K][npad]
+  std::vector<char> ell_data;      // per-stage blocks: step records int4[nsteps], u16 slot pairs [W][npad], values [K][npad]
   const int32_t* d_ell_recs = nullptr;
   const char* d_ell_data = nullptr;
   void* d_trace = nullptr;          // debug trace (SPTRSV_TRACE)
@@ -62,6 +80,12 @@ struct Workspace {
   void* stage_b = nullptr;  // host-pointer path staging (col-major n x nrhs)
   void* stage_x = nullptr;
   size_t stage_bytes = 0;
+  void* flags = nullptr;    // nrhs > 1 sync-free: per-row ready flags (n x u32), epoch-valued
+};
+
+// SpMM lane geometry for nrhs > 1 (exec.cu: dispatch_multi_un)
+struct SpmmCfg {
+  int rpt_max = 8, un = 2;  // measured best on C5 (round 1 sweep, profiles/r01_sweeps.md)
 };
 
 struct Plan {
@@ -74,11 +98,13 @@ struct Plan {
   int32_t sm_count = 148;
   int64_t min_block_rows = 0;
   double analyse_ms = 0.0;
+  int32_t reorder_eff = 0;  // reorder actually applied (0 level, 1 none)
   size_t vbytes = 8;
 
   std::vector<Segment> segs;
   std::vector<int32_t> perm;        // new -> old (original indexing; UPPER composed with J)
   std::vector<int32_t> leaf_level;  // level of every new row inside its leaf
+  std::vector<int32_t> lower_old;   // new row -> row of the (J U J for UPPER) lower input
   std::vector<char> diag_new;       // diagonal in new order (dtype)
   std::vector<char> rdiag_new;      // 1 / diagonal in new order (dtype), what kernels read
   // P L P^T kept on the host for introspection (sptrsv_plan_matrix)
@@ -100,6 +126,9 @@ struct Plan {
   int32_t* h_error = nullptr;  // mapped pinned host word set by the watchdog
   int32_t* d_error = nullptr;  // its device alias
   Workspace ws;
+  SpmmCfg spmm;
+  uint32_t backoff_ns = 128;  // sync-free polling backoff cap
+  uint32_t epoch = 0;  // last multi-RHS solve's epoch (flags hold it when a row is solved)
   int launches_per_solve = 0;
 
   // profiling

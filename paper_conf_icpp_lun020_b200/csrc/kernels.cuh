@@ -75,6 +75,9 @@ struct SolveState {
   uint32_t* tickets;  // per-segment row-claim counters, zeroed by permute-in
   int nticket;
   int* error;         // mapped host word (watchdog)
+  uint32_t* flags;    // nrhs > 1: per-row ready flags (global row index), value = epoch when solved
+  uint32_t epoch;     // this solve's epoch (>= 1; flags start at 0)
+  uint32_t backoff_ns;  // cap of the sync-free polling backoff (0 = spin)
 };
 
 __device__ __forceinline__ void reset_tickets(const SolveState& st, int tid, int nthreads) {
@@ -214,8 +217,49 @@ __global__ void sq_vector_1(int nzr, int r0, const int* __restrict__ rows, const
 }
 
 // SpMM update for nrhs > 1 (K9): a group of G lanes per row, lanes over the
-// RHS columns (RPT per lane per pass), entries of the row sequential.
-template <typename T, int G, int RPT, bool DCSR>
+// RHS columns (RPT per lane per pass), entries of the row two at a time so
+// 2*RPT independent X gathers per lane are in flight (round-1 ncu: one entry
+// at a time left the kernel latency-bound at 3.5 TB/s, long_scoreboard 116).
+template <typename T, bool NC>
+__device__ __forceinline__ T ldx(const T* p) {
+  if constexpr (NC) return ldg_nc(p);
+  else return *p;
+}
+
+template <typename T, int RPT, bool NC = true, int UN = 1>
+__device__ __forceinline__ void gather_row_update(T (&acc)[RPT], int a, int e, const int* __restrict__ ci,
+                                                  const T* __restrict__ val, const T* __restrict__ xs, int nrhs,
+                                                  int cbase, int G, int ncol) {
+  int p = a;
+  if constexpr (UN == 2) {
+    for (; p + 1 < e; p += 2) {
+      const int j0 = ldg_nc(ci + p), j1 = ldg_nc(ci + p + 1);
+      const T v0 = ldg_nc(val + p), v1 = ldg_nc(val + p + 1);
+      const T* x0 = xs + (int64_t)j0 * nrhs + cbase;
+      const T* x1 = xs + (int64_t)j1 * nrhs + cbase;
+      T y0[RPT], y1[RPT];
+#pragma unroll
+      for (int t = 0; t < RPT; ++t)
+        if (G * t < ncol) {
+          y0[t] = ldx<T, NC>(x0 + G * t);
+          y1[t] = ldx<T, NC>(x1 + G * t);
+        }
+#pragma unroll
+      for (int t = 0; t < RPT; ++t)
+        if (G * t < ncol) acc[t] += v0 * y0[t] + v1 * y1[t];
+    }
+  }
+  for (; p < e; ++p) {
+    const int j0 = ldg_nc(ci + p);
+    const T v0 = ldg_nc(val + p);
+    const T* x0 = xs + (int64_t)j0 * nrhs + cbase;
+#pragma unroll
+    for (int t = 0; t < RPT; ++t)
+      if (G * t < ncol) acc[t] += v0 * ldx<T, NC>(x0 + G * t);
+  }
+}
+
+template <typename T, int G, int RPT, int UN, bool DCSR>
 __global__ void sq_multi(int nzr, int r0, const int* __restrict__ rows, const int* __restrict__ rp,
                          const int* __restrict__ ci, const T* __restrict__ val, const T* __restrict__ xs,
                          T* __restrict__ bw, int nrhs) {
@@ -227,13 +271,8 @@ __global__ void sq_multi(int nzr, int r0, const int* __restrict__ rows, const in
     T acc[RPT];
 #pragma unroll
     for (int t = 0; t < RPT; ++t) acc[t] = 0;
-    for (int p = a; p < e; ++p) {
-      T v = ldg_nc(val + p);
-      const T* xr = xs + (int64_t)ldg_nc(ci + p) * nrhs + c0 + lane;
-#pragma unroll
-      for (int t = 0; t < RPT; ++t)
-        if (c0 + lane + G * t < nrhs) acc[t] += v * ldg_nc(xr + G * t);
-    }
+    // columns c0 + lane + G*t < nrhs  <=>  G*t < nrhs - c0 - lane
+    gather_row_update<T, RPT, true, UN>(acc, a, e, ci, val, xs, nrhs, c0 + lane, G, nrhs - c0 - lane);
     T* br = bw + (int64_t)r * nrhs + c0 + lane;
 #pragma unroll
     for (int t = 0; t < RPT; ++t)
@@ -263,36 +302,33 @@ __global__ void tri_level_1(int ra, int rb, int r0, const int* __restrict__ rp, 
   }
 }
 
-template <typename T, int G, int RPT>
+// x_r = b'_r - sum_j l'_rj x_j for the RHS columns this lane owns.  NC:
+// the x_j come from earlier launches (level-set) and may use the
+// non-coherent path; the single-CTA chain reads them with plain loads.
+template <typename T, int G, int RPT, bool NC, int UN>
 __device__ __forceinline__ void row_multi_solve(int r, int a, int e, const int* __restrict__ ci,
                                                 const T* __restrict__ val, const T* __restrict__ bw,
                                                 T* __restrict__ xs, int nrhs, int lane) {
   for (int c0 = 0; c0 < nrhs; c0 += G * RPT) {
     T acc[RPT];
 #pragma unroll
-    for (int t = 0; t < RPT; ++t)
-      acc[t] = (c0 + lane + G * t < nrhs) ? bw[(int64_t)r * nrhs + c0 + lane + G * t] : T(0);
-    for (int p = a; p < e; ++p) {
-      T v = ldg_nc(val + p);
-      const T* xr = xs + (int64_t)ldg_nc(ci + p) * nrhs + c0 + lane;
-#pragma unroll
-      for (int t = 0; t < RPT; ++t)
-        if (c0 + lane + G * t < nrhs) acc[t] -= v * xr[G * t];
-    }
+    for (int t = 0; t < RPT; ++t) acc[t] = 0;
+    gather_row_update<T, RPT, NC, UN>(acc, a, e, ci, val, xs, nrhs, c0 + lane, G, nrhs - c0 - lane);
     T* xo = xs + (int64_t)r * nrhs + c0 + lane;
+    const T* bo = bw + (int64_t)r * nrhs + c0 + lane;
 #pragma unroll
     for (int t = 0; t < RPT; ++t)
-      if (c0 + lane + G * t < nrhs) xo[G * t] = acc[t];
+      if (c0 + lane + G * t < nrhs) xo[G * t] = bo[G * t] - acc[t];
   }
 }
 
-template <typename T, int G, int RPT>
+template <typename T, int G, int RPT, int UN>
 __global__ void tri_level_multi(int ra, int rb, int r0, const int* __restrict__ rp, const int* __restrict__ ci,
                                 const T* __restrict__ val, const T* __restrict__ bw, T* __restrict__ xs,
                                 int nrhs) {
   int r = ra + (blockIdx.x * blockDim.x + threadIdx.x) / G, lane = threadIdx.x % G;
   if (r >= rb) return;
-  row_multi_solve<T, G, RPT>(r, rp[r - r0], rp[r - r0 + 1], ci, val, bw, xs, nrhs, lane);
+  row_multi_solve<T, G, RPT, true, UN>(r, rp[r - r0], rp[r - r0 + 1], ci, val, bw, xs, nrhs, lane);
 }
 
 // ---------------------------------------- K4: single-CTA level chain (unstaged)
@@ -330,7 +366,7 @@ __global__ void __launch_bounds__(1024) tri_chain_1(int r0, int nlev, const int*
   }
 }
 
-template <typename T, int G, int RPT>
+template <typename T, int G, int RPT, int UN>
 __global__ void __launch_bounds__(1024) tri_chain_multi(int r0, int nlev, const int* __restrict__ lp,
                                                         const int* __restrict__ rp, const int* __restrict__ ci,
                                                         const T* __restrict__ val, const T* __restrict__ bw,
@@ -339,7 +375,7 @@ __global__ void __launch_bounds__(1024) tri_chain_multi(int r0, int nlev, const 
   for (int l = 0; l < nlev; ++l) {
     int ra = r0 + lp[l], rb = r0 + lp[l + 1];
     for (int r = ra + grp; r < rb; r += ng)
-      row_multi_solve<T, G, RPT>(r, rp[r - r0], rp[r - r0 + 1], ci, val, bw, xs, nrhs, lane);
+      row_multi_solve<T, G, RPT, false, UN>(r, rp[r - r0], rp[r - r0 + 1], ci, val, bw, xs, nrhs, lane);
     __syncthreads();
   }
 }
@@ -349,13 +385,48 @@ __global__ void __launch_bounds__(1024) tri_chain_multi(int r0, int nlev, const 
 // Components are claimed from a per-segment ticket in row order, so every
 // dependency of a claimed row was claimed earlier by a running warp: no
 // deadlock whatever the CTA scheduling.  A dependency is "satisfied" (the
-// in-degree test of Alg 3) when its x_j is no longer the sentinel.
+// in-degree test of Alg 3) when its x_j is no longer the sentinel
+// (nrhs == 1) or its row flag carries this solve's epoch (nrhs > 1).
 //
-// Thread-per-component: a warp claims 32 consecutive rows; each lane
-// consumes its dependencies in batches of U independent loads, stopping at
-// the first unsolved one and retrying on the next pass (non-blocking, so a
-// lane never blocks a lower lane of its own warp that it depends on).
-template <typename T, int U>
+// Polling discipline: in the thread-per-row and multi-RHS kernels a warp
+// whose polls made no progress sleeps (__nanosleep, exponential backoff
+// capped at SolveState::backoff_ns, SPTRSV_SF_BACKOFF) before polling again,
+// so blocked warps do not saturate the LSU / L2 with strong loads (round-1
+// ncu: the un-throttled kernel ran L1TEX at 95% with lg_throttle the second
+// stall reason, profiles/r01_c3_v0_ncu.md).  The warp-per-row kernel spins
+// (measured faster on C3/C4: its warps poll few, long rows).  The resident
+// grid is also sized to ~2 levels of rows (exec.cu), so few warps spin.
+constexpr unsigned kBackoffMinNs = 32;
+
+__device__ __forceinline__ unsigned backoff(unsigned ns, unsigned max_ns) {
+  if (max_ns == 0) return 0;  // pure spinning
+  ns = ns ? min(ns * 2u, max_ns) : min(kBackoffMinNs, max_ns);
+  __nanosleep(ns);
+  return ns;
+}
+
+__device__ __forceinline__ uint32_t ld_flag(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_flag(uint32_t* p, uint32_t v) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// Thread-per-component with warp help for long rows: a warp claims 32
+// consecutive rows.  A row with <= LONG dependencies is solved by its own
+// lane, which consumes its dependencies in batches of U independent loads,
+// stopping at the first unsolved one and retrying on the next pass
+// (non-blocking, so a lane never blocks a lower lane of its own warp that it
+// depends on).  A longer row (the power-law hubs of L136, which serialise a
+// lane for thousands of cycles) is solved by the WHOLE warp, 32*U entries per
+// attempt, lowest such row first; an attempt that meets an unsolved
+// dependency is abandoned without side effects and retried after the next
+// thread pass, so rows of the same chunk that the long row waits for keep
+// progressing (no deadlock: the long row only waits on lower rows, and the
+// lower long rows are finished first).
+template <typename T, int U, int LONG>
 __global__ void __launch_bounds__(256) tri_syncfree_thread(int r0, int m, const int* __restrict__ rp,
                                                            const int* __restrict__ ci, const T* __restrict__ val,
                                                            const T* __restrict__ bw, T* __restrict__ xs,
@@ -377,9 +448,12 @@ __global__ void __launch_bounds__(256) tri_syncfree_thread(int r0, int m, const 
       e = rp[k + 1];
       s = bw[r];
     }
+    const bool islong = !done && e - p > LONG;
     uint32_t spins = 0;
+    unsigned ns = 0;
     while (__any_sync(0xffffffffu, !done)) {
-      if (!done) {
+      bool prog = false;
+      if (!done && !islong) {
         bool progress = true;
         while (p < e && progress) {
           const int cnt = min(U, e - p);
@@ -402,23 +476,76 @@ __global__ void __launch_bounds__(256) tri_syncfree_thread(int r0, int m, const 
               ++took;
             }
           p += took;
+          prog |= took > 0;
           progress = took == cnt;
         }
         if (p == e) {
           st_strong(xs + r, s);
           done = true;
-        } else if (++spins > kWatchdogSpins) {
-          watchdog_trip(st);
-          p = e;  // give up: garbage result, reported to the host
+          prog = true;
         }
+      }
+      // warp pass: the lowest pending long row, 32*U entries per attempt
+      const unsigned lm = __ballot_sync(0xffffffffu, !done && islong);
+      if (lm) {
+        const int ow = __ffs(lm) - 1;
+        int wp = __shfl_sync(0xffffffffu, p, ow);
+        const int we = __shfl_sync(0xffffffffu, e, ow);
+        T acc = 0;
+        while (wp < we) {
+          int j[U];
+          T v[U], x[U];
+          bool ready = true;
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            const int q = wp + lane + 32 * u;
+            if (q < we) {
+              j[u] = ldg_nc(ci + q);
+              v[u] = ldg_nc(val + q);
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < U; ++u)
+            if (wp + lane + 32 * u < we) {
+              x[u] = ld_strong(xs + j[u]);
+              ready &= !is_sent(x[u]);
+            }
+          if (!__all_sync(0xffffffffu, ready)) break;  // abandon; retry after the next thread pass
+#pragma unroll
+          for (int u = 0; u < U; ++u)
+            if (wp + lane + 32 * u < we) acc += v[u] * x[u];
+          wp += 32 * U;
+          prog = true;
+        }
+        acc = warp_sum(acc);
+        if (lane == ow) {
+          s -= acc;
+          p = min(wp, we);
+          if (p == e) {
+            st_strong(xs + r, s);
+            done = true;
+          }
+        }
+      }
+      if (!__any_sync(0xffffffffu, prog)) {
+        if (++spins > kWatchdogSpins) {
+          if (!done) watchdog_trip(st);
+          done = true;  // give up: garbage result, reported to the host
+        } else {
+          ns = backoff(ns, st.backoff_ns);
+        }
+      } else {
+        ns = 0;
       }
     }
   }
 }
 
 // Warp-per-component (long rows): lanes stride the dependencies, U per lane
-// per batch, all loads of a batch in flight together; a lane spins only on
-// dependencies, which all precede the row in ticket order.
+// per round (32*U entries: every column index and value of the round is
+// loaded BEFORE the first poll, so the matrix stream never sits behind a
+// dependency wait); a lane spins only on dependencies, which all precede the
+// row in ticket order.
 template <typename T, int U>
 __global__ void __launch_bounds__(256) tri_syncfree_warp(int r0, int m, const int* __restrict__ rp,
                                                          const int* __restrict__ ci, const T* __restrict__ val,
@@ -468,8 +595,90 @@ __global__ void __launch_bounds__(256) tri_syncfree_warp(int r0, int m, const in
   }
 }
 
-// Multi-RHS sync-free: a group of G lanes per component, lanes over RHS
-// columns; each lane polls exactly the x_j values it consumes.
+// Supernodal sync-free (B200 selector, nrhs == 1): a warp per fundamental
+// supernode piece J = rows [s, s+w), w <= 32, claimed in row order from the
+// segment's ticket (deadlock-free like K3).  Lane t owns row s+t:
+//   1. y_t = b'_t - sum_q V_J[t][q] x_{E_J[q]}: the piece's rows share one
+//      list E_J of external columns, so 32 columns per round are polled by
+//      32 lanes (value-as-flag), broadcast by shuffles, and met by a
+//      coalesced column of V_J (loaded before the poll);
+//   2. x = T_J^{-1} y for the dense unit-lower diagonal block T_J (after the
+//      D^-1 scaling, R27): w-1 steps of shfl x_c -> DFMA, lane t's row of
+//      T_J in registers;
+//   3. x_t stored with a strong store, which publishes it (value-as-flag).
+// The critical path is one dependency hop per PIECE instead of one per row
+// (a 64-wide supernode is 64 levels of the row DAG).
+struct SnDesc {
+  int s, w, ne, coff;          // first global row, width, |E_J|, offset of E_J in cols
+  long long voff, boff;        // offsets (elements) of V_J and of the packed T_J
+};
+
+template <typename T>
+__global__ void __launch_bounds__(256) tri_supernode(int npieces, const SnDesc* __restrict__ desc,
+                                                     const int* __restrict__ cols, const T* __restrict__ V,
+                                                     const T* __restrict__ Tb, const T* __restrict__ bw,
+                                                     T* __restrict__ xs, SolveState st, int slot) {
+  const int lane = threadIdx.x & 31;
+  uint32_t* ticket = st.tickets + slot;
+  while (true) {
+    int J = 0;
+    if (lane == 0) J = (int)atomicAdd(ticket, 1u);
+    J = __shfl_sync(0xffffffffu, J, 0);
+    if (J >= npieces) break;
+    const SnDesc d = desc[J];
+    const bool act = lane < d.w;
+    T y = act ? bw[d.s + lane] : T(0);
+    for (int q0 = 0; q0 < d.ne; q0 += 32) {
+      const int nq = min(32, d.ne - q0);
+      const bool inq = lane < nq;
+      const int j = inq ? ldg_nc(cols + d.coff + q0 + lane) : 0;
+      T vr[32];
+      const T* Vq = V + d.voff + (long long)q0 * d.w + lane;
+#pragma unroll
+      for (int c = 0; c < 32; ++c) vr[c] = (c < nq && act) ? ldg_nc(Vq + (long long)c * d.w) : T(0);
+      T xj = inq ? ld_strong(xs + j) : T(0);
+      uint32_t spins = 0;
+      unsigned ns = 0;
+      while (__any_sync(0xffffffffu, inq && is_sent(xj))) {
+        if (++spins > kWatchdogSpins) {
+          watchdog_trip(st);
+          break;
+        }
+        ns = backoff(ns, st.backoff_ns);
+        if (inq && is_sent(xj)) xj = ld_strong(xs + j);
+      }
+#pragma unroll
+      for (int c = 0; c < 32; ++c) {
+        if (c < nq) {  // warp-uniform
+          const T xc = __shfl_sync(0xffffffffu, xj, c);
+          y -= vr[c] * xc;
+        }
+      }
+    }
+    // dense unit-lower diagonal block: column c of T_J holds rows c+1 .. w-1
+    // at Tb[boff + c(w-1) - c(c-1)/2 + (t - c - 1)]
+    T tl[31];
+#pragma unroll
+    for (int c = 0; c < 31; ++c) {
+      const long long off = d.boff + (long long)c * (d.w - 1) - (long long)c * (c - 1) / 2 + (lane - c - 1);
+      tl[c] = (act && lane > c && c < d.w - 1) ? ldg_nc(Tb + off) : T(0);
+    }
+#pragma unroll
+    for (int c = 0; c < 31; ++c) {
+      if (c < d.w - 1) {  // warp-uniform
+        const T xc = __shfl_sync(0xffffffffu, y, c);
+        y -= tl[c] * xc;  // lanes <= c hold tl[c] = 0
+      }
+    }
+    if (act) st_strong(xs + d.s + lane, y);
+  }
+}
+
+// Multi-RHS sync-free (SpTRSM): a group of G lanes per component, lanes over
+// the RHS columns.  Readiness is a per-row flag holding the solve's epoch
+// (no per-solve reset, no n x nrhs sentinel fill): the G lanes store the row,
+// each fences (membar.gl), the group syncs, lane 0 publishes the flag; a
+// reader polls the flag and then reads the row with strong (L2) loads.
 template <typename T, int G, int RPT>
 __global__ void __launch_bounds__(256) tri_syncfree_multi(int r0, int m, const int* __restrict__ rp,
                                                           const int* __restrict__ ci, const T* __restrict__ val,
@@ -478,6 +687,7 @@ __global__ void __launch_bounds__(256) tri_syncfree_multi(int r0, int m, const i
   const int lane = threadIdx.x % G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << ((threadIdx.x & 31) / G * G));
   uint32_t* ticket = st.tickets + slot;
+  const uint32_t epoch = st.epoch;
   while (true) {
     int k = 0;
     if (lane == 0) k = (int)atomicAdd(ticket, 1u);
@@ -493,6 +703,17 @@ __global__ void __launch_bounds__(256) tri_syncfree_multi(int r0, int m, const i
       for (int p = a; p < e; ++p) {
         const int j = ldg_nc(ci + p);
         const T v = ldg_nc(val + p);
+        if (c0 == 0) {  // later column chunks of this row find j already published
+          uint32_t spins = 0;
+          unsigned ns = 0;
+          while (ld_flag(st.flags + j) != epoch) {
+            if (++spins > kWatchdogSpins) {
+              watchdog_trip(st);
+              break;
+            }
+            ns = backoff(ns, st.backoff_ns);
+          }
+        }
         const T* xr = xs + (int64_t)j * nrhs + c0 + lane;
         T x[RPT];
 #pragma unroll
@@ -500,23 +721,16 @@ __global__ void __launch_bounds__(256) tri_syncfree_multi(int r0, int m, const i
           if (c0 + lane + G * t < nrhs) x[t] = ld_strong(xr + G * t);
 #pragma unroll
         for (int t = 0; t < RPT; ++t)
-          if (c0 + lane + G * t < nrhs) {
-            uint32_t spins = 0;
-            while (is_sent(x[t])) {
-              if (++spins > kWatchdogSpins) {
-                watchdog_trip(st);
-                break;
-              }
-              x[t] = ld_strong(xr + G * t);
-            }
-            acc[t] -= v * x[t];
-          }
+          if (c0 + lane + G * t < nrhs) acc[t] -= v * x[t];
       }
       T* xo = xs + (int64_t)r * nrhs + c0 + lane;
 #pragma unroll
       for (int t = 0; t < RPT; ++t)
-        if (c0 + lane + G * t < nrhs) st_strong(xo + G * t, acc[t]);
+        if (c0 + lane + G * t < nrhs) xo[G * t] = acc[t];
     }
+    __threadfence();  // this lane's x stores are visible at gpu scope ...
+    __syncwarp(gmask);
+    if (lane == 0) st_flag(st.flags + r, epoch);  // ... before the row's flag
   }
 }
 
@@ -749,83 +963,141 @@ __global__ void __launch_bounds__(1024, 1)
 // ------------------------- K4 (staged, ELL): narrow rows, window-resident deps
 // When every row of a chain triangle has at most K dependencies and every
 // dependency lies inside the x window of its level (both checked by the
-// analysis), each stage ships an ELL block instead of CSR: for slot k and
-// stage row i, the dependency's WINDOW SLOT (j mod XW; XW = a zero slot for
-// padding) and its value, column-major so lanes read consecutive words.  A
-// row is then K x {LDS slot, LDS value, LDS x, DFMA}: no row pointers, no
-// branches, no modulo on the dependency chain.
+// analysis), the triangle is cut into STEPS (a level, or a chunk of a level
+// wider than the CTA's row capacity) and every step into groups of 32 rows.
+// Step q's group gi is owned by consumer warp gi % NW (gi / NW < RG), lane l
+// owns row row_start(q) + 32 gi + l.  Per padded row a stage ships its K
+// dependency WINDOW SLOTS (u16, two per word; slot XW is a zero) and K
+// values, so one row is: LDS x_j (K, addresses computed before the barrier)
+// -> K DFMA -> STS x_i.  Consequences:
+//   * no row pointers, level pointers, bounds or modulo on the dependency
+//     chain; the per-step overhead is one 16-byte step record (broadcast);
+//   * the operands of step q+1 are loaded into registers before step q's
+//     barrier (software pipeline across levels);
+//   * x never goes to global memory from the consumers: when a stage is
+//     done, the producer warp copies its rows from the window to xs with one
+//     cp.async.bulk shared->global store (stages never wrap the window).
 struct EllRec {
-  int sa, sb, l0, nl, off16, npad, pad0, pad1;  // off16: stage block offset in 16-byte units
+  int sa, sb, nsteps, off16, bytes, npad, pad0, pad1;  // off16: stage block offset in 16-byte units
 };
 
+__host__ __device__ inline uint32_t ell_words(int K) { return (uint32_t)(K + 1) / 2; }
+
 template <typename T>
-__host__ __device__ inline uint32_t ell_stage_bytes(int K, int RMAX) {
-  const int npad = (RMAX + 3) & ~3;
-  return 64 + al16(K * npad * 4) + al16(K * npad * (uint32_t)sizeof(T)) + al16((RMAX + 4) * (uint32_t)sizeof(T)) +
-         al16((RMAX + 8) * 4);
+__host__ __device__ inline uint32_t ell_stage_bytes(int K, int RMAX, int PMAX, int SMAX) {
+  return 64 + 16u * SMAX + al16(ell_words(K) * PMAX * 4) + al16(K * PMAX * (uint32_t)sizeof(T)) +
+         al16((RMAX + 4) * (uint32_t)sizeof(T));
 }
 
-template <typename T, int K, int RPT>
+__device__ __forceinline__ double lds_x(uint32_t a, double) {
+  double v;
+  asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ float lds_x(uint32_t a, float) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts_x(uint32_t a, double v) {
+  asm volatile("st.shared.f64 [%0], %1;" ::"r"(a), "d"(v) : "memory");
+}
+__device__ __forceinline__ void sts_x(uint32_t a, float v) {
+  asm volatile("st.shared.f32 [%0], %1;" ::"r"(a), "f"(v) : "memory");
+}
+__device__ __forceinline__ void bulk_s2g(void* dst, uint32_t src_smem, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(src_smem), "r"(bytes)
+               : "memory");
+}
+
+template <typename T, int K, int RG>
 __global__ void __launch_bounds__(1024, 1)
-    tri_chain_ell(int r0, int nstage, const EllRec* __restrict__ recs, const int* __restrict__ lp,
-                  const char* __restrict__ ell, const T* __restrict__ bw, T* __restrict__ xs, int NST, int RMAX,
-                  int XW, long long* __restrict__ trace) {
+    tri_chain_ell(int r0, int nstage, const EllRec* __restrict__ recs, const char* __restrict__ ell,
+                  const T* __restrict__ bw, T* __restrict__ xs, int NST, int RMAX, int PMAX, int SMAX, int XW,
+                  long long* __restrict__ trace) {
   extern __shared__ __align__(128) unsigned char smem[];
+  constexpr int W = (K + 1) / 2;
+  constexpr uint32_t SH = sizeof(T) == 8 ? 3 : 2;
   const int tid = threadIdx.x;
   const int NC = blockDim.x - 32;
-  const int xmask = XW - 1;
-  const int npad_max = (RMAX + 3) & ~3;
-  const uint32_t cap_idx = al16(K * npad_max * 4), cap_val = al16(K * npad_max * (uint32_t)sizeof(T));
-  const uint32_t cap_b = al16((RMAX + 4) * (uint32_t)sizeof(T));
-  const uint32_t sbytes = ell_stage_bytes<T>(K, RMAX);
-  T* xw = (T*)(smem + NST * sbytes);  // XW slots + one zero slot
-  uint64_t* full = (uint64_t*)(smem + NST * sbytes + al16((XW + 2) * (uint32_t)sizeof(T)));
+  const int NW = NC >> 5, warp = tid >> 5, lane = tid & 31;
+  const uint32_t xmask = (uint32_t)XW - 1;
+  const uint32_t sbytes = ell_stage_bytes<T>(K, RMAX, PMAX, SMAX);
+  const uint32_t o_b = 64 + 16u * SMAX + al16(W * PMAX * 4) + al16(K * PMAX * (uint32_t)sizeof(T));
+  unsigned char* xw_p = smem + (size_t)NST * sbytes;  // XW slots + one zero slot
+  const uint32_t xw = smem_addr(xw_p);
+  uint64_t* full = (uint64_t*)(xw_p + al16((XW + 2) * (uint32_t)sizeof(T)));
   uint64_t* empty = full + NST;
   if (tid == 0) {
     for (int b = 0; b < NST; ++b) {
       mbar_init(&full[b], 1);
       mbar_init(&empty[b], 1);
     }
-    xw[XW] = T(0);
+    ((T*)xw_p)[XW] = T(0);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  auto base_of = [&](int b) { return smem + (size_t)b * sbytes; };
 
-  if (tid >= NC) {  // ---------------- producer warp
+  if (tid >= NC) {  // ---------------- producer warp: stage loads and x stores
     if (tid == NC) {
+      for (int s = 0; s < nstage && s < NST; ++s) {
+        unsigned char* B = smem + (size_t)s * sbytes;
+        const EllRec R = recs[2 * s];
+        Win wb = win(bw, (int64_t)r0 + R.sa, R.sb - R.sa);
+        mbar_expect_tx(&full[s], 64 + R.bytes + wb.bytes);
+        tma_bulk_g2s(B, recs + 2 * s, 64, &full[s]);
+        tma_bulk_g2s(B + 64, ell + (size_t)R.off16 * 16, R.bytes, &full[s]);
+        tma_bulk_g2s(B + o_b, wb.src, wb.bytes, &full[s]);
+      }
       int b = 0;
       uint32_t ph = 0;
       for (int s = 0; s < nstage; ++s) {
-        unsigned char* B = base_of(b);
-        EllRec R;
-        if (s < NST) {
-          R = recs[2 * s];
-        } else {
-          mbar_wait(&empty[b], ph ^ 1u);
-          R = ((const EllRec*)B)[1];
+        unsigned char* B = smem + (size_t)b * sbytes;
+        mbar_wait(&empty[b], ph);  // stage s solved (its window rows final)
+        const EllRec R = ((const EllRec*)B)[0];
+        // x rows [sa, sb) of the stage: window slots are contiguous (no wrap)
+        int g0 = r0 + R.sa, g1 = r0 + R.sb;
+        const T* xwT = (const T*)xw_p;
+        if (g0 & 1 && sizeof(T) == 8) {  // 16-byte alignment of the bulk copy
+          xs[g0] = xwT[(uint32_t)g0 & xmask];
+          ++g0;
         }
-        const int n = R.sb - R.sa;
-        const uint32_t blk_idx = al16(K * R.npad * 4), blk_val = al16(K * R.npad * (uint32_t)sizeof(T));
-        Win wb = win(bw, (int64_t)r0 + R.sa, n);
-        Win wl = win(lp, R.l0, R.nl);
-        uint32_t tot = 64 + blk_idx + blk_val + wb.bytes + wl.bytes;
-        mbar_expect_tx(&full[b], tot);
-        tma_bulk_g2s(B, recs + 2 * s, 64, &full[b]);
-        const char* src = ell + (size_t)R.off16 * 16;
-        tma_bulk_g2s(B + 64, src, blk_idx, &full[b]);
-        tma_bulk_g2s(B + 64 + cap_idx, src + blk_idx, blk_val, &full[b]);
-        tma_bulk_g2s(B + 64 + cap_idx + cap_val, wb.src, wb.bytes, &full[b]);
-        tma_bulk_g2s(B + 64 + cap_idx + cap_val + cap_b, wl.src, wl.bytes, &full[b]);
+        if (sizeof(T) == 4) {
+          while ((g0 & 3) && g0 < g1) {
+            xs[g0] = xwT[(uint32_t)g0 & xmask];
+            ++g0;
+          }
+        }
+        const int per16 = 16 / (int)sizeof(T);
+        int g1a = g0 + (g1 - g0) / per16 * per16;
+        for (int g = g1a; g < g1; ++g) xs[g] = xwT[(uint32_t)g & xmask];
+        if (g1a > g0) {
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          bulk_s2g(xs + g0, xw + (((uint32_t)g0 & xmask) << SH), (uint32_t)(g1a - g0) * sizeof(T));
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+        if (s + NST < nstage) {
+          // the stores must have read their window slots before the
+          // consumers can reach stage s + NST + 1 (which needs the load below)
+          asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+          const EllRec Rn = ((const EllRec*)B)[1];  // rode in with stage s
+          Win wb = win(bw, (int64_t)r0 + Rn.sa, Rn.sb - Rn.sa);
+          mbar_expect_tx(&full[b], 64 + Rn.bytes + wb.bytes);
+          tma_bulk_g2s(B, recs + 2 * (s + NST), 64, &full[b]);
+          tma_bulk_g2s(B + 64, ell + (size_t)Rn.off16 * 16, Rn.bytes, &full[b]);
+          tma_bulk_g2s(B + o_b, wb.src, wb.bytes, &full[b]);
+        }
         if (++b == NST) {
           b = 0;
           ph ^= 1u;
         }
       }
+      asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
     }
     return;
   }
 
+  // ---------------- consumer warps
   int b = 0;
   uint32_t ph = 0;
   for (int s = 0; s < nstage; ++s) {
@@ -836,68 +1108,59 @@ __global__ void __launch_bounds__(1024, 1)
       trace[3 * s] = t0;
       trace[3 * s + 1] = clock64();
     }
-    unsigned char* B = base_of(b);
+    const unsigned char* B = smem + (size_t)b * sbytes;
     const EllRec R = ((const EllRec*)B)[0];
+    // the stage block as copied: step records, slot words, values (packed
+    // to this stage's own nsteps / npad, not to the buffer capacity)
+    const int4* steps = (const int4*)(B + 64);
+    const uint32_t* src = (const uint32_t*)(B + 64 + 16 * R.nsteps);
+    const T* vv = (const T*)(B + 64 + 16 * R.nsteps + al16(W * R.npad * 4));
+    const T* sbw = (const T*)(B + o_b) + shift_of(bw, (int64_t)r0 + R.sa);
     const int npad = R.npad;
-    const int* s_idx = (const int*)(B + 64);
-    const T* s_val = (const T*)(B + 64 + cap_idx);
-    const T* s_b = (const T*)(B + 64 + cap_idx + cap_val) + shift_of(bw, (int64_t)r0 + R.sa);
-    const int* s_lp = (const int*)(B + 64 + cap_idx + cap_val + cap_b) + shift_of(lp, R.l0);
-    // Software pipeline across levels: this thread's rows of level li+1
-    // (rows la + tid + q*NC, q < RPT) -- their b, slots and values, none of
-    // which depend on x -- are loaded before the barrier that ends level li,
-    // so after it only ld.shared x -> DFMA -> store remains on the dependency
-    // chain.  Branch-free: a row slot past the level end loads row 0 of the
-    // stage and is neutralised (slot = the zero slot, value 0, b 0); only the
-    // stores are predicated.
-    const int nrow = R.sb - R.sa;
-    int la = max(s_lp[0], R.sa) - R.sa, lb = min(s_lp[1], R.sb) - R.sa;  // stage-local
-    T pb[RPT], pv[RPT][K];
-    int ps[RPT][K];
-    auto prefetch = [&](int la_, int lb_) {
+    const uint32_t gbase = (uint32_t)(r0 + R.sa);  // global row of stage row 0
+    T pb[RG], pv[RG][K];
+    uint32_t pa[RG][K], pd[RG];
+    bool pact[RG], pok[RG];
+    auto prefetch = [&](int q) {
+      const int4 st4 = steps[q];  // {first_group, ngroups, row_start, nrows}
 #pragma unroll
-      for (int q = 0; q < RPT; ++q) {
-        const int i = la_ + tid + q * NC;
-        const bool ok = i < lb_;
-        const int ic = ok ? i : 0;
-        pb[q] = ok ? s_b[ic] : T(0);
+      for (int g = 0; g < RG; ++g) {
+        const int gi = warp + g * NW;
+        pact[g] = gi < st4.y;
+        const int rl = gi * 32 + lane;
+        pok[g] = pact[g] && rl < st4.w;
+        const int idx = pact[g] ? (st4.x + gi) * 32 + lane : 0;
+        const int row = st4.z + (pok[g] ? rl : 0);  // stage-local row
+        pb[g] = pok[g] ? sbw[row] : T(0);
+        pd[g] = xw + (((gbase + (uint32_t)row) & xmask) << SH);
+        uint32_t wd[W];
 #pragma unroll
-        for (int k = 0; k < K; ++k) {
-          const int sl = s_idx[k * npad + ic];
-          const T v = s_val[k * npad + ic];
-          ps[q][k] = ok ? sl : XW;
-          pv[q][k] = ok ? v : T(0);
+        for (int w = 0; w < W; ++w) wd[w] = src[w * npad + idx];
+#pragma unroll
+        for (int k2 = 0; k2 < K; ++k2) {
+          const uint32_t sl = (k2 & 1) ? (wd[k2 >> 1] >> 16) : (wd[k2 >> 1] & 0xffffu);
+          pa[g][k2] = xw + (sl << SH);
+          pv[g][k2] = vv[k2 * npad + idx];
         }
       }
     };
-    prefetch(la, lb);
-    T* const xs_stage = xs + r0 + R.sa;
-    const int sa_mask = R.sa;  // row r = sa + i; window slot (sa + i) & xmask
-    for (int li = 0; li + 1 < R.nl; ++li) {
+    prefetch(0);
+    for (int q = 0; q < R.nsteps; ++q) {
 #pragma unroll
-      for (int q = 0; q < RPT; ++q) {  // operands already in registers
-        T acc = pb[q];
+      for (int g = 0; g < RG; ++g) {
+        if (pact[g]) {  // warp-uniform
+          T acc = pb[g];
 #pragma unroll
-        for (int k = 0; k < K; ++k) acc -= pv[q][k] * xw[ps[q][k]];
-        const int i = la + tid + q * NC;
-        if (i < lb) {
-          xw[(sa_mask + i) & xmask] = acc;
-          xs_stage[i] = acc;
+          for (int k2 = 0; k2 < K; ++k2) acc -= pv[g][k2] * lds_x(pa[g][k2], T(0));
+          if (pok[g]) sts_x(pd[g], acc);
         }
       }
-      if (lb - la > RPT * NC) {  // warp-uniform: a level wider than NC * RPT rows
-        for (int i = la + tid + RPT * NC; i < lb; i += NC) {
-          T a2 = s_b[i];
-#pragma unroll
-          for (int k = 0; k < K; ++k) a2 -= s_val[k * npad + i] * xw[s_idx[k * npad + i]];
-          xw[(sa_mask + i) & xmask] = a2;
-          xs_stage[i] = a2;
-        }
-      }
-      if (li + 2 < R.nl) {
-        la = max(s_lp[li + 1] - R.sa, 0);
-        lb = min(s_lp[li + 2] - R.sa, nrow);
-        prefetch(la, lb);
+      if (q + 1 < R.nsteps) {
+        prefetch(q + 1);
+      } else {
+        // the producer's bulk store reads this stage's window rows through
+        // the async proxy
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       }
       asm volatile("bar.sync 1, %0;" ::"r"(NC) : "memory");  // level barrier (Alg 2 L96)
     }
@@ -907,6 +1170,220 @@ __global__ void __launch_bounds__(1024, 1)
       b = 0;
       ph ^= 1u;
     }
+  }
+}
+
+// ------------------- K4' (B200): partitioned chain, shared-memory spin flags
+// The rows of a narrow-level triangle are split into P partitions by their
+// ORIGINAL row index (contiguous ranges).  L is lower in the original
+// numbering, so a row only depends on rows of its own or a LOWER partition:
+// the partitions form a pipeline, and partition q can run a few levels
+// behind partition q-1.  One CTA (one SM) per partition, claimed in order
+// through the segment ticket (a CTA only waits on partitions claimed before
+// it, so any CTA schedule makes progress).
+// Inside a CTA the partition's rows are processed in level order as groups
+// of 32 rows of one level (padded); group gi belongs to consumer warp
+// gi % NW.  There is no per-level barrier: a dependency computed by this CTA
+// is read from a shared-memory window slot (local position mod XW) whose
+// value is its own ready flag (sentinel until written; ld.volatile.shared
+// spin, ~30-cycle detection), a dependency of another partition (or one too
+// old for the window) is polled in global memory (value-as-flag, L2).  The
+// only barriers are at stage ends (TMA buffer ring + window slot recycling).
+// Stage block (TMA'd): int4 group records {first padded row, level, -, -}
+// are not needed -- groups are 32 padded rows in order -- so a stage is:
+//   grow[npad] (global permuted row, -1 = padding), words[K+1][npad]
+//   (k < K: bit 31 = global, low bits = global row; else window slot;
+//   k = K: the row's own window slot), vals[K][npad], then room for the
+//   gathered b'[npad].
+struct PipeRec {
+  int pos0, pos1, ngroups, off16, bytes, npad, pad0, pad1;  // real local positions [pos0,pos1)
+};
+
+template <typename T>
+__host__ __device__ inline uint32_t pipe_stage_bytes(int K, int GMAX) {
+  const uint32_t np = (uint32_t)GMAX * 32;
+  return 64 + al16(np * 4) + al16((uint32_t)(K + 1) * np * 4) + al16((uint32_t)K * np * (uint32_t)sizeof(T)) +
+         al16(np * (uint32_t)sizeof(T));  // + gathered b'
+}
+
+// offsets inside one stage block (packed to the stage's own npad)
+__host__ __device__ inline uint32_t pipe_off_words(int npad) { return 64 + al16((uint32_t)npad * 4); }
+__host__ __device__ inline uint32_t pipe_off_vals(int K, int npad) {
+  return pipe_off_words(npad) + al16((uint32_t)(K + 1) * npad * 4);
+}
+template <typename T>
+__host__ __device__ inline uint32_t pipe_off_b(int K, int npad) {
+  return pipe_off_vals(K, npad) + al16((uint32_t)K * npad * (uint32_t)sizeof(T));
+}
+
+__device__ __forceinline__ double lds_volatile(uint32_t a, double) {
+  double v;
+  asm volatile("ld.volatile.shared.f64 %0, [%1];" : "=d"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ float lds_volatile(uint32_t a, float) {
+  float v;
+  asm volatile("ld.volatile.shared.f32 %0, [%1];" : "=f"(v) : "r"(a) : "memory");
+  return v;
+}
+
+template <typename T, int K>
+__global__ void __launch_bounds__(1024, 1)
+    tri_chain_pipe(int nparts, const int* __restrict__ part_stage0, const PipeRec* __restrict__ recs,
+                   const char* __restrict__ data, const T* __restrict__ bw, T* __restrict__ xs, int NST, int GMAX,
+                   int XW, SolveState st, int slot) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  constexpr uint32_t SH = sizeof(T) == 8 ? 3 : 2;
+  const int tid = threadIdx.x;
+  const int NC = blockDim.x - 32;
+  const int NW = NC >> 5, warp = tid >> 5, lane = tid & 31;
+  const uint32_t xmask = (uint32_t)XW - 1;
+  const uint32_t sbytes = pipe_stage_bytes<T>(K, GMAX);
+  unsigned char* xw_p = smem + (size_t)NST * sbytes;
+  const uint32_t xw = smem_addr(xw_p);
+  uint64_t* full = (uint64_t*)(xw_p + al16((XW + 2) * (uint32_t)sizeof(T)));
+  uint64_t* empty = full + NST;
+  __shared__ int s_part;
+  if (tid == 0) {
+    s_part = (int)atomicAdd(st.tickets + slot, 1u);
+    for (int b = 0; b < NST; ++b) {
+      mbar_init(&full[b], 1);
+      mbar_init(&empty[b], 1);
+    }
+    ((T*)xw_p)[XW] = T(0);  // the zero slot of padding rows
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  // all window slots start as the sentinel
+  for (int i = tid; i < XW; i += blockDim.x) ((T*)xw_p)[i] = sent<T>();
+  __syncthreads();
+  const int part = s_part;
+  if (part >= nparts) return;
+  const int s0 = part_stage0[part], nstage = part_stage0[part + 1] - s0;
+
+  if (tid >= NC) {  // ---------------- producer warp: stage loads
+    if (tid == NC) {
+      int b = 0;
+      uint32_t ph = 0;
+      for (int s = 0; s < nstage; ++s) {
+        unsigned char* B = smem + (size_t)b * sbytes;
+        if (s >= NST) mbar_wait(&empty[b], ph ^ 1u);
+        const PipeRec R = recs[2 * (s0 + s)];
+        mbar_expect_tx(&full[b], 64 + R.bytes);
+        tma_bulk_g2s(B, recs + 2 * (s0 + s), 64, &full[b]);
+        tma_bulk_g2s(B + 64, data + (size_t)R.off16 * 16, R.bytes, &full[b]);
+        if (++b == NST) {
+          b = 0;
+          ph ^= 1u;
+        }
+      }
+    }
+    return;
+  }
+
+  // ---------------- consumer warps
+  uint32_t spins = 0;
+  int b = 0;
+  uint32_t ph = 0;
+  // b' of the NEXT stage's rows is gathered from global memory during the
+  // current stage (8 per thread in flight) and parked in its stage buffer
+  constexpr int BG = 8;
+  T bnext[BG];
+  auto gather_issue = [&](const unsigned char* B) {
+    const PipeRec R = ((const PipeRec*)B)[0];
+    const int* grow = (const int*)(B + 64);
+#pragma unroll
+    for (int u = 0; u < BG; ++u) {
+      const int i = tid + u * NC;
+      const int g = i < R.npad ? grow[i] : -1;
+      bnext[u] = g >= 0 ? ldg_nc(bw + g) : T(0);
+    }
+  };
+  auto gather_park = [&](unsigned char* B) {
+    const PipeRec R = ((const PipeRec*)B)[0];
+    T* sb = (T*)(B + pipe_off_b<T>(K, R.npad));
+#pragma unroll
+    for (int u = 0; u < BG; ++u) {
+      const int i = tid + u * NC;
+      if (i < R.npad) sb[i] = bnext[u];
+    }
+    for (int i = tid + BG * NC; i < R.npad; i += NC) {  // rare: more rows than BG * NC
+      const int g = ((const int*)(B + 64))[i];
+      sb[i] = g >= 0 ? ldg_nc(bw + g) : T(0);
+    }
+  };
+  if (nstage > 0) {
+    mbar_wait(&full[0], 0);
+    gather_issue(smem);
+    gather_park(smem);
+  }
+  asm volatile("bar.sync 1, %0;" ::"r"(NC) : "memory");
+  for (int s = 0; s < nstage; ++s) {
+    unsigned char* B = smem + (size_t)b * sbytes;
+    const PipeRec R = ((const PipeRec*)B)[0];
+    const int nb = b + 1 == NST ? 0 : b + 1;
+    const uint32_t nph = b + 1 == NST ? ph ^ 1u : ph;
+    unsigned char* Bn = smem + (size_t)nb * sbytes;
+    const bool has_next = s + 1 < nstage;
+    if (has_next) {
+      mbar_wait(&full[nb], nph);  // TMA runs ahead; normally already complete
+      gather_issue(Bn);
+      // recycle the window slots of the next stage's rows: their previous
+      // occupants (XW positions back) have no readers left (analysis bound)
+      const PipeRec Rn = ((const PipeRec*)Bn)[0];
+      for (int q = Rn.pos0 + tid; q < Rn.pos1; q += NC) ((T*)xw_p)[(uint32_t)q & xmask] = sent<T>();
+    }
+    const int npad = R.npad;
+    const int* grow = (const int*)(B + 64);
+    const uint32_t* words = (const uint32_t*)(B + pipe_off_words(npad));
+    const T* vals = (const T*)(B + pipe_off_vals(K, npad));
+    const T* sb = (const T*)(B + pipe_off_b<T>(K, npad));
+    for (int gi = warp; gi < R.ngroups; gi += NW) {
+      const int i = gi * 32 + lane;
+      const int g = grow[i];
+      T acc = sb[i];
+      uint32_t wd[K];
+      T v[K];
+#pragma unroll
+      for (int k2 = 0; k2 < K; ++k2) {
+        wd[k2] = words[k2 * npad + i];
+        v[k2] = vals[k2 * npad + i];
+      }
+#pragma unroll
+      for (int k2 = 0; k2 < K; ++k2) {
+        T x;
+        if (wd[k2] & 0x80000000u) {
+          const T* px = xs + (wd[k2] & 0x7fffffffu);
+          x = ld_strong(px);
+          while (is_sent(x)) {
+            if (++spins > kWatchdogSpins) {
+              watchdog_trip(st);
+              break;
+            }
+            x = ld_strong(px);
+          }
+        } else {
+          const uint32_t a = xw + (wd[k2] << SH);
+          x = lds_volatile(a, T(0));
+          while (is_sent(x)) {
+            if (++spins > kWatchdogSpins) {
+              watchdog_trip(st);
+              break;
+            }
+            x = lds_volatile(a, T(0));
+          }
+        }
+        acc -= v[k2] * x;
+      }
+      if (g >= 0) {
+        sts_x(xw + (words[K * npad + i] << SH), acc);  // word K: this row's window slot
+        st_strong(xs + g, acc);
+      }
+    }
+    if (has_next) gather_park(Bn);
+    asm volatile("bar.sync 1, %0;" ::"r"(NC) : "memory");  // stage end: slots recycled, buffer free
+    if (tid == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(&empty[b])) : "memory");
+    b = nb;
+    ph = nph;
   }
 }
 

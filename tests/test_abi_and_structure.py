@@ -39,6 +39,7 @@ def test_exports_every_declared_symbol():
 
 def _analyse(M, **kw):
     kw.setdefault("host_only", True)
+    kw.setdefault("reorder", True)  # the paper's level-set reordering (L231); "auto" is tested below
     kw.setdefault("min_block_rows", B200_T)
     return sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, fill=M.uplo, **kw)
 
@@ -168,3 +169,29 @@ def test_host_only_plan_refuses_solve():
     with pytest.raises(sp.SptrsvError) as e:
         plan.solve(np.ones(4))
     assert e.value.status_name == "NOT_SUPPORTED"
+
+
+@pytest.mark.parametrize("name,expect_none", [("C1", False), ("C2", False), ("C3", False), ("C4", True),
+                                              ("C5", False)])
+def test_reorder_auto_keeps_supernodal_inputs(name, expect_none):
+    """reorder="auto" (R29) skips the level sort only for supernodal
+    inputs; whatever it picks, the structure equals the oracle's for that
+    choice."""
+    M, _ = g.gen_config(name, small=True)
+    plan = _analyse(M, depth=2, reorder="auto")
+    eff_none = plan.info()["reorder"] == 1
+    assert eff_none == expect_none
+    _compare(M, plan, st.analyse(M, depth=2, reorder=not eff_none))
+
+
+def test_supernode_pieces_cover_dense_blocks():
+    """The supernodal selector only fires on triangles made of dense diagonal
+    blocks: the C4 factor (64-wide supernodes -> 32-row pieces), the dense
+    lower triangle; never on a bidiagonal chain (its diagonal blocks are not
+    dense) or on C2/C3."""
+    for M, want in [(g.gen_config("C4", small=True)[0], True), (g.shape_dense_lower(150), True),
+                    (g.shape_bidiagonal(3000), False), (g.gen_config("C2", small=True)[0], False),
+                    (g.gen_config("C3", small=True)[0], False)]:
+        plan = _analyse(M, depth=0, reorder="auto")
+        seg = plan.segments()[0]
+        assert (seg["impl"] == "TRI_SUPERNODE") == want, (M.name, seg["impl"])

@@ -58,13 +58,13 @@ def test_small_configs_default(gpu, name, selector):
 
 
 @pytest.mark.parametrize("name", CONFIGS)
-@pytest.mark.parametrize("tri", ["TRI_LEVELSET", "TRI_SYNCFREE", "TRI_CHAIN"])
+@pytest.mark.parametrize("tri", ["TRI_LEVELSET", "TRI_SYNCFREE", "TRI_CHAIN", "TRI_SUPERNODE", "TRI_PIPE"])
 @pytest.mark.parametrize("sq", ["SQ_SCALAR", "SQ_VECTOR"])
 def test_forced_kernels(gpu, name, tri, sq):
     M, b = g.gen_config(name, small=True, nrhs=1)
     if tri == "TRI_LEVELSET" and name in ("C2",):
         pytest.skip("thousands of per-level launches; covered by C1/C3-C5")
-    x, plan = _solve(M, b, depth=2, force_tri_impl=tri, force_sq_impl=sq)
+    x, plan = _solve(M, b, depth=2, force_tri_impl=tri, force_sq_impl=sq, reorder=True)
     assert all(s["impl"] == tri for s in plan.segments() if s["kind"] == "TRI" and s["nlevels"] > 1)
     _check64(M, b, x)
 
@@ -79,12 +79,35 @@ def test_variants(gpu, name, variant):
 
 @pytest.mark.parametrize("name", CONFIGS)
 @pytest.mark.parametrize("nrhs", [2, 7, 33, 70])
-@pytest.mark.parametrize("tri", ["TRI_LEVELSET", "TRI_SYNCFREE", "TRI_CHAIN"])
+@pytest.mark.parametrize("tri", ["TRI_LEVELSET", "TRI_SYNCFREE", "TRI_CHAIN", "TRI_SUPERNODE", "TRI_PIPE"])
 def test_multi_rhs(gpu, name, nrhs, tri):
     if tri == "TRI_LEVELSET" and name == "C2":
         pytest.skip("per-level launches")
     M, b = g.gen_config(name, small=True, nrhs=nrhs)
-    x, _ = _solve(M, b, depth=2, force_tri_impl=tri)
+    x, _ = _solve(M, b, depth=2, force_tri_impl=tri, reorder=True)
+    _check64(M, b, x)
+
+
+@pytest.mark.parametrize("tri", ["TRI_LEVELSET", "TRI_CHAIN", "TRI_SYNCFREE", "TRI_SUPERNODE", "TRI_PIPE"])
+def test_no_reorder_never_walks_levels(gpu, tri):
+    """Without the level-set reordering, levels are not contiguous row
+    ranges: a forced level-set / chain kernel falls back to sync-free."""
+    M, b = g.gen_config("C3", small=True, nrhs=1)
+    x, plan = _solve(M, b, depth=2, force_tri_impl=tri, reorder=False)
+    assert all(s["impl"] in ("TRI_SYNCFREE", "TRI_SUPERNODE", "TRI_DIAG") for s in plan.segments()
+               if s["kind"] == "TRI")
+    _check64(M, b, x)
+
+
+@pytest.mark.parametrize("name", ["C4", "C1"])
+@pytest.mark.parametrize("reorder", ["auto", True, False])
+def test_supernodal_default_and_reorders(gpu, name, reorder):
+    """C4 (supernodal) under the B200 default picks reorder=none + the
+    supernodal kernel; every reorder choice solves to the oracle."""
+    M, b = g.gen_config(name, small=True, nrhs=1)
+    x, plan = _solve(M, b, depth=1, reorder=reorder)
+    if name == "C4" and reorder != True:  # noqa: E712
+        assert any(s["impl"] == "TRI_SUPERNODE" for s in plan.segments())
     _check64(M, b, x)
 
 
@@ -186,8 +209,9 @@ def test_full_size_configs(gpu, name):
     M, b = g.gen_config(name, nrhs=1)
     x, plan = _solve(M, b)
     err = _check64(M, b, x)
-    # the plan's structure at full size is the oracle's
-    A = st.analyse(M, min_block_rows=B200_T)
+    # the plan's structure at full size is the oracle's (for the reorder the
+    # B200 default chose: none for the supernodal C4, level otherwise, R29)
+    A = st.analyse(M, min_block_rows=B200_T, reorder=plan.info()["reorder"] == 0)
     segs = plan.segments()
     assert [(s["row0"], s["row1"], s["col0"], s["col1"], s["nnz"], s["nlevels"], s["kernel"])
             for s in segs] == [(o.row0, o.row1, o.col0, o.col1, o.nnz, o.nlevels, o.kernel) for o in A.segs]
@@ -208,3 +232,14 @@ def test_full_size_c5_multi_rhs_sampled(gpu):
     assert on.rel_err(xs, ref) <= TOL64
     ok, worst = on.residual_bound_ok(M, xs, b[cols])
     assert ok, worst
+
+
+@pytest.mark.parametrize("P", ["1", "3", "8"])
+def test_pipe_partitions(gpu, P, monkeypatch):
+    """The partitioned pipeline chain at several partition counts (each
+    partition one CTA; cross-partition dependencies polled in L2)."""
+    monkeypatch.setenv("SPTRSV_PIPE_P", P)
+    for name in ("C2", "C1"):
+        M, b = g.gen_config(name, small=True, nrhs=1)
+        x, plan = _solve(M, b, depth=1, force_tri_impl="TRI_PIPE", reorder=True)
+        _check64(M, b, x)
