@@ -82,9 +82,11 @@ typedef enum {
   SPTRSV_IMPL_SQ_VECTOR = 5,     /* K6/K8: warp per row, CSR or DCSR                                */
   SPTRSV_IMPL_TRI_SUPERNODE = 6, /* B200: warp per fundamental supernode (<= 32 rows): dense GEMV of its
                                     shared external columns + register-resident dense triangle     */
-  SPTRSV_IMPL_TRI_PIPE = 7       /* B200: narrow-level triangle split by original row index over P CTAs
-                                    (a pipeline); shared-memory spin flags inside a CTA, no per-level
-                                    barrier; cross-CTA dependencies polled in L2                     */
+  SPTRSV_IMPL_TRI_PIPE = 7       /* B200: strand wavefront -- narrow-level triangle split by original row
+                                    index into C x W strands (one warp each, one thread-block cluster);
+                                    no level barrier; cross-strand x pushed into the consumer's shared
+                                    memory (DSMEM).  Replaced by TRI_CHAIN at upload when a row has > 8
+                                    dependencies (or > 10% would be polled in global memory)          */
 } sptrsv_impl_t;
 
 /* Which kernel implements each Alg 7 label. PAPER maps labels 1:1 onto the

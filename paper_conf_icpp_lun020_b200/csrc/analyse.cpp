@@ -506,12 +506,13 @@ void choose_impls(Plan& p) {
         // narrow levels: one CTA walks the level chain with bar.sync (no
         // cross-SM flag round trips); wide levels: all SMs
         if (I.max_level_rows <= 2048 || (m / std::max(1, I.nlevels)) <= 256) {
-          // narrow levels: one SM per partition walks the level chain at
-          // shared-memory latency (pipeline of P CTAs for big triangles with
-          // <= 4 dependencies per row, one CTA otherwise)
+          // narrow levels with few dependencies per row: the strand
+          // wavefront over one thread-block cluster (exec.cu build_wave, which
+          // falls back to the single-CTA chain when the rows' dependencies
+          // do not stay inside their strands); else one CTA walks the chain
           int32_t kmax = 0;
           for (int64_t r = 0; r < m; ++r) kmax = std::max(kmax, S.in_degree[r]);
-          impl = (kmax >= 1 && kmax <= 4 && m >= 4096 && std::getenv("SPTRSV_NO_PIPE") == nullptr)
+          impl = (kmax >= 1 && kmax <= 8 && m >= 4096 && std::getenv("SPTRSV_NO_WAVE") == nullptr)
                      ? SPTRSV_IMPL_TRI_PIPE
                      : SPTRSV_IMPL_TRI_CHAIN;
         }

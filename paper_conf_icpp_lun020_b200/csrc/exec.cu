@@ -8,6 +8,8 @@
 #include <cstdlib>
 #include <cstring>
 #include <string>
+#include <unordered_map>
+#include <array>
 
 #include "internal.h"
 #include "kernels.cuh"
@@ -386,139 +388,291 @@ void build_supernodes(Segment& S, size_t vb) {
   std::memcpy(S.sn_desc.data(), desc.data(), S.sn_desc.size());
 }
 
-// Partitioned pipeline chain (see k::tri_chain_pipe).  Partitions are
-// contiguous ranges of the ORIGINAL (lower) row index, balanced in rows; a
-// partition's rows keep the triangle's level order; groups are 32 rows of
-// one level; stages are GMAX consecutive groups.
-void build_pipeline(const Plan& p, Segment& S, size_t vb) {
-  S.pipe_P = 0;
-  S.pipe_K = 0;
-  S.pipe_recs.clear();
-  S.pipe_data.clear();
-  S.pipe_stage0.clear();
-  const auto& I = S.info;
+// Strand wavefront (k::tri_wave): strands = contiguous ranges of the
+// ORIGINAL (lower) row index balanced in rows, C CTAs (one cluster) x W warps;
+// groups = <= 32 rows of one level of a strand; the device row order of the
+// triangle becomes strand-major, group-major (wave_tau).  Leaves wave_K == 0
+// and switches the segment to the chain kernel when the triangle does not
+// suit it (a row with > 8 dependencies, or > 10% of the dependencies would
+// have to be polled in global memory).
+void build_wave(const Plan& p, Segment& S, size_t vb) {
+  S.wave_K = 0;
+  S.wave_tau.clear();
+  S.wave_strands.clear();
+  S.wave_data.clear();
+  auto& I = S.info;
   if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_PIPE) return;
   const int m = I.row1 - I.row0;
+  int C = 8, W = 4, GPC = 8, NCH = 4;
+  if (const char* e = std::getenv("SPTRSV_WAVE")) {
+    int a, b2, c, d;
+    if (std::sscanf(e, "%d,%d,%d,%d", &a, &b2, &c, &d) == 4 && a >= 1 && a <= 16 && b2 >= 1 && b2 <= 8 &&
+        c >= 1 && c <= 32 && d >= 2 && d <= 4) {
+      C = a; W = b2; GPC = c; NCH = d;
+    }
+  }
+  auto give_up = [&]() {
+    S.wave_K = 0;
+    S.wave_tau.clear();
+    I.impl = SPTRSV_IMPL_TRI_CHAIN;
+  };
   int K = 0;
   for (int r = 0; r < m; ++r) K = std::max(K, S.rp[r + 1] - S.rp[r]);
-  if (K < 1 || K > 4 || m < 1) return;  // the launcher falls back to the chain kernel
-  const int XW = 8192, NST = 3, GMAX = K <= 2 ? 32 : 16;
-  const int RM = GMAX * 32;
-  int P = (int)std::max<int64_t>(1, std::min<int64_t>(p.sm_count / 2, m / 32768));
-  if (const char* e = std::getenv("SPTRSV_PIPE_P")) P = std::max(1, std::min(p.sm_count, std::atoi(e)));
-  // partition by rank of the original (lower) row index
-  std::vector<int32_t> order(m), part(m), pos(m);
+  if (m < 1 || K < 1 || K > 8) return give_up();
+  const int Kt = K <= 1 ? 1 : K <= 2 ? 2 : K <= 4 ? 4 : 8;
+  while (C > 1 && (int64_t)C * W * 256 > m) --C;  // at least ~256 rows per strand
+  const int NS = C * W;
+  // strands by rank of the original row index
+  std::vector<int32_t> order(m), strand(m);
   std::iota(order.begin(), order.end(), 0);
-  std::sort(order.begin(), order.end(),
-            [&](int a, int b) { return p.lower_old[I.row0 + a] < p.lower_old[I.row0 + b]; });
-  for (int q = 0; q < m; ++q) part[order[q]] = (int)((int64_t)q * P / m);
-  std::vector<std::vector<int32_t>> rows(P);
-  for (int r = 0; r < m; ++r) {
-    pos[r] = (int32_t)rows[part[r]].size();
-    rows[part[r]].push_back(r);
-  }
-  const uint32_t mask = (uint32_t)XW - 1;
-  S.pipe_stage0.push_back(0);
-  std::vector<std::pair<std::vector<int32_t>, int>> stage_rows;  // padded rows (-1 = pad), pos0
-  int g90src = 0;
-  std::vector<int> gpl;  // groups per (partition, level)
-  for (int q = 0; q < P; ++q) {
-    const auto& R = rows[q];
-    // groups: runs of one level, chunks of 32
-    std::vector<std::vector<int32_t>> groups;
+  std::stable_sort(order.begin(), order.end(),
+                   [&](int a, int b2) { return p.lower_old[I.row0 + a] < p.lower_old[I.row0 + b2]; });
+  for (int q = 0; q < m; ++q) strand[order[q]] = (int)((int64_t)q * NS / m);
+  // rows of every strand in level order (= local row order); groups
+  std::vector<std::vector<int32_t>> srows(NS);
+  for (int r = 0; r < m; ++r) srows[strand[r]].push_back(r);
+  std::vector<int32_t> pos(m), qpos(m), s_start(NS + 1, 0);
+  std::vector<std::vector<std::pair<int32_t, int32_t>>> groups(NS);  // (first pos, count) per strand
+  int q = 0;
+  for (int s2 = 0; s2 < NS; ++s2) {
+    s_start[s2] = q;
+    const auto& R = srows[s2];
     for (size_t a = 0; a < R.size();) {
       const int lv = p.leaf_level[I.row0 + R[a]];
-      size_t b = a;
-      while (b < R.size() && p.leaf_level[I.row0 + R[b]] == lv) ++b;
-      gpl.push_back((int)((b - a + 31) / 32));
-      for (size_t c = a; c < b; c += 32) {
-        std::vector<int32_t> gr(32, -1);
-        for (size_t d = c; d < std::min(b, c + 32); ++d) gr[d - c] = R[d];
-        groups.push_back(gr);
-      }
-      a = b;
+      size_t b2 = a;
+      while (b2 < R.size() && b2 - a < 32 && p.leaf_level[I.row0 + R[b2]] == lv) ++b2;
+      groups[s2].push_back({(int32_t)a, (int32_t)(b2 - a)});
+      a = b2;
     }
-    for (size_t g0 = 0; g0 < groups.size(); g0 += GMAX) {
-      std::vector<int32_t> pr;
-      int pos0 = -1;
-      for (size_t g = g0; g < std::min(groups.size(), g0 + GMAX); ++g)
-        for (int r : groups[g]) {
-          pr.push_back(r);
-          if (r >= 0 && pos0 < 0) pos0 = pos[r];
+    for (size_t a = 0; a < R.size(); ++a) {
+      pos[R[a]] = (int32_t)a;
+      qpos[R[a]] = q++;
+    }
+  }
+  s_start[NS] = q;
+  // own window: the smallest power of two covering every same-strand distance
+  int maxd = 0;
+  for (int r = 0; r < m; ++r)
+    for (int e = S.rp[r]; e < S.rp[r + 1]; ++e) {
+      const int j = S.ci[e] - I.row0;
+      if (strand[j] == strand[r]) maxd = std::max(maxd, pos[r] - pos[j]);
+    }
+  int xw_cap = 4096;  // SPTRSV_WAVE_XW / SPTRSV_WAVE_ICAP: test hooks forcing the global-memory fallback
+  if (const char* e = std::getenv("SPTRSV_WAVE_XW")) xw_cap = std::max(64, std::min(4096, std::atoi(e)));
+  int XW = 64;
+  while (XW < maxd + 32 && XW < xw_cap) XW *= 2;
+  // shared-memory budget (E = 2 is the upper bound of the chunk size): the
+  // deepest ring (GPC x NCH) that leaves >= 1024 import slots per strand
+  const uint32_t gb2 = vb == 8 ? k::wave_group_bytes<double>(Kt, 2) : k::wave_group_bytes<float>(Kt, 2);
+  uint32_t bring = 0;
+  int64_t icap = -1;
+  for (;;) {
+    bring = vb == 8 ? k::wave_bring_bytes<double>(GPC) : k::wave_bring_bytes<float>(GPC);
+    const int64_t rings = (int64_t)W * NCH * (k::wave_hdr_bytes(GPC) + (int64_t)GPC * gb2 + bring + 8);
+    const int64_t slots_avail = (232448 - 512 - rings) / (int64_t)vb;
+    icap = (slots_avail - 2) / W - XW;
+    if (icap >= 1024 || (GPC == 1 && NCH == 2)) break;
+    if (NCH > 2) --NCH;
+    else { GPC = std::max(1, GPC / 2); NCH = 4; }
+  }
+  if (const char* e = std::getenv("SPTRSV_WAVE_ICAP")) icap = std::min<int64_t>(icap, std::max(0, std::atoi(e)));
+  if (icap < 0) return give_up();
+  // classify every dependency (rows in execution order so imports are
+  // numbered in first-use order): kind 0 own, 1 import (strand, idx), 2 global
+  struct Dep { int8_t kind; int32_t a, b; };
+  std::vector<Dep> dep(S.ci.size());
+  std::vector<int32_t> nimp(NS, 0);
+  std::vector<uint8_t> npush(m, 0);
+  std::vector<std::array<int32_t, 4>> push(m, {-1, -1, -1, -1});  // (strand, idx) x 2
+  std::unordered_map<int64_t, int32_t> imp;
+  int64_t nglobal = 0;
+  for (int s2 = 0; s2 < NS; ++s2)
+    for (int r : srows[s2])
+      for (int e = S.rp[r]; e < S.rp[r + 1]; ++e) {
+        const int j = S.ci[e] - I.row0;
+        if (strand[j] == s2 && pos[r] - pos[j] <= XW - 32) {
+          dep[e] = {0, j, 0};
+          continue;
         }
-      stage_rows.push_back({pr, pos0});
+        if (strand[j] != s2) {
+          const int64_t key = (int64_t)s2 * m + j;
+          auto it = imp.find(key);
+          if (it != imp.end()) {
+            dep[e] = {1, s2, it->second};
+            continue;
+          }
+          if (npush[j] < 2 && nimp[s2] < icap) {
+            const int idx = nimp[s2]++;
+            imp.emplace(key, idx);
+            push[j][2 * npush[j]] = s2;
+            push[j][2 * npush[j] + 1] = idx;
+            ++npush[j];
+            dep[e] = {1, s2, idx};
+            continue;
+          }
+        }
+        dep[e] = {2, j, 0};
+        ++nglobal;
+      }
+  if (nglobal * 10 > (int64_t)S.ci.size() && p.opts.force_tri_impl != SPTRSV_IMPL_TRI_PIPE) return give_up();
+  int E = 0;
+  for (int r = 0; r < m; ++r) E = std::max<int>(E, npush[r]);
+  // x-area layout per CTA: slots 0-1 zero, then per warp own window + imports
+  std::vector<int32_t> own_base(NS), imp_base(NS);
+  int xa = 2;
+  for (int c = 0; c < C; ++c) {
+    int cur = 2;
+    for (int w = 0; w < W; ++w) {
+      const int s2 = c * W + w;
+      own_base[s2] = cur;
+      cur += XW;
+      imp_base[s2] = cur;
+      cur += nimp[s2];
     }
-    S.pipe_stage0.push_back((int32_t)stage_rows.size());
+    xa = std::max(xa, cur);
   }
-  (void)g90src;
-  const int ns = (int)stage_rows.size();
-  S.pipe_recs.assign((size_t)ns * 16, 0);
-  std::vector<size_t> offs(ns);
+  const uint32_t gbytes = vb == 8 ? k::wave_group_bytes<double>(Kt, E) : k::wave_group_bytes<float>(Kt, E);
+  const uint32_t hbytes = k::wave_hdr_bytes(GPC);
+  const uint32_t cbytes = hbytes + (uint32_t)GPC * gbytes;
+  // chunks
+  std::vector<k::WaveStrand> sr(NS);
+  std::vector<int32_t> nchunk(NS);
+  size_t total = 0;
+  for (int s2 = 0; s2 < NS; ++s2) {
+    nchunk[s2] = (int)((groups[s2].size() + GPC - 1) / GPC);
+    total += (size_t)nchunk[s2] * cbytes;
+  }
+  S.wave_data.assign(std::max<size_t>(total, 16), 0);
   size_t off = 0;
-  for (int t = 0; t < ns; ++t) {
-    const int npad = (int)stage_rows[t].first.size();
-    offs[t] = off;
-    off += vb == 8 ? k::pipe_off_b<double>(K, npad) - 64 : k::pipe_off_b<float>(K, npad) - 64;
-  }
-  S.pipe_data.assign(std::max<size_t>(off, 16), 0);
-  for (int t = 0; t < ns; ++t) {
-    const auto& pr = stage_rows[t].first;
-    const int npad = (int)pr.size();
-    char* blk = &S.pipe_data[offs[t]];  // == stage buffer + 64
-    int32_t* grow = (int32_t*)blk;
-    uint32_t* words = (uint32_t*)(blk + k::pipe_off_words(npad) - 64);
-    char* vals = blk + k::pipe_off_vals(K, npad) - 64;
-    int pos1 = stage_rows[t].second;
-    for (int i = 0; i < npad; ++i) {
-      const int r = pr[i];
-      for (int k2 = 0; k2 <= K; ++k2) words[(size_t)k2 * npad + i] = (uint32_t)XW;  // zero slot
-      if (r < 0) {
-        grow[i] = -1;
-        continue;
-      }
-      grow[i] = I.row0 + r;
-      pos1 = std::max(pos1, pos[r] + 1);
-      words[(size_t)K * npad + i] = (uint32_t)pos[r] & mask;
-      int kk = 0;
-      for (int q = S.rp[r]; q < S.rp[r + 1]; ++q, ++kk) {
-        const int j = S.ci[q] - I.row0;  // local row of the dependency
-        const bool local = part[j] == part[r] && pos[r] - pos[j] <= XW - 2 * RM;
-        words[(size_t)kk * npad + i] = local ? ((uint32_t)pos[j] & mask) : (0x80000000u | (uint32_t)S.ci[q]);
-        std::memcpy(vals + ((size_t)kk * npad + i) * vb, &S.val[(size_t)q * vb], vb);
+  const int r0 = I.row0;
+  auto word = [&](int e) -> uint32_t {
+    const Dep& d = dep[e];
+    if (d.kind == 0) return (uint32_t)(own_base[strand[d.a]] + (pos[d.a] & (XW - 1)));
+    if (d.kind == 1) return k::kWaveIMP | (uint32_t)(imp_base[d.a] + d.b);
+    return k::kWaveGLB | (uint32_t)(r0 + qpos[d.a]);
+  };
+  for (int s2 = 0; s2 < NS; ++s2) {
+    k::WaveStrand& W2 = sr[s2];
+    std::memset(&W2, 0, sizeof(W2));
+    W2.off16 = (int)(off / 16);
+    W2.nchunk = nchunk[s2];
+    W2.ngroups = (int)groups[s2].size();
+    W2.own_base = own_base[s2];
+    W2.row0 = r0 + s_start[s2];
+    const auto& Gs = groups[s2];
+    const auto& R = srows[s2];
+    auto chunk_rows = [&](int c, int& lo, int& hi) {
+      const int g0 = c * GPC, g1 = std::min<int>((int)Gs.size(), g0 + GPC) - 1;
+      lo = r0 + s_start[s2] + Gs[g0].first;
+      hi = r0 + s_start[s2] + Gs[g1].first + Gs[g1].second;
+    };
+    for (int c = 0; c < nchunk[s2]; ++c) {
+      char* B = &S.wave_data[off + (size_t)c * cbytes];
+      int32_t* hdr = (int32_t*)B;
+      chunk_rows(c, hdr[0], hdr[1]);
+      if (c + NCH < nchunk[s2]) chunk_rows(c + NCH, hdr[2], hdr[3]);
+      if (c < 4) chunk_rows(c, W2.lo[c], W2.hi[c]);
+      for (int gi = 0; gi < GPC; ++gi) {
+        const int g = c * GPC + gi;
+        int32_t* gh = (int32_t*)(B + 16) + 2 * gi;
+        uint32_t* wd = (uint32_t*)(B + hbytes + (size_t)gi * gbytes);
+        uint32_t* pw = wd + 32 * Kt;
+        char* vv = (char*)(pw + 32 * E);
+        for (int l = 0; l < 32 * E; ++l) pw[l] = 0xffffffffu;
+        if (g >= (int)Gs.size()) continue;  // padding group (cnt 0, zero slots)
+        int flags = 0;
+        gh[0] = r0 + s_start[s2] + Gs[g].first;
+        for (int l = 0; l < Gs[g].second; ++l) {
+          const int r = R[Gs[g].first + l];
+          int kk = 0;
+          for (int e = S.rp[r]; e < S.rp[r + 1]; ++e, ++kk) {
+            wd[kk * 32 + l] = word(e);
+            if (dep[e].kind == 2) flags |= k::kWaveGF_GLOBAL;
+            std::memcpy(vv + ((size_t)kk * 32 + l) * vb, &S.val[(size_t)e * vb], vb);
+          }
+          for (int e2 = 0; e2 < npush[r]; ++e2) {
+            const int cs = push[r][2 * e2], ci2 = push[r][2 * e2 + 1];
+            pw[e2 * 32 + l] = ((uint32_t)(cs / W) << 24) | (uint32_t)(imp_base[cs] + ci2);
+            flags |= k::kWaveGF_PUSH;
+          }
+        }
+        gh[1] = Gs[g].second | flags;
       }
     }
-    int32_t* R = &S.pipe_recs[(size_t)t * 16];
-    const size_t bytes = vb == 8 ? k::pipe_off_b<double>(K, npad) - 64 : k::pipe_off_b<float>(K, npad) - 64;
-    R[0] = stage_rows[t].second; R[1] = pos1; R[2] = npad / 32; R[3] = (int32_t)(offs[t] / 16);
-    R[4] = (int32_t)bytes; R[5] = npad;
+    off += (size_t)nchunk[s2] * cbytes;
   }
-  // consumer warps: twice the typical groups per level (warps on level l+1
-  // wait on level l through the shared-memory flags: a pipeline, not a barrier)
-  std::nth_element(gpl.begin(), gpl.begin() + gpl.size() * 9 / 10, gpl.end());
-  const int g90 = gpl.empty() ? 1 : gpl[gpl.size() * 9 / 10];
-  int nw = std::max(4, std::min(16, 2 * g90));
-  if (const char* e = std::getenv("SPTRSV_PIPE_WARPS")) nw = std::max(1, std::min(31, std::atoi(e)));
-  S.pipe_NW = nw;
-  S.pipe_P = P;
-  S.pipe_K = K;
-  S.pipe_GMAX = GMAX;
-  S.pipe_XW = XW;
-  S.pipe_NST = NST;
+  S.wave_strands.resize(sizeof(k::WaveStrand) * NS);
+  std::memcpy(S.wave_strands.data(), sr.data(), S.wave_strands.size());
+  S.wave_tau.assign(m, 0);
+  for (int r = 0; r < m; ++r) S.wave_tau[qpos[r]] = r;
+  S.wave_K = Kt;
+  S.wave_E = E;
+  S.wave_C = C;
+  S.wave_W = W;
+  S.wave_GPC = GPC;
+  S.wave_NCH = NCH;
+  S.wave_XW = XW;
+  S.wave_xa = xa;
+  S.wave_chunk_bytes = cbytes;
+  S.wave_bring_bytes = bring;
+  S.wave_group_bytes = gbytes;
+  S.wave_global = nglobal;
+}
+
+template <typename T, int K, int E>
+Error launch_wave_t(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
+  k::WaveGeom g{S.wave_W,           S.wave_GPC,         S.wave_NCH,         S.wave_XW,
+                S.wave_xa,          S.wave_chunk_bytes, S.wave_bring_bytes, S.wave_group_bytes,
+                k::wave_hdr_bytes(S.wave_GPC)};
+  const uint32_t smem = k::wave_smem_bytes<T>(g);
+  static uint32_t attr_bytes = 0;  // per template instance
+  if (smem > attr_bytes) {
+    CUDA_TRY(cudaFuncSetAttribute(k::tri_wave<T, K, E>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    CUDA_TRY(cudaFuncSetAttribute(k::tri_wave<T, K, E>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+    attr_bytes = smem;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(S.wave_C);
+  cfg.blockDim = dim3(32 * S.wave_W);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = S.wave_C;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  long long* tr = nullptr;
+  if (p.trace) {  // debug: SPTRSV_TRACE=1, per-strand clock64 stamps
+    const size_t nt = (size_t)S.wave_C * S.wave_W * 8;
+    if (S.h_trace.size() < nt) S.h_trace.assign(nt, 0);
+    if (!S.d_trace) CUDA_TRY(cudaMalloc(&S.d_trace, nt * 8));
+    CUDA_TRY(cudaMemsetAsync(S.d_trace, 0, nt * 8, s));
+    tr = (long long*)S.d_trace;
+  }
+  CUDA_TRY(cudaLaunchKernelEx(&cfg, k::tri_wave<T, K, E>, (const k::WaveStrand*)S.d_wave_strands, S.d_wave_data, bw,
+                              xs, g, st, tr));
+  return {SPTRSV_SUCCESS, ""};
 }
 
 template <typename T, int K>
-Error launch_pipe(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
-  const uint32_t smem = S.pipe_NST * k::pipe_stage_bytes<T>(K, S.pipe_GMAX) +
-                        k::al16((S.pipe_XW + 2) * (uint32_t)sizeof(T)) + 16 * S.pipe_NST;
-  static uint32_t attr_bytes = 0;  // per template instance
-  if (smem > attr_bytes) {
-    CUDA_TRY(cudaFuncSetAttribute(k::tri_chain_pipe<T, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    attr_bytes = smem;
+Error launch_wave_k(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
+  switch (S.wave_E) {
+    case 0: return launch_wave_t<T, K, 0>(p, S, bw, xs, st, s);
+    case 1: return launch_wave_t<T, K, 1>(p, S, bw, xs, st, s);
+    default: return launch_wave_t<T, K, 2>(p, S, bw, xs, st, s);
   }
-  k::tri_chain_pipe<T, K><<<S.pipe_P, 32 * (S.pipe_NW + 1), smem, s>>>(
-      S.pipe_P, S.d_pipe_stage0, (const k::PipeRec*)S.d_pipe_recs, S.d_pipe_data, bw, xs, S.pipe_NST, S.pipe_GMAX,
-      S.pipe_XW, st, S.ticket_slot);
-  return {SPTRSV_SUCCESS, ""};
+}
+
+template <typename T>
+Error launch_wave(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
+  switch (S.wave_K) {
+    case 1: return launch_wave_k<T, 1>(p, S, bw, xs, st, s);
+    case 2: return launch_wave_k<T, 2>(p, S, bw, xs, st, s);
+    case 4: return launch_wave_k<T, 4>(p, S, bw, xs, st, s);
+    default: return launch_wave_k<T, 8>(p, S, bw, xs, st, s);
+  }
 }
 
 template <typename T>
@@ -529,30 +683,30 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
     const int m = I.row1 - I.row0;
     const T* val = (const T*)S.d_val;
     if (I.kind == 1) {  // square: b -= A x
-      if (S.nzr > 0 && I.nnz > 0) {
-        bool dcsr = I.format == SPTRSV_FMT_DCSR;
+      if (S.dev_nzr > 0 && I.nnz > 0) {
+        const bool dcsr = S.dev_dcsr;
         if (nrhs == 1) {
           if (I.impl == SPTRSV_IMPL_SQ_VECTOR) {
-            unsigned g = cdiv((int64_t)S.nzr * 32, 256);
+            unsigned g = cdiv((int64_t)S.dev_nzr * 32, 256);
             if (dcsr)
-              k::sq_vector_1<T, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
+              k::sq_vector_1<T, true><<<g, 256, 0, s>>>(S.dev_nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
             else
-              k::sq_vector_1<T, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
+              k::sq_vector_1<T, false><<<g, 256, 0, s>>>(S.dev_nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
           } else {
-            unsigned g = cdiv(S.nzr, 256);
+            unsigned g = cdiv(S.dev_nzr, 256);
             if (dcsr)
-              k::sq_scalar_1<T, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
+              k::sq_scalar_1<T, true><<<g, 256, 0, s>>>(S.dev_nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
             else
-              k::sq_scalar_1<T, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
+              k::sq_scalar_1<T, false><<<g, 256, 0, s>>>(S.dev_nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
           }
         } else {
           dispatch_multi_un(nrhs, p.spmm, [&](auto G, auto R, auto U) {
-            unsigned g = cdiv((int64_t)S.nzr * G, 256);
+            unsigned g = cdiv((int64_t)S.dev_nzr * G, 256);
             if (dcsr)
-              k::sq_multi<T, G, R, U, true><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs,
+              k::sq_multi<T, G, R, U, true><<<g, 256, 0, s>>>(S.dev_nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs,
                                                               bw, nrhs);
             else
-              k::sq_multi<T, G, R, U, false><<<g, 256, 0, s>>>(S.nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs,
+              k::sq_multi<T, G, R, U, false><<<g, 256, 0, s>>>(S.dev_nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs,
                                                                bw, nrhs);
           });
         }
@@ -584,18 +738,18 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
           break;
         }
         case SPTRSV_IMPL_TRI_PIPE:
-          if (nrhs == 1 && S.pipe_K > 0) {
-            Error e;
-            switch (S.pipe_K) {
-              case 1: e = launch_pipe<T, 1>(p, S, bw, xs, st, s); break;
-              case 2: e = launch_pipe<T, 2>(p, S, bw, xs, st, s); break;
-              case 3: e = launch_pipe<T, 3>(p, S, bw, xs, st, s); break;
-              default: e = launch_pipe<T, 4>(p, S, bw, xs, st, s); break;
-            }
+          if (nrhs == 1 && S.wave_K > 0) {
+            Error e = launch_wave<T>(p, S, bw, xs, st, s);
             if (e.status) return e;
-            break;
+          } else {  // nrhs > 1: the device row order is not level-contiguous; the
+                    // multi-RHS sync-free kernel runs on the execution-order CSR
+            dispatch_multi(nrhs, [&](auto G, auto R) {
+              k::tri_syncfree_multi<T, G, R><<<std::max(1u, std::min<unsigned>(cdiv(m, 256 / G), p.sm_count * 2)),
+                                               256, 0, s>>>(I.row0, m, S.d_rp, S.d_ci, val, bw, xs, st,
+                                                            S.ticket_slot, nrhs);
+            });
           }
-          [[fallthrough]];  // nrhs > 1 or not buildable: the single-CTA chain
+          break;
         case SPTRSV_IMPL_TRI_CHAIN: {
           if (nrhs == 1 && S.ell_K > 0) {
             Error e;
@@ -708,6 +862,17 @@ void dump_trace(Plan& p, cudaStream_t s) {
   for (size_t si = 0; si < p.segs.size(); ++si) {
     Segment& S = p.segs[si];
     if (!S.d_trace) continue;
+    if (S.wave_K > 0) {  // raw per-strand stamps -> $SPTRSV_TRACE_DIR/wave_seg<i>.bin
+      const size_t nt = (size_t)S.wave_C * S.wave_W * 8;
+      cudaMemcpy(S.h_trace.data(), S.d_trace, nt * 8, cudaMemcpyDeviceToHost);
+      const char* dir = std::getenv("SPTRSV_TRACE_DIR");
+      std::string path = std::string(dir ? dir : ".") + "/wave_seg" + std::to_string(si) + ".bin";
+      if (FILE* f = std::fopen(path.c_str(), "wb")) {
+        std::fwrite(S.h_trace.data(), 8, nt, f);
+        std::fclose(f);
+      }
+      continue;
+    }
     const int nst = S.ell_K ? (int)(S.ell_recs.size() / 16) : (int)(S.chain_recs.size() / 16);
     cudaMemcpy(S.h_trace.data(), S.d_trace, (size_t)nst * 24, cudaMemcpyDeviceToHost);
     long long wait = 0, work = 0, gap = 0;
@@ -750,7 +915,7 @@ Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs
   // as the sentinel; nrhs > 1: they poll per-row epoch flags instead
   const int fill = (p.needs_sentinel && nrhs == 1) ? 1 : 0;
   uint32_t epoch = 0;
-  if (nrhs > 1 && p.needs_sentinel) {
+  if (nrhs > 1 && p.needs_flags) {
     if (!p.ws.flags) {
       if (cudaMalloc(&p.ws.flags, (size_t)std::max(1, n) * 4) != cudaSuccess) {
         cudaGetLastError();
@@ -835,7 +1000,7 @@ Error upload(Plan& p, void* stream_v) {
   };
   size_t o_perm = take((size_t)2 * n * 4);  // perm (new->old) then iperm (old->new)
   size_t o_rdiag = take((size_t)n * vb);
-  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed, sd, sc, sv, sbk, ps, pr, pd; };
+  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed, sd, sc, sv, sbk, ps, pd; };
   std::vector<Offs> so(p.segs.size());
   p.trace = std::getenv("SPTRSV_TRACE") != nullptr;
   p.spmm = spmm_cfg();
@@ -846,31 +1011,91 @@ Error upload(Plan& p, void* stream_v) {
   p.chain_geom[3] = cg.XW; p.chain_geom[4] = cg.LMAX;
   p.nticket = 0;
   p.needs_sentinel = false;
+  p.needs_flags = false;
+  for (size_t i = 0; i < p.segs.size(); ++i) build_wave(p, p.segs[i], vb);  // may switch a segment to CHAIN
+  // execution order of the rows on the device: identity except inside wave
+  // triangles (strand-major, group-major); sigma: new (plan) index -> device row
+  std::vector<int32_t> sigma;
+  for (auto& S : p.segs)
+    if (S.wave_K > 0) {
+      if (sigma.empty()) {
+        sigma.resize(n);
+        std::iota(sigma.begin(), sigma.end(), 0);
+      }
+      for (size_t q2 = 0; q2 < S.wave_tau.size(); ++q2) sigma[S.info.row0 + S.wave_tau[q2]] = S.info.row0 + (int)q2;
+    }
+  auto sg = [&](int32_t k2) { return sigma.empty() ? k2 : sigma[k2]; };
+  // device copies of the segment CSR in device row order
+  struct Dev { std::vector<int32_t> rp, ci, rows; std::vector<char> val; };
+  std::vector<Dev> dv(p.segs.size());
+  for (size_t i = 0; i < p.segs.size(); ++i) {
+    Segment& S = p.segs[i];
+    Dev& D = dv[i];
+    const auto& I = S.info;
+    if (I.kind == 0 && S.wave_K > 0) {  // rows permuted by wave_tau
+      const int m = I.row1 - I.row0;
+      D.rp.assign(m + 1, 0);
+      D.ci.reserve(S.ci.size());
+      D.val.reserve(S.val.size());
+      for (int q2 = 0; q2 < m; ++q2) {
+        const int r = S.wave_tau[q2];
+        for (int e = S.rp[r]; e < S.rp[r + 1]; ++e) D.ci.push_back(sg(S.ci[e]));
+        D.val.insert(D.val.end(), S.val.begin() + (size_t)S.rp[r] * vb, S.val.begin() + (size_t)S.rp[r + 1] * vb);
+        D.rp[q2 + 1] = (int32_t)D.ci.size();
+      }
+    } else {
+      D.rp = S.rp;
+      D.ci = S.ci;
+      if (!sigma.empty())
+        for (auto& c : D.ci) c = sigma[c];
+      D.val = S.val;
+    }
+    S.dev_dcsr = I.kind == 1 && I.format == SPTRSV_FMT_DCSR;
+    S.dev_nzr = S.nzr;
+    if (I.kind == 1) {
+      if (S.dev_dcsr) {
+        D.rows = S.rows;
+        for (auto& r : D.rows) r = sg(r);
+      } else {
+        bool moved = false;
+        for (int r = I.row0; r < I.row1 && !sigma.empty() && !moved; ++r) moved = sigma[r] != r;
+        if (moved) {  // CSR rows reordered: upload as DCSR with every row listed
+          S.dev_dcsr = true;
+          D.rows.resize(I.row1 - I.row0);
+          for (int r = I.row0; r < I.row1; ++r) D.rows[r - I.row0] = sigma[r];
+          S.dev_nzr = I.row1 - I.row0;
+        }
+      }
+    } else {
+      D.rows = S.rows;
+    }
+  }
   for (size_t i = 0; i < p.segs.size(); ++i) {
     Segment& S = p.segs[i];
     build_chain_stages(S, cg);
     build_chain_ell(S, vb);
     build_supernodes(S, vb);
-    build_pipeline(p, S, vb);
     so[i].er = take(S.ell_recs.size() * 4);
     so[i].ed = take(S.ell_data.size());
-    so[i].rp = take(S.rp.size() * 4);
-    so[i].ci = take(S.ci.size() * 4);
-    so[i].val = take(S.val.size());
-    so[i].rows = take(S.rows.size() * 4);
+    so[i].rp = take(dv[i].rp.size() * 4);
+    so[i].ci = take(dv[i].ci.size() * 4);
+    so[i].val = take(dv[i].val.size());
+    so[i].rows = take(dv[i].rows.size() * 4);
     so[i].lp = take(S.level_ptr.size() * 4);
     so[i].st = take(S.chain_recs.size() * 4);
     so[i].sd = take(S.sn_desc.size());
     so[i].sc = take(S.sn_cols.size() * 4);
     so[i].sv = take(S.sn_vals.size());
     so[i].sbk = take(S.sn_blk.size());
-    so[i].ps = take(S.pipe_stage0.size() * 4);
-    so[i].pr = take(S.pipe_recs.size() * 4);
-    so[i].pd = take(S.pipe_data.size());
+    so[i].ps = take(S.wave_strands.size());
+    so[i].pd = take(S.wave_data.size());
     if (S.info.kind == 0) S.ticket_slot = p.nticket++;
     if (S.info.kind == 0 && (S.info.impl == SPTRSV_IMPL_TRI_SYNCFREE || S.info.impl == SPTRSV_IMPL_TRI_SUPERNODE ||
-                             S.info.impl == SPTRSV_IMPL_TRI_PIPE))
+                             (S.info.impl == SPTRSV_IMPL_TRI_PIPE && (S.wave_K == 0 || S.wave_global > 0))))
       p.needs_sentinel = true;
+    if (S.info.kind == 0 && (S.info.impl == SPTRSV_IMPL_TRI_SYNCFREE || S.info.impl == SPTRSV_IMPL_TRI_SUPERNODE ||
+                             S.info.impl == SPTRSV_IMPL_TRI_PIPE))
+      p.needs_flags = true;
   }
   size_t o_tickets = take((size_t)std::max(1, p.nticket) * 4);
   p.arena_bytes = off;
@@ -884,20 +1109,27 @@ Error upload(Plan& p, void* stream_v) {
   }
   // host staging of the whole arena, then one copy
   std::vector<char> h(off, 0);
-  std::vector<int32_t> iperm(n);
-  // p.perm is already in ORIGINAL indexing (UPPER: composed with J), so the
-  // kernels gather b[perm[k]] / scatter x[perm[k]] directly.
-  for (int k2 = 0; k2 < n; ++k2) iperm[p.perm[k2]] = k2;
-  std::memcpy(&h[o_perm], p.perm.data(), (size_t)n * 4);
-  std::memcpy(&h[o_perm + (size_t)n * 4], iperm.data(), (size_t)n * 4);
-  std::memcpy(&h[o_rdiag], p.rdiag_new.data(), (size_t)n * vb);
+  // p.perm is in ORIGINAL indexing (UPPER: composed with J); the device
+  // gathers b[perm_dev[k]] into device row k and scatters x back
+  {
+    int32_t* pd = (int32_t*)&h[o_perm];
+    int32_t* ip = pd + n;
+    char* rd = &h[o_rdiag];
+    for (int k2 = 0; k2 < n; ++k2) {
+      const int d = sg(k2);
+      pd[d] = p.perm[k2];
+      ip[p.perm[k2]] = d;
+      std::memcpy(rd + (size_t)d * vb, &p.rdiag_new[(size_t)k2 * vb], vb);
+    }
+  }
   char* A = (char*)p.arena;
   for (size_t i = 0; i < p.segs.size(); ++i) {
     Segment& S = p.segs[i];
-    std::memcpy(&h[so[i].rp], S.rp.data(), S.rp.size() * 4);
-    std::memcpy(&h[so[i].ci], S.ci.data(), S.ci.size() * 4);
-    std::memcpy(&h[so[i].val], S.val.data(), S.val.size());
-    std::memcpy(&h[so[i].rows], S.rows.data(), S.rows.size() * 4);
+    const Dev& D = dv[i];
+    std::memcpy(&h[so[i].rp], D.rp.data(), D.rp.size() * 4);
+    std::memcpy(&h[so[i].ci], D.ci.data(), D.ci.size() * 4);
+    std::memcpy(&h[so[i].val], D.val.data(), D.val.size());
+    std::memcpy(&h[so[i].rows], D.rows.data(), D.rows.size() * 4);
     std::memcpy(&h[so[i].lp], S.level_ptr.data(), S.level_ptr.size() * 4);
     std::memcpy(&h[so[i].st], S.chain_recs.data(), S.chain_recs.size() * 4);
     S.d_rp = (const int32_t*)(A + so[i].rp);
@@ -918,12 +1150,10 @@ Error upload(Plan& p, void* stream_v) {
     S.d_sn_cols = (const int32_t*)(A + so[i].sc);
     S.d_sn_vals = (const void*)(A + so[i].sv);
     S.d_sn_blk = (const void*)(A + so[i].sbk);
-    std::memcpy(&h[so[i].ps], S.pipe_stage0.data(), S.pipe_stage0.size() * 4);
-    std::memcpy(&h[so[i].pr], S.pipe_recs.data(), S.pipe_recs.size() * 4);
-    std::memcpy(&h[so[i].pd], S.pipe_data.data(), S.pipe_data.size());
-    S.d_pipe_stage0 = (const int32_t*)(A + so[i].ps);
-    S.d_pipe_recs = (const int32_t*)(A + so[i].pr);
-    S.d_pipe_data = (const char*)(A + so[i].pd);
+    std::memcpy(&h[so[i].ps], S.wave_strands.data(), S.wave_strands.size());
+    std::memcpy(&h[so[i].pd], S.wave_data.data(), S.wave_data.size());
+    S.d_wave_strands = (const void*)(A + so[i].ps);
+    S.d_wave_data = (const char*)(A + so[i].pd);
   }
   p.d_perm = (const int32_t*)(A + o_perm);
   p.d_rdiag = (const void*)(A + o_rdiag);

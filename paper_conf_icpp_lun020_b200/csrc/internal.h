@@ -51,14 +51,19 @@ struct Segment {
   const int32_t* d_sn_cols = nullptr;
   const void* d_sn_vals = nullptr;
   const void* d_sn_blk = nullptr;
-  // partitioned pipeline chain (nrhs == 1): P partitions, per-partition stages
-  int pipe_P = 0, pipe_K = 0, pipe_NW = 4, pipe_GMAX = 32, pipe_XW = 8192, pipe_NST = 3;
-  std::vector<int32_t> pipe_stage0;  // [P+1] first stage of every partition
-  std::vector<int32_t> pipe_recs;    // 16 ints per stage (k::PipeRec + pad)
-  std::vector<char> pipe_data;       // stage blocks
-  const int32_t* d_pipe_stage0 = nullptr;
-  const int32_t* d_pipe_recs = nullptr;
-  const char* d_pipe_data = nullptr;
+  // strand wavefront over a cluster (k::tri_wave, nrhs == 1); wave_K == 0: not built
+  int wave_K = 0, wave_E = 0, wave_C = 0, wave_W = 0, wave_GPC = 0, wave_NCH = 0, wave_XW = 0, wave_xa = 0;
+  uint32_t wave_chunk_bytes = 0, wave_bring_bytes = 0, wave_group_bytes = 0;
+  int64_t wave_global = 0;         // dependencies polled in global memory (needs the xs sentinel)
+  std::vector<int32_t> wave_tau;   // execution position q -> local row (the device row order of the triangle)
+  std::vector<char> wave_strands;  // k::WaveStrand[C * W]
+  std::vector<char> wave_data;     // chunk blocks
+  const void* d_wave_strands = nullptr;
+  const char* d_wave_data = nullptr;
+  // device-side square format: a CSR square whose rows are reordered by a
+  // wave triangle is uploaded as DCSR with explicit (execution-order) rows
+  bool dev_dcsr = false;
+  int32_t dev_nzr = 0;
   // TMA-staged chain kernel (nrhs == 1): 8-int stage records (k::StageRec),
   // empty = not staged
   std::vector<int32_t> chain_recs;
@@ -120,7 +125,8 @@ struct Plan {
   const void* d_rdiag = nullptr;  // 1/d in new order (permute-in scaling)
   uint32_t* d_tickets = nullptr;  // [nticket] sync-free row-claim counters
   int32_t nticket = 0;
-  bool needs_sentinel = false;    // a sync-free triangle polls xs
+  bool needs_sentinel = false;    // nrhs == 1: a triangle polls xs (value-as-flag)
+  bool needs_flags = false;       // nrhs > 1: a sync-free triangle polls per-row epoch flags
   int chain_geom[5] = {0, 0, 0, 0, 0};  // NST, RMAX, EMAX, XW, LMAX frozen at upload
   bool trace = false;                   // SPTRSV_TRACE debug stamps
   int32_t* h_error = nullptr;  // mapped pinned host word set by the watchdog

@@ -1173,218 +1173,302 @@ __global__ void __launch_bounds__(1024, 1)
   }
 }
 
-// ------------------- K4' (B200): partitioned chain, shared-memory spin flags
-// The rows of a narrow-level triangle are split into P partitions by their
-// ORIGINAL row index (contiguous ranges).  L is lower in the original
-// numbering, so a row only depends on rows of its own or a LOWER partition:
-// the partitions form a pipeline, and partition q can run a few levels
-// behind partition q-1.  One CTA (one SM) per partition, claimed in order
-// through the segment ticket (a CTA only waits on partitions claimed before
-// it, so any CTA schedule makes progress).
-// Inside a CTA the partition's rows are processed in level order as groups
-// of 32 rows of one level (padded); group gi belongs to consumer warp
-// gi % NW.  There is no per-level barrier: a dependency computed by this CTA
-// is read from a shared-memory window slot (local position mod XW) whose
-// value is its own ready flag (sentinel until written; ld.volatile.shared
-// spin, ~30-cycle detection), a dependency of another partition (or one too
-// old for the window) is polled in global memory (value-as-flag, L2).  The
-// only barriers are at stage ends (TMA buffer ring + window slot recycling).
-// Stage block (TMA'd): int4 group records {first padded row, level, -, -}
-// are not needed -- groups are 32 padded rows in order -- so a stage is:
-//   grow[npad] (global permuted row, -1 = padding), words[K+1][npad]
-//   (k < K: bit 31 = global, low bits = global row; else window slot;
-//   k = K: the row's own window slot), vals[K][npad], then room for the
-//   gathered b'[npad].
-struct PipeRec {
-  int pos0, pos1, ngroups, off16, bytes, npad, pad0, pad1;  // real local positions [pos0,pos1)
+// ------------- K4' (B200): strand wavefront over a thread-block cluster
+// For a narrow-level triangle (the near-serial / level-set role of Alg 7,
+// L256, where the levels are too narrow to fill the GPU and each level would
+// cost a grid-wide synchronisation), the rows are split into NS = C x W
+// STRANDS: contiguous ranges of the ORIGINAL (lower) row index, balanced in
+// rows.  L is lower in the original numbering, so a row depends only on rows
+// of its own or of a lower strand; strands form a pipeline, and strand s runs
+// a few levels behind strand s-1 (the wavefront).  One warp owns a strand
+// and walks its rows in level order as GROUPS of <= 32 rows of one level
+// (lane = row), with no barrier at all: the level order inside the warp
+// replaces Alg 2's level barrier (L96), and a dependency on another strand
+// is a shared-memory value that is its own ready flag (the sentinel of the
+// sync-free kernels, Alg 3, kept on-chip):
+//   * own strand, within XW positions: the warp's private ring window
+//     (written by this warp in an earlier group; __syncwarp orders it);
+//   * another strand of the cluster: a unique IMPORT slot in this warp's
+//     shared memory; the producing lane PUSHES its x there (st.shared::cluster
+//     to the consumer CTA, DSMEM, ~200 cycles) right after computing it, and
+//     the consumer spins on its own shared memory (~30 cycles), so the
+//     cross-SM hop overlaps the producer's lead instead of sitting on the
+//     chain;
+//   * anything else (window / import capacity overflow): xs in global memory,
+//     polled with strong loads (value-as-flag).
+// The execution order of the triangle's rows on the device is strand-major,
+// group-major (the upload applies that permutation to the plan's device
+// indices), so a group is a contiguous range of rows: its b' arrives by TMA
+// and its x stores are coalesced.  Per strand the operands stream through a
+// ring of NCH chunks (GPC groups each) filled by cp.async.bulk (lane 0) on
+// one mbarrier per chunk; the chunk header carries the row range of chunk
+// c + NCH, so no control word is read from global memory inside the loop.
+//
+// Chunk block: int4 {row_lo, row_hi, next_lo, next_hi} (b' rows of this chunk
+// and of chunk c + NCH), int2 {row_start, cnt | flags} per group (GPC, padded
+// to 16 bytes), then GPC group blocks {u32 words[K][32], u32 push[E][32],
+// T vals[K][32]}.
+// word: bit 31 clear = slot (in T units) of the CTA's x area; set = global
+// (execution-order) row of xs.  push: (cta rank << 24) | slot, ~0u = none.
+// Group flags (high bits of cnt): GF_GLOBAL = a lane has a global word,
+// GF_PUSH = a lane pushes.  A group with cnt == 0 is padding.
+//
+// Single-warp critical path per group (the level chain of the strand):
+// __syncwarp -> LDS x_j -> sentinel vote -> 2 x DFMA -> STS x_i.  Everything
+// else (the next group's operands, the TMA ring, the global store and the
+// pushes) is issued in the shadow of that chain: the loop is software-
+// pipelined by one group (round-1 trace: a straightforward loop spent ~700
+// cycles per group in dependent address/branch latency of one warp).
+constexpr int kWaveGF_GLOBAL = 1 << 30, kWaveGF_PUSH = 1 << 29, kWaveCntMask = (1 << 29) - 1;
+struct WaveStrand {
+  int off16, nchunk, own_base, row0;  // row0: first execution-order row of the strand
+  int lo[4], hi[4];                   // b' row ranges of chunks 0..3 (the prologue loads)
+  int ngroups, pad[3];
+};
+struct WaveGeom {
+  int W, GPC, NCH, XW;   // warps per CTA, groups per chunk, ring depth, own window
+  int xa_slots;          // x area slots per CTA
+  uint32_t chunk_bytes, bring_bytes, group_bytes, hdr_bytes;
 };
 
 template <typename T>
-__host__ __device__ inline uint32_t pipe_stage_bytes(int K, int GMAX) {
-  const uint32_t np = (uint32_t)GMAX * 32;
-  return 64 + al16(np * 4) + al16((uint32_t)(K + 1) * np * 4) + al16((uint32_t)K * np * (uint32_t)sizeof(T)) +
-         al16(np * (uint32_t)sizeof(T));  // + gathered b'
+__host__ __device__ inline uint32_t wave_group_bytes(int K, int E) {
+  return 128u * (uint32_t)K + 128u * (uint32_t)E + 32u * (uint32_t)K * (uint32_t)sizeof(T);
 }
-
-// offsets inside one stage block (packed to the stage's own npad)
-__host__ __device__ inline uint32_t pipe_off_words(int npad) { return 64 + al16((uint32_t)npad * 4); }
-__host__ __device__ inline uint32_t pipe_off_vals(int K, int npad) {
-  return pipe_off_words(npad) + al16((uint32_t)(K + 1) * npad * 4);
+__host__ __device__ inline uint32_t wave_hdr_bytes(int GPC) { return 16u + al16(8u * (uint32_t)GPC); }
+template <typename T>
+__host__ __device__ inline uint32_t wave_bring_bytes(int GPC) {
+  return al16((uint32_t)GPC * 32u * (uint32_t)sizeof(T) + 32u);
 }
 template <typename T>
-__host__ __device__ inline uint32_t pipe_off_b(int K, int npad) {
-  return pipe_off_vals(K, npad) + al16((uint32_t)K * npad * (uint32_t)sizeof(T));
+__host__ __device__ inline uint32_t wave_smem_bytes(const WaveGeom& g) {
+  return al16((uint32_t)g.xa_slots * (uint32_t)sizeof(T)) +
+         (uint32_t)(g.W * g.NCH) * (g.chunk_bytes + g.bring_bytes) + (uint32_t)(g.W * g.NCH) * 8u;
 }
 
-__device__ __forceinline__ double lds_volatile(uint32_t a, double) {
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t mapa_shared(uint32_t a, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ void st_cluster(uint32_t a, double v) {
+  asm volatile("st.relaxed.cluster.shared::cluster.f64 [%0], %1;" ::"r"(a), "d"(v) : "memory");
+}
+__device__ __forceinline__ void st_cluster(uint32_t a, float v) {
+  asm volatile("st.relaxed.cluster.shared::cluster.f32 [%0], %1;" ::"r"(a), "f"(v) : "memory");
+}
+// x loads / stores of the wave loop: volatile (never cached or dropped) and
+// ordered among themselves, but without a "memory" clobber so the compiler
+// may schedule the operand prefetch around them
+__device__ __forceinline__ double lds_x_v(uint32_t a, double) {
   double v;
-  asm volatile("ld.volatile.shared.f64 %0, [%1];" : "=d"(v) : "r"(a) : "memory");
+  asm volatile("ld.volatile.shared.f64 %0, [%1];" : "=d"(v) : "r"(a));
   return v;
 }
-__device__ __forceinline__ float lds_volatile(uint32_t a, float) {
+__device__ __forceinline__ float lds_x_v(uint32_t a, float) {
   float v;
-  asm volatile("ld.volatile.shared.f32 %0, [%1];" : "=f"(v) : "r"(a) : "memory");
+  asm volatile("ld.volatile.shared.f32 %0, [%1];" : "=f"(v) : "r"(a));
   return v;
+}
+__device__ __forceinline__ void sts_x_v(uint32_t a, double v) {
+  asm volatile("st.volatile.shared.f64 [%0], %1;" ::"r"(a), "d"(v));
+}
+__device__ __forceinline__ void sts_x_v(uint32_t a, float v) {
+  asm volatile("st.volatile.shared.f32 [%0], %1;" ::"r"(a), "f"(v));
+}
+__device__ __forceinline__ double ldg_x_v(const double* p) {
+  double v;
+  asm volatile("ld.relaxed.gpu.global.f64 %0, [%1];" : "=d"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ float ldg_x_v(const float* p) {
+  float v;
+  asm volatile("ld.relaxed.gpu.global.f32 %0, [%1];" : "=f"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void stg_x_v(double* p, double v) {
+  asm volatile("st.relaxed.gpu.global.f64 [%0], %1;" ::"l"(p), "d"(v));
+}
+__device__ __forceinline__ void stg_x_v(float* p, float v) {
+  asm volatile("st.relaxed.gpu.global.f32 [%0], %1;" ::"l"(p), "f"(v));
 }
 
-template <typename T, int K>
-__global__ void __launch_bounds__(1024, 1)
-    tri_chain_pipe(int nparts, const int* __restrict__ part_stage0, const PipeRec* __restrict__ recs,
-                   const char* __restrict__ data, const T* __restrict__ bw, T* __restrict__ xs, int NST, int GMAX,
-                   int XW, SolveState st, int slot) {
+template <typename T, int K, int E>
+struct WaveOp {
+  uint32_t w[K];  // words (own slot, import slot | WAVE_IMP, global row | WAVE_GLB)
+  T v[K];
+  T xi[K];        // import / global operands, polled one group ahead
+  T b;
+  int row, cnt;   // cnt with the group flags
+  uint32_t push[E > 0 ? E : 1];
+};
+constexpr uint32_t kWaveGLB = 0x80000000u, kWaveIMP = 0x40000000u, kWaveIdx = 0x3fffffffu;
+
+template <typename T, int K, int E>
+__global__ void __launch_bounds__(256, 1)
+    tri_wave(const WaveStrand* __restrict__ strands, const char* __restrict__ data, const T* __restrict__ bw,
+             T* __restrict__ xs, WaveGeom g, SolveState st, long long* __restrict__ trace) {
   extern __shared__ __align__(128) unsigned char smem[];
   constexpr uint32_t SH = sizeof(T) == 8 ? 3 : 2;
-  const int tid = threadIdx.x;
-  const int NC = blockDim.x - 32;
-  const int NW = NC >> 5, warp = tid >> 5, lane = tid & 31;
-  const uint32_t xmask = (uint32_t)XW - 1;
-  const uint32_t sbytes = pipe_stage_bytes<T>(K, GMAX);
-  unsigned char* xw_p = smem + (size_t)NST * sbytes;
-  const uint32_t xw = smem_addr(xw_p);
-  uint64_t* full = (uint64_t*)(xw_p + al16((XW + 2) * (uint32_t)sizeof(T)));
-  uint64_t* empty = full + NST;
-  __shared__ int s_part;
-  if (tid == 0) {
-    s_part = (int)atomicAdd(st.tickets + slot, 1u);
-    for (int b = 0; b < NST; ++b) {
-      mbar_init(&full[b], 1);
-      mbar_init(&empty[b], 1);
-    }
-    ((T*)xw_p)[XW] = T(0);  // the zero slot of padding rows
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  // all window slots start as the sentinel
-  for (int i = tid; i < XW; i += blockDim.x) ((T*)xw_p)[i] = sent<T>();
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const uint32_t rank = cluster_ctarank();
+  const WaveStrand* Sp = strands + rank * g.W + warp;
+  const int s_nchunk = Sp->nchunk, s_ng = Sp->ngroups, s_own = Sp->own_base, s_row0 = Sp->row0;
+  const char* s_data = data + (size_t)Sp->off16 * 16;
+  long long* tr = trace ? trace + (size_t)(rank * g.W + warp) * 8 : nullptr;
+  if (tr && lane == 0) tr[0] = clock64();
+  T* xa = (T*)smem;
+  const uint32_t xa_s = smem_addr(smem);
+  unsigned char* ring = smem + al16((uint32_t)g.xa_slots * (uint32_t)sizeof(T));
+  unsigned char* bring = ring + (size_t)(g.W * g.NCH) * g.chunk_bytes;
+  uint64_t* full = (uint64_t*)(bring + (size_t)(g.W * g.NCH) * g.bring_bytes) + warp * g.NCH;
+  ring += (size_t)warp * g.NCH * g.chunk_bytes;
+  bring += (size_t)warp * g.NCH * g.bring_bytes;
+  // x area: two zero slots (padding dependencies), the rest the sentinel
+  // (import slots must read "not ready" until pushed)
+  for (int i = tid; i < g.xa_slots; i += blockDim.x) xa[i] = i < 2 ? T(0) : sent<T>();
+  if (lane == 0)
+    for (int c = 0; c < g.NCH; ++c) mbar_init(&full[c], 1);
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncthreads();
-  const int part = s_part;
-  if (part >= nparts) return;
-  const int s0 = part_stage0[part], nstage = part_stage0[part + 1] - s0;
+  cluster_sync_all();  // every import area is initialised before any push
 
-  if (tid >= NC) {  // ---------------- producer warp: stage loads
-    if (tid == NC) {
-      int b = 0;
-      uint32_t ph = 0;
-      for (int s = 0; s < nstage; ++s) {
-        unsigned char* B = smem + (size_t)b * sbytes;
-        if (s >= NST) mbar_wait(&empty[b], ph ^ 1u);
-        const PipeRec R = recs[2 * (s0 + s)];
-        mbar_expect_tx(&full[b], 64 + R.bytes);
-        tma_bulk_g2s(B, recs + 2 * (s0 + s), 64, &full[b]);
-        tma_bulk_g2s(B + 64, data + (size_t)R.off16 * 16, R.bytes, &full[b]);
-        if (++b == NST) {
-          b = 0;
+  auto issue_chunk = [&](int slot, int c, int lo, int hi) {
+    const Win wb = win(bw, (int64_t)lo, hi - lo);
+    mbar_expect_tx(&full[slot], g.chunk_bytes + wb.bytes);
+    tma_bulk_g2s(ring + (size_t)slot * g.chunk_bytes, s_data + (size_t)c * g.chunk_bytes, g.chunk_bytes, &full[slot]);
+    tma_bulk_g2s(bring + (size_t)slot * g.bring_bytes, wb.src, wb.bytes, &full[slot]);
+  };
+  if (lane == 0)
+    for (int c = 0; c < g.NCH && c < s_nchunk; ++c) issue_chunk(c, c, Sp->lo[c], Sp->hi[c]);
+  if (tr && lane == 0) tr[1] = clock64();
+
+  const uint32_t xmask = (uint32_t)g.XW - 1;
+  uint32_t spins = 0, npolls = 0;
+  // position of the NEXT group: chunk c_n (ring slot `slot`, phase `ph`),
+  // index gi_n inside it; B_n / bb_n: that chunk's block and b' base
+  int slot = 0, c_n = 0, gi_n = 0;
+  uint32_t ph = 0;
+  const unsigned char* B_n = ring;
+  const T* bb_n = nullptr;
+  auto enter_chunk = [&]() {
+    mbar_wait(&full[slot], ph);
+    B_n = ring + (size_t)slot * g.chunk_bytes;
+    const int lo = *(const int*)B_n;
+    bb_n = (const T*)(bring + (size_t)slot * g.bring_bytes) + shift_of(bw, (int64_t)lo) - lo;
+  };
+  auto load_op = [&](WaveOp<T, K, E>& o) {
+    const int2 gh = ((const int2*)(B_n + 16))[gi_n];
+    const uint32_t* wd = (const uint32_t*)(B_n + g.hdr_bytes + (uint32_t)gi_n * g.group_bytes);
+    const T* vv = (const T*)(wd + 32 * (K + E));
+#pragma unroll
+    for (int k2 = 0; k2 < K; ++k2) {
+      o.w[k2] = wd[k2 * 32 + lane];
+      o.v[k2] = vv[k2 * 32 + lane];
+    }
+#pragma unroll
+    for (int e = 0; e < E; ++e) o.push[e] = wd[(K + e) * 32 + lane];
+    o.row = gh.x + lane;
+    o.cnt = gh.y;
+    o.b = lane < (gh.y & kWaveCntMask) ? bb_n[o.row] : T(0);
+    // dependencies on OTHER strands are polled now, a group ahead of use, so
+    // their readiness test is off the level chain
+#pragma unroll
+    for (int k2 = 0; k2 < K; ++k2)
+      o.xi[k2] = (o.w[k2] & kWaveGLB)   ? ldg_x_v(xs + (o.w[k2] & kWaveIdx))
+                 : (o.w[k2] & kWaveIMP) ? lds_x_v(xa_s + ((o.w[k2] & kWaveIdx) << SH), T(0))
+                                        : T(0);
+  };
+
+  WaveOp<T, K, E> nxt;
+  if (s_ng > 0) {
+    enter_chunk();
+    load_op(nxt);
+  }
+  for (int gidx = 0; gidx < s_ng; ++gidx) {
+    WaveOp<T, K, E> cur = nxt;
+    const bool act = lane < (cur.cnt & kWaveCntMask);
+    // ---- other-strand operands: normally ready since the last group
+    bool pend = false;
+#pragma unroll
+    for (int k2 = 0; k2 < K; ++k2) pend |= (cur.w[k2] & (kWaveGLB | kWaveIMP)) && is_sent(cur.xi[k2]);
+    if (__any_sync(0xffffffffu, pend)) {  // a producer strand is behind: wait for it
+      while (__any_sync(0xffffffffu, pend)) {
+        ++npolls;
+        pend = false;
+#pragma unroll
+        for (int k2 = 0; k2 < K; ++k2) {
+          if ((cur.w[k2] & (kWaveGLB | kWaveIMP)) && is_sent(cur.xi[k2])) {
+            cur.xi[k2] = (cur.w[k2] & kWaveGLB) ? ldg_x_v(xs + (cur.w[k2] & kWaveIdx))
+                                                : lds_x_v(xa_s + ((cur.w[k2] & kWaveIdx) << SH), T(0));
+            pend |= is_sent(cur.xi[k2]);
+          }
+        }
+        if (pend && ++spins > kWatchdogSpins) {
+          watchdog_trip(st);
+#pragma unroll
+          for (int k2 = 0; k2 < K; ++k2) cur.xi[k2] = is_sent(cur.xi[k2]) ? T(0) : cur.xi[k2];
+          pend = false;
+        }
+      }
+    }
+    // ---- critical chain: own-strand x_j (written by this warp before the
+    // last __syncwarp: always ready, no test)
+    T x[K];
+#pragma unroll
+    for (int k2 = 0; k2 < K; ++k2)
+      x[k2] = (cur.w[k2] & (kWaveGLB | kWaveIMP)) ? cur.xi[k2] : lds_x_v(xa_s + (cur.w[k2] << SH), T(0));
+    // ---- prefetch the next group's operands in the shadow of the loads
+    int refill_slot = -1, refill_c = 0;
+    if (gidx + 1 < s_ng) {
+      if (++gi_n == g.GPC) {  // next group opens a new chunk: the current one
+        gi_n = 0;             // is consumed once this group is done
+        refill_slot = slot;
+        refill_c = c_n;
+        ++c_n;
+        if (++slot == g.NCH) {
+          slot = 0;
           ph ^= 1u;
         }
+        enter_chunk();
       }
+      load_op(nxt);
     }
-    return;
+    T acc = cur.b;
+#pragma unroll
+    for (int k2 = 0; k2 < K; ++k2) acc = fma(-cur.v[k2], x[k2], acc);
+    if (act) {
+      sts_x_v(xa_s + ((uint32_t)(s_own + ((uint32_t)(cur.row - s_row0) & xmask)) << SH), acc);
+      if (E > 0 && (cur.cnt & kWaveGF_PUSH)) {
+#pragma unroll
+        for (int e = 0; e < E; ++e)
+          if (cur.push[e] != 0xffffffffu)
+            st_cluster(mapa_shared(xa_s + ((cur.push[e] & 0xffffffu) << SH), cur.push[e] >> 24), acc);
+      }
+      stg_x_v(xs + cur.row, acc);
+    }
+    if (refill_slot >= 0 && lane == 0 && refill_c + g.NCH < s_nchunk) {
+      // every operand of chunk refill_c is consumed: reuse its ring slot
+      const int4 hdr = *(const int4*)(ring + (size_t)refill_slot * g.chunk_bytes);
+      issue_chunk(refill_slot, refill_c + g.NCH, hdr.z, hdr.w);
+    }
+    __syncwarp();
   }
-
-  // ---------------- consumer warps
-  uint32_t spins = 0;
-  int b = 0;
-  uint32_t ph = 0;
-  // b' of the NEXT stage's rows is gathered from global memory during the
-  // current stage (8 per thread in flight) and parked in its stage buffer
-  constexpr int BG = 8;
-  T bnext[BG];
-  auto gather_issue = [&](const unsigned char* B) {
-    const PipeRec R = ((const PipeRec*)B)[0];
-    const int* grow = (const int*)(B + 64);
-#pragma unroll
-    for (int u = 0; u < BG; ++u) {
-      const int i = tid + u * NC;
-      const int g = i < R.npad ? grow[i] : -1;
-      bnext[u] = g >= 0 ? ldg_nc(bw + g) : T(0);
-    }
-  };
-  auto gather_park = [&](unsigned char* B) {
-    const PipeRec R = ((const PipeRec*)B)[0];
-    T* sb = (T*)(B + pipe_off_b<T>(K, R.npad));
-#pragma unroll
-    for (int u = 0; u < BG; ++u) {
-      const int i = tid + u * NC;
-      if (i < R.npad) sb[i] = bnext[u];
-    }
-    for (int i = tid + BG * NC; i < R.npad; i += NC) {  // rare: more rows than BG * NC
-      const int g = ((const int*)(B + 64))[i];
-      sb[i] = g >= 0 ? ldg_nc(bw + g) : T(0);
-    }
-  };
-  if (nstage > 0) {
-    mbar_wait(&full[0], 0);
-    gather_issue(smem);
-    gather_park(smem);
+  if (tr && lane == 0) {
+    tr[2] = clock64();
+    tr[3] = npolls;
+    tr[4] = s_ng;
   }
-  asm volatile("bar.sync 1, %0;" ::"r"(NC) : "memory");
-  for (int s = 0; s < nstage; ++s) {
-    unsigned char* B = smem + (size_t)b * sbytes;
-    const PipeRec R = ((const PipeRec*)B)[0];
-    const int nb = b + 1 == NST ? 0 : b + 1;
-    const uint32_t nph = b + 1 == NST ? ph ^ 1u : ph;
-    unsigned char* Bn = smem + (size_t)nb * sbytes;
-    const bool has_next = s + 1 < nstage;
-    if (has_next) {
-      mbar_wait(&full[nb], nph);  // TMA runs ahead; normally already complete
-      gather_issue(Bn);
-      // recycle the window slots of the next stage's rows: their previous
-      // occupants (XW positions back) have no readers left (analysis bound)
-      const PipeRec Rn = ((const PipeRec*)Bn)[0];
-      for (int q = Rn.pos0 + tid; q < Rn.pos1; q += NC) ((T*)xw_p)[(uint32_t)q & xmask] = sent<T>();
-    }
-    const int npad = R.npad;
-    const int* grow = (const int*)(B + 64);
-    const uint32_t* words = (const uint32_t*)(B + pipe_off_words(npad));
-    const T* vals = (const T*)(B + pipe_off_vals(K, npad));
-    const T* sb = (const T*)(B + pipe_off_b<T>(K, npad));
-    for (int gi = warp; gi < R.ngroups; gi += NW) {
-      const int i = gi * 32 + lane;
-      const int g = grow[i];
-      T acc = sb[i];
-      uint32_t wd[K];
-      T v[K];
-#pragma unroll
-      for (int k2 = 0; k2 < K; ++k2) {
-        wd[k2] = words[k2 * npad + i];
-        v[k2] = vals[k2 * npad + i];
-      }
-#pragma unroll
-      for (int k2 = 0; k2 < K; ++k2) {
-        T x;
-        if (wd[k2] & 0x80000000u) {
-          const T* px = xs + (wd[k2] & 0x7fffffffu);
-          x = ld_strong(px);
-          while (is_sent(x)) {
-            if (++spins > kWatchdogSpins) {
-              watchdog_trip(st);
-              break;
-            }
-            x = ld_strong(px);
-          }
-        } else {
-          const uint32_t a = xw + (wd[k2] << SH);
-          x = lds_volatile(a, T(0));
-          while (is_sent(x)) {
-            if (++spins > kWatchdogSpins) {
-              watchdog_trip(st);
-              break;
-            }
-            x = lds_volatile(a, T(0));
-          }
-        }
-        acc -= v[k2] * x;
-      }
-      if (g >= 0) {
-        sts_x(xw + (words[K * npad + i] << SH), acc);  // word K: this row's window slot
-        st_strong(xs + g, acc);
-      }
-    }
-    if (has_next) gather_park(Bn);
-    asm volatile("bar.sync 1, %0;" ::"r"(NC) : "memory");  // stage end: slots recycled, buffer free
-    if (tid == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(&empty[b])) : "memory");
-    b = nb;
-    ph = nph;
-  }
+  __syncthreads();
+  cluster_sync_all();  // no CTA leaves while a peer may still push into it
 }
 
 }  // namespace k

@@ -65,7 +65,9 @@ def test_forced_kernels(gpu, name, tri, sq):
     if tri == "TRI_LEVELSET" and name in ("C2",):
         pytest.skip("thousands of per-level launches; covered by C1/C3-C5")
     x, plan = _solve(M, b, depth=2, force_tri_impl=tri, force_sq_impl=sq, reorder=True)
-    assert all(s["impl"] == tri for s in plan.segments() if s["kind"] == "TRI" and s["nlevels"] > 1)
+    # the wavefront hands rows with > 8 dependencies to the chain kernel
+    ok = (tri, "TRI_CHAIN") if tri == "TRI_PIPE" and name in ("C3", "C4", "C5") else (tri,)
+    assert all(s["impl"] in ok for s in plan.segments() if s["kind"] == "TRI" and s["nlevels"] > 1)
     _check64(M, b, x)
 
 
@@ -234,12 +236,40 @@ def test_full_size_c5_multi_rhs_sampled(gpu):
     assert ok, worst
 
 
-@pytest.mark.parametrize("P", ["1", "3", "8"])
-def test_pipe_partitions(gpu, P, monkeypatch):
-    """The partitioned pipeline chain at several partition counts (each
-    partition one CTA; cross-partition dependencies polled in L2)."""
-    monkeypatch.setenv("SPTRSV_PIPE_P", P)
-    for name in ("C2", "C1"):
+@pytest.mark.parametrize("geom", ["1,1,1,2", "1,4,2,2", "3,3,2,3", "8,4,8,4", "16,2,8,3"])
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_wave_geometries(gpu, geom, dtype, monkeypatch):
+    """The strand wavefront at several cluster geometries (SPTRSV_WAVE =
+    CTAs,warps,groups-per-chunk,ring-depth): one strand, one CTA, odd
+    shapes, the default 8x4 and a non-portable 16-CTA cluster."""
+    monkeypatch.setenv("SPTRSV_WAVE", geom)
+    for name in ("C2", "C5", "C1"):
+        M, b = g.gen_config(name, small=True, nrhs=1)
+        x, plan = _solve(M, b, dtype=dtype, depth=1, force_tri_impl="TRI_PIPE", reorder=True)
+        assert all(s["impl"] == "TRI_PIPE" for s in plan.segments() if s["kind"] == "TRI" and s["nlevels"] > 1)
+        if dtype == torch.float64:
+            _check64(M, b, x)
+        else:
+            assert on.rel_err(x, on.solve(M, b)) <= TOL32
+
+
+@pytest.mark.parametrize("hook", [("SPTRSV_WAVE_XW", "64"), ("SPTRSV_WAVE_ICAP", "0"), ("SPTRSV_WAVE_ICAP", "5")])
+def test_wave_global_fallbacks(gpu, hook, monkeypatch):
+    """Own-window and import-capacity overflow: those dependencies are polled
+    in global memory (value-as-flag) instead of shared memory."""
+    monkeypatch.setenv(*hook)
+    for name in ("C2", "C5"):
         M, b = g.gen_config(name, small=True, nrhs=1)
         x, plan = _solve(M, b, depth=1, force_tri_impl="TRI_PIPE", reorder=True)
         _check64(M, b, x)
+
+
+def test_wave_is_the_c2_default(gpu):
+    """C2 (2D stencil IC(0), narrow anti-diagonal levels) runs its triangles on
+    the wavefront by default, and nrhs > 1 on the same plan solves too."""
+    M, b = g.gen_config("C2", small=True, nrhs=3)
+    x, plan = _solve(M, b[:1], depth=1)
+    assert [s["impl"] for s in plan.segments() if s["kind"] == "TRI"] == ["TRI_PIPE", "TRI_PIPE"]
+    _check64(M, b[:1], x)
+    x3, _ = _solve(M, b, depth=1)
+    _check64(M, b, x3)
