@@ -408,7 +408,7 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
     int a, b2, c, d;
     if (std::sscanf(e, "%d,%d,%d,%d", &a, &b2, &c, &d) == 4 && a >= 1 && a <= 16 && b2 >= 1 && b2 <= 8 &&
         c >= 1 && c <= 32 && d >= 2 && d <= 4) {
-      C = a; W = b2; GPC = c; NCH = d;
+      C = a; W = b2; GPC = c <= 4 ? 4 : 8; NCH = d;
     }
   }
   auto give_up = [&]() {
@@ -419,7 +419,7 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   int K = 0;
   for (int r = 0; r < m; ++r) K = std::max(K, S.rp[r + 1] - S.rp[r]);
   if (m < 1 || K < 1 || K > 8) return give_up();
-  const int Kt = K <= 1 ? 1 : K <= 2 ? 2 : K <= 4 ? 4 : 8;
+  const int Kt = K <= 2 ? 2 : K <= 4 ? 4 : 8;
   while (C > 1 && (int64_t)C * W * 256 > m) --C;  // at least ~256 rows per strand
   const int NS = C * W;
   // strands by rank of the original row index
@@ -471,9 +471,9 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
     const int64_t rings = (int64_t)W * NCH * (k::wave_hdr_bytes(GPC) + (int64_t)GPC * gb2 + bring + 8);
     const int64_t slots_avail = (232448 - 512 - rings) / (int64_t)vb;
     icap = (slots_avail - 2) / W - XW;
-    if (icap >= 1024 || (GPC == 1 && NCH == 2)) break;
+    if (icap >= 1024 || (GPC == 4 && NCH == 2)) break;
     if (NCH > 2) --NCH;
-    else { GPC = std::max(1, GPC / 2); NCH = 4; }
+    else { GPC = 4; NCH = 4; }
   }
   if (const char* e = std::getenv("SPTRSV_WAVE_ICAP")) icap = std::min<int64_t>(icap, std::max(0, std::atoi(e)));
   if (icap < 0) return give_up();
@@ -545,19 +545,20 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   S.wave_data.assign(std::max<size_t>(total, 16), 0);
   size_t off = 0;
   const int r0 = I.row0;
-  auto word = [&](int e) -> uint32_t {
+  const uint32_t VB = (uint32_t)vb;
+  auto word = [&](int e) -> uint32_t {  // byte offset in the x area, or bit 31 | global row
     const Dep& d = dep[e];
-    if (d.kind == 0) return (uint32_t)(own_base[strand[d.a]] + (pos[d.a] & (XW - 1)));
-    if (d.kind == 1) return k::kWaveIMP | (uint32_t)(imp_base[d.a] + d.b);
-    return k::kWaveGLB | (uint32_t)(r0 + qpos[d.a]);
+    if (d.kind == 0) return (uint32_t)(own_base[strand[d.a]] + (pos[d.a] & (XW - 1))) * VB;
+    if (d.kind == 1) return (uint32_t)(imp_base[d.a] + d.b) * VB;
+    return 0x80000000u | (uint32_t)(r0 + qpos[d.a]);
   };
+  const int bshift_mask = vb == 8 ? 1 : 3;  // bw is 256-byte aligned: TMA window shift of row lo
   for (int s2 = 0; s2 < NS; ++s2) {
     k::WaveStrand& W2 = sr[s2];
     std::memset(&W2, 0, sizeof(W2));
     W2.off16 = (int)(off / 16);
     W2.nchunk = nchunk[s2];
     W2.ngroups = (int)groups[s2].size();
-    W2.own_base = own_base[s2];
     W2.row0 = r0 + s_start[s2];
     const auto& Gs = groups[s2];
     const auto& R = srows[s2];
@@ -572,18 +573,23 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
       chunk_rows(c, hdr[0], hdr[1]);
       if (c + NCH < nchunk[s2]) chunk_rows(c + NCH, hdr[2], hdr[3]);
       if (c < 4) chunk_rows(c, W2.lo[c], W2.hi[c]);
+      const int lo = hdr[0];
       for (int gi = 0; gi < GPC; ++gi) {
         const int g = c * GPC + gi;
-        int32_t* gh = (int32_t*)(B + 16) + 2 * gi;
+        int32_t* gh = (int32_t*)(B + 16) + 4 * gi;
         uint32_t* wd = (uint32_t*)(B + hbytes + (size_t)gi * gbytes);
-        uint32_t* pw = wd + 32 * Kt;
+        uint32_t* so = wd + 32 * Kt;
+        uint32_t* pw = so + 32;
         char* vv = (char*)(pw + 32 * E);
+        for (int l = 0; l < 32; ++l) so[l] = VB;  // sink slot (padding lanes)
         for (int l = 0; l < 32 * E; ++l) pw[l] = 0xffffffffu;
-        if (g >= (int)Gs.size()) continue;  // padding group (cnt 0, zero slots)
+        if (g >= (int)Gs.size()) continue;  // padding group: never executed
         int flags = 0;
         gh[0] = r0 + s_start[s2] + Gs[g].first;
+        gh[2] = gh[0] - lo + (lo & bshift_mask);
         for (int l = 0; l < Gs[g].second; ++l) {
           const int r = R[Gs[g].first + l];
+          so[l] = (uint32_t)(own_base[s2] + (pos[r] & (XW - 1))) * VB;
           int kk = 0;
           for (int e = S.rp[r]; e < S.rp[r + 1]; ++e, ++kk) {
             wd[kk * 32 + l] = word(e);
@@ -592,7 +598,7 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
           }
           for (int e2 = 0; e2 < npush[r]; ++e2) {
             const int cs = push[r][2 * e2], ci2 = push[r][2 * e2 + 1];
-            pw[e2 * 32 + l] = ((uint32_t)(cs / W) << 24) | (uint32_t)(imp_base[cs] + ci2);
+            pw[e2 * 32 + l] = ((uint32_t)(cs / W) << 24) | ((uint32_t)(imp_base[cs] + ci2) * VB);
             flags |= k::kWaveGF_PUSH;
           }
         }
@@ -619,16 +625,16 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   S.wave_global = nglobal;
 }
 
-template <typename T, int K, int E>
+template <typename T, int K, int E, int GPC, bool GLB>
 Error launch_wave_t(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
-  k::WaveGeom g{S.wave_W,           S.wave_GPC,         S.wave_NCH,         S.wave_XW,
-                S.wave_xa,          S.wave_chunk_bytes, S.wave_bring_bytes, S.wave_group_bytes,
-                k::wave_hdr_bytes(S.wave_GPC)};
+  k::WaveGeom g{S.wave_W,           S.wave_GPC,         S.wave_NCH,         S.wave_xa,
+                S.wave_chunk_bytes, S.wave_bring_bytes, S.wave_group_bytes, k::wave_hdr_bytes(S.wave_GPC)};
   const uint32_t smem = k::wave_smem_bytes<T>(g);
+  auto kern = k::tri_wave<T, K, E, GPC, GLB>;
   static uint32_t attr_bytes = 0;  // per template instance
   if (smem > attr_bytes) {
-    CUDA_TRY(cudaFuncSetAttribute(k::tri_wave<T, K, E>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    CUDA_TRY(cudaFuncSetAttribute(k::tri_wave<T, K, E>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+    CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
     attr_bytes = smem;
   }
   cudaLaunchConfig_t cfg = {};
@@ -651,24 +657,30 @@ Error launch_wave_t(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, c
     CUDA_TRY(cudaMemsetAsync(S.d_trace, 0, nt * 8, s));
     tr = (long long*)S.d_trace;
   }
-  CUDA_TRY(cudaLaunchKernelEx(&cfg, k::tri_wave<T, K, E>, (const k::WaveStrand*)S.d_wave_strands, S.d_wave_data, bw,
-                              xs, g, st, tr));
+  CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, (const k::WaveStrand*)S.d_wave_strands, S.d_wave_data, bw, xs, g, st, tr));
   return {SPTRSV_SUCCESS, ""};
+}
+
+template <typename T, int K, int E>
+Error launch_wave_e(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
+  const bool glb = S.wave_global > 0;
+  if (S.wave_GPC == 4)
+    return glb ? launch_wave_t<T, K, E, 4, true>(p, S, bw, xs, st, s) : launch_wave_t<T, K, E, 4, false>(p, S, bw, xs, st, s);
+  return glb ? launch_wave_t<T, K, E, 8, true>(p, S, bw, xs, st, s) : launch_wave_t<T, K, E, 8, false>(p, S, bw, xs, st, s);
 }
 
 template <typename T, int K>
 Error launch_wave_k(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
   switch (S.wave_E) {
-    case 0: return launch_wave_t<T, K, 0>(p, S, bw, xs, st, s);
-    case 1: return launch_wave_t<T, K, 1>(p, S, bw, xs, st, s);
-    default: return launch_wave_t<T, K, 2>(p, S, bw, xs, st, s);
+    case 0: return launch_wave_e<T, K, 0>(p, S, bw, xs, st, s);
+    case 1: return launch_wave_e<T, K, 1>(p, S, bw, xs, st, s);
+    default: return launch_wave_e<T, K, 2>(p, S, bw, xs, st, s);
   }
 }
 
 template <typename T>
 Error launch_wave(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
   switch (S.wave_K) {
-    case 1: return launch_wave_k<T, 1>(p, S, bw, xs, st, s);
     case 2: return launch_wave_k<T, 2>(p, S, bw, xs, st, s);
     case 4: return launch_wave_k<T, 4>(p, S, bw, xs, st, s);
     default: return launch_wave_k<T, 8>(p, S, bw, xs, st, s);

@@ -1205,40 +1205,52 @@ __global__ void __launch_bounds__(1024, 1)
 // c + NCH, so no control word is read from global memory inside the loop.
 //
 // Chunk block: int4 {row_lo, row_hi, next_lo, next_hi} (b' rows of this chunk
-// and of chunk c + NCH), int2 {row_start, cnt | flags} per group (GPC, padded
-// to 16 bytes), then GPC group blocks {u32 words[K][32], u32 push[E][32],
+// and of chunk c + NCH), one int4 {row_start, cnt | flags, boff, -} per group
+// (boff: index of the group's first b' value in the chunk's b' window), then
+// GPC group blocks {u32 xoff[K][32], u32 soff[32], u32 push[E][32],
 // T vals[K][32]}.
-// word: bit 31 clear = slot (in T units) of the CTA's x area; set = global
-// (execution-order) row of xs.  push: (cta rank << 24) | slot, ~0u = none.
-// Group flags (high bits of cnt): GF_GLOBAL = a lane has a global word,
-// GF_PUSH = a lane pushes.  A group with cnt == 0 is padding.
+//   xoff: BYTE offset in the CTA's x area of the dependency (own-window or
+//         import slot; padding: the zero slot at byte 0).  In a group flagged
+//         GF_GLOBAL: bit 31 set = execution-order row of xs polled in global
+//         memory instead.
+//   soff: byte offset of the row's own-window slot (padding lanes: the sink
+//         slot at byte 8).
+//   push: (cta rank << 24) | byte offset of an import slot of a consumer
+//         strand, ~0u = none.
 //
-// Single-warp critical path per group (the level chain of the strand):
-// __syncwarp -> LDS x_j -> sentinel vote -> 2 x DFMA -> STS x_i.  Everything
-// else (the next group's operands, the TMA ring, the global store and the
-// pushes) is issued in the shadow of that chain: the loop is software-
-// pipelined by one group (round-1 trace: a straightforward loop spent ~700
-// cycles per group in dependent address/branch latency of one warp).
+// The loop (one warp = one strand) keeps only this on the level chain:
+//   __syncwarp -> LDS x_j -> 2 x DFMA -> STS x_i
+// (single-warp microbenchmark: ~51 cycles, scripts/microbench/wave_loop.cu).
+// Everything else is off it: the next group's operands are loaded during the
+// current group, and so is a first poll of its dependencies -- the readiness
+// test of other-strand values (import slots start as the sentinel) is made on
+// that early poll, so no branch waits on a fresh load (the microbenchmark
+// measured +65..90 cycles per group for any test of a just-loaded x).  The
+// value loaded at use time is always ready: own-strand values were stored by
+// this warp before the last __syncwarp, imports passed the early test (an
+// import slot is written once).  An early poll that still sees the sentinel
+// (producer strand behind; or, in a strand's first XW rows, an own slot not
+// yet written) sends the warp to the wait loop.
 constexpr int kWaveGF_GLOBAL = 1 << 30, kWaveGF_PUSH = 1 << 29, kWaveCntMask = (1 << 29) - 1;
 struct WaveStrand {
-  int off16, nchunk, own_base, row0;  // row0: first execution-order row of the strand
-  int lo[4], hi[4];                   // b' row ranges of chunks 0..3 (the prologue loads)
-  int ngroups, pad[3];
+  int off16, nchunk, ngroups, row0;  // row0: first execution-order row of the strand
+  int lo[4], hi[4];                  // b' row ranges of chunks 0..3 (the prologue loads)
 };
 struct WaveGeom {
-  int W, GPC, NCH, XW;   // warps per CTA, groups per chunk, ring depth, own window
-  int xa_slots;          // x area slots per CTA
+  int W, GPC, NCH, xa_slots;  // warps per CTA, groups per chunk, ring depth, x area slots per CTA
   uint32_t chunk_bytes, bring_bytes, group_bytes, hdr_bytes;
 };
 
 template <typename T>
 __host__ __device__ inline uint32_t wave_group_bytes(int K, int E) {
-  return 128u * (uint32_t)K + 128u * (uint32_t)E + 32u * (uint32_t)K * (uint32_t)sizeof(T);
+  return 128u * (uint32_t)K + 128u + 128u * (uint32_t)E + 32u * (uint32_t)K * (uint32_t)sizeof(T);
 }
-__host__ __device__ inline uint32_t wave_hdr_bytes(int GPC) { return 16u + al16(8u * (uint32_t)GPC); }
+__host__ __device__ inline uint32_t wave_hdr_bytes(int GPC) { return 16u + 16u * (uint32_t)GPC; }
 template <typename T>
 __host__ __device__ inline uint32_t wave_bring_bytes(int GPC) {
-  return al16((uint32_t)GPC * 32u * (uint32_t)sizeof(T) + 32u);
+  // + 32 rows of slack: padding lanes of a chunk's last group read (and
+  // discard) past the window
+  return al16((uint32_t)GPC * 32u * (uint32_t)sizeof(T) + 32u) + 32u * (uint32_t)sizeof(T);
 }
 template <typename T>
 __host__ __device__ inline uint32_t wave_smem_bytes(const WaveGeom& g) {
@@ -1253,17 +1265,6 @@ __device__ __forceinline__ uint32_t cluster_ctarank() {
 }
 __device__ __forceinline__ void cluster_sync_all() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-__device__ __forceinline__ uint32_t mapa_shared(uint32_t a, uint32_t rank) {
-  uint32_t r;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(rank));
-  return r;
-}
-__device__ __forceinline__ void st_cluster(uint32_t a, double v) {
-  asm volatile("st.relaxed.cluster.shared::cluster.f64 [%0], %1;" ::"r"(a), "d"(v) : "memory");
-}
-__device__ __forceinline__ void st_cluster(uint32_t a, float v) {
-  asm volatile("st.relaxed.cluster.shared::cluster.f32 [%0], %1;" ::"r"(a), "f"(v) : "memory");
 }
 // x loads / stores of the wave loop: volatile (never cached or dropped) and
 // ordered among themselves, but without a "memory" clobber so the compiler
@@ -1300,28 +1301,59 @@ __device__ __forceinline__ void stg_x_v(double* p, double v) {
 __device__ __forceinline__ void stg_x_v(float* p, float v) {
   asm volatile("st.relaxed.gpu.global.f32 [%0], %1;" ::"l"(p), "f"(v));
 }
+// push x into a consumer strand's import slot (DSMEM), unless p == ~0u
+__device__ __forceinline__ void wave_push(uint32_t p, uint32_t xa_s, double v) {
+  asm volatile(
+      "{\n .reg .pred q;\n .reg .b32 ra;\n setp.ne.u32 q, %0, -1;\n"
+      " @q mapa.shared::cluster.u32 ra, %1, %2;\n @q st.relaxed.cluster.shared::cluster.f64 [ra], %3;\n}\n" ::"r"(p),
+      "r"(xa_s + (p & 0xffffffu)), "r"(p >> 24), "d"(v)
+      : "memory");
+}
+__device__ __forceinline__ void wave_push(uint32_t p, uint32_t xa_s, float v) {
+  asm volatile(
+      "{\n .reg .pred q;\n .reg .b32 ra;\n setp.ne.u32 q, %0, -1;\n"
+      " @q mapa.shared::cluster.u32 ra, %1, %2;\n @q st.relaxed.cluster.shared::cluster.f32 [ra], %3;\n}\n" ::"r"(p),
+      "r"(xa_s + (p & 0xffffffu)), "r"(p >> 24), "f"(v)
+      : "memory");
+}
+// "might be the sentinel": the high word only (exact test in the wait loop)
+__device__ __forceinline__ bool maybe_sent(double v) { return __double2hiint(v) == 0x7FF40000; }
+__device__ __forceinline__ bool maybe_sent(float v) { return __float_as_uint(v) == 0x7FA00BADu; }
 
 template <typename T, int K, int E>
 struct WaveOp {
-  uint32_t w[K];  // words (own slot, import slot | WAVE_IMP, global row | WAVE_GLB)
-  T v[K];
-  T xi[K];        // import / global operands, polled one group ahead
-  T b;
-  int row, cnt;   // cnt with the group flags
+  uint32_t xo[K], so;
   uint32_t push[E > 0 ? E : 1];
+  T v[K];
+  T xe[K];  // early poll of the dependencies (readiness test only)
+  T b;
+  int row, cnt;  // cnt with the group flags
 };
-constexpr uint32_t kWaveGLB = 0x80000000u, kWaveIMP = 0x40000000u, kWaveIdx = 0x3fffffffu;
 
-template <typename T, int K, int E>
+__device__ __forceinline__ void warp_sync_all() { asm volatile("bar.warp.sync -1;" ::: "memory"); }
+__device__ __forceinline__ bool vote_any(bool p) {
+  uint32_t r;
+  asm volatile("{\n .reg .pred q, r;\n setp.ne.u32 q, %1, 0;\n vote.sync.any.pred r, q, -1;\n selp.u32 %0, 1, 0, r;\n}\n"
+               : "=r"(r)
+               : "r"((uint32_t)p));
+  return r != 0;
+}
+
+// GPC (groups per chunk, even) is a template parameter so the group loop of
+// a chunk is fully unrolled: the operand sets alternate between two register
+// sets without copies, the chunk switch happens only at the last group, and
+// padding groups (cnt 0: zero-slot operands, sink store, no global store, no
+// push) execute as no-ops instead of being branched around.  GLB: some group
+// polls xs in global memory (window / import overflow).
+template <typename T, int K, int E, int GPC, bool GLB>
 __global__ void __launch_bounds__(256, 1)
     tri_wave(const WaveStrand* __restrict__ strands, const char* __restrict__ data, const T* __restrict__ bw,
              T* __restrict__ xs, WaveGeom g, SolveState st, long long* __restrict__ trace) {
   extern __shared__ __align__(128) unsigned char smem[];
-  constexpr uint32_t SH = sizeof(T) == 8 ? 3 : 2;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const uint32_t rank = cluster_ctarank();
   const WaveStrand* Sp = strands + rank * g.W + warp;
-  const int s_nchunk = Sp->nchunk, s_ng = Sp->ngroups, s_own = Sp->own_base, s_row0 = Sp->row0;
+  const int s_nchunk = Sp->nchunk;
   const char* s_data = data + (size_t)Sp->off16 * 16;
   long long* tr = trace ? trace + (size_t)(rank * g.W + warp) * 8 : nullptr;
   if (tr && lane == 0) tr[0] = clock64();
@@ -1332,8 +1364,8 @@ __global__ void __launch_bounds__(256, 1)
   uint64_t* full = (uint64_t*)(bring + (size_t)(g.W * g.NCH) * g.bring_bytes) + warp * g.NCH;
   ring += (size_t)warp * g.NCH * g.chunk_bytes;
   bring += (size_t)warp * g.NCH * g.bring_bytes;
-  // x area: two zero slots (padding dependencies), the rest the sentinel
-  // (import slots must read "not ready" until pushed)
+  // x area: slot 0 zero (padding dependencies), slot 1 sink (padding lanes'
+  // stores), the rest the sentinel (import slots read "not ready" until pushed)
   for (int i = tid; i < g.xa_slots; i += blockDim.x) xa[i] = i < 2 ? T(0) : sent<T>();
   if (lane == 0)
     for (int c = 0; c < g.NCH; ++c) mbar_init(&full[c], 1);
@@ -1351,121 +1383,121 @@ __global__ void __launch_bounds__(256, 1)
     for (int c = 0; c < g.NCH && c < s_nchunk; ++c) issue_chunk(c, c, Sp->lo[c], Sp->hi[c]);
   if (tr && lane == 0) tr[1] = clock64();
 
-  const uint32_t xmask = (uint32_t)g.XW - 1;
   uint32_t spins = 0, npolls = 0;
-  // position of the NEXT group: chunk c_n (ring slot `slot`, phase `ph`),
-  // index gi_n inside it; B_n / bb_n: that chunk's block and b' base
-  int slot = 0, c_n = 0, gi_n = 0;
-  uint32_t ph = 0;
-  const unsigned char* B_n = ring;
-  const T* bb_n = nullptr;
-  auto enter_chunk = [&]() {
-    mbar_wait(&full[slot], ph);
-    B_n = ring + (size_t)slot * g.chunk_bytes;
-    const int lo = *(const int*)B_n;
-    bb_n = (const T*)(bring + (size_t)slot * g.bring_bytes) + shift_of(bw, (int64_t)lo) - lo;
-  };
-  auto load_op = [&](WaveOp<T, K, E>& o) {
-    const int2 gh = ((const int2*)(B_n + 16))[gi_n];
-    const uint32_t* wd = (const uint32_t*)(B_n + g.hdr_bytes + (uint32_t)gi_n * g.group_bytes);
-    const T* vv = (const T*)(wd + 32 * (K + E));
+  auto load_op = [&](const unsigned char* B, const T* bb, int gi, WaveOp<T, K, E>& o) {
+    const int4 gh = ((const int4*)(B + 16))[gi];
+    const uint32_t* wd = (const uint32_t*)(B + g.hdr_bytes + (uint32_t)gi * g.group_bytes);
+    const T* vv = (const T*)(wd + 32 * (K + 1 + E));
 #pragma unroll
-    for (int k2 = 0; k2 < K; ++k2) {
-      o.w[k2] = wd[k2 * 32 + lane];
-      o.v[k2] = vv[k2 * 32 + lane];
-    }
+    for (int k2 = 0; k2 < K; ++k2) o.xo[k2] = wd[k2 * 32 + lane];
+    o.so = wd[K * 32 + lane];
 #pragma unroll
-    for (int e = 0; e < E; ++e) o.push[e] = wd[(K + e) * 32 + lane];
+    for (int e = 0; e < E; ++e) o.push[e] = wd[(K + 1 + e) * 32 + lane];
+#pragma unroll
+    for (int k2 = 0; k2 < K; ++k2) o.v[k2] = vv[k2 * 32 + lane];
+    o.b = bb[gh.z + lane];
     o.row = gh.x + lane;
     o.cnt = gh.y;
-    o.b = lane < (gh.y & kWaveCntMask) ? bb_n[o.row] : T(0);
-    // dependencies on OTHER strands are polled now, a group ahead of use, so
-    // their readiness test is off the level chain
+    if (!GLB) {
 #pragma unroll
-    for (int k2 = 0; k2 < K; ++k2)
-      o.xi[k2] = (o.w[k2] & kWaveGLB)   ? ldg_x_v(xs + (o.w[k2] & kWaveIdx))
-                 : (o.w[k2] & kWaveIMP) ? lds_x_v(xa_s + ((o.w[k2] & kWaveIdx) << SH), T(0))
-                                        : T(0);
+      for (int k2 = 0; k2 < K; ++k2) o.xe[k2] = lds_x_v(xa_s + o.xo[k2], T(0));
+    }
   };
-
-  WaveOp<T, K, E> nxt;
-  if (s_ng > 0) {
-    enter_chunk();
-    load_op(nxt);
-  }
-  for (int gidx = 0; gidx < s_ng; ++gidx) {
-    WaveOp<T, K, E> cur = nxt;
-    const bool act = lane < (cur.cnt & kWaveCntMask);
-    // ---- other-strand operands: normally ready since the last group
-    bool pend = false;
+  // the level-chain part of one group (cur resident)
+  auto solve_op = [&](WaveOp<T, K, E>& cur) -> T {
+    T x[K];
+    if (!GLB) {
+      bool pend = false;
 #pragma unroll
-    for (int k2 = 0; k2 < K; ++k2) pend |= (cur.w[k2] & (kWaveGLB | kWaveIMP)) && is_sent(cur.xi[k2]);
-    if (__any_sync(0xffffffffu, pend)) {  // a producer strand is behind: wait for it
-      while (__any_sync(0xffffffffu, pend)) {
-        ++npolls;
-        pend = false;
+      for (int k2 = 0; k2 < K; ++k2) pend |= maybe_sent(cur.xe[k2]);
+      if (vote_any(pend)) {  // a producer strand is behind: wait for it
+        for (;;) {
+          pend = false;
 #pragma unroll
-        for (int k2 = 0; k2 < K; ++k2) {
-          if ((cur.w[k2] & (kWaveGLB | kWaveIMP)) && is_sent(cur.xi[k2])) {
-            cur.xi[k2] = (cur.w[k2] & kWaveGLB) ? ldg_x_v(xs + (cur.w[k2] & kWaveIdx))
-                                                : lds_x_v(xa_s + ((cur.w[k2] & kWaveIdx) << SH), T(0));
-            pend |= is_sent(cur.xi[k2]);
+          for (int k2 = 0; k2 < K; ++k2) pend |= is_sent(lds_x_v(xa_s + cur.xo[k2], T(0)));
+          if (!vote_any(pend)) break;
+          ++npolls;
+          if (++spins > kWatchdogSpins) {
+            watchdog_trip(st);
+            break;
           }
         }
-        if (pend && ++spins > kWatchdogSpins) {
-          watchdog_trip(st);
+      }
+      // ---- level chain: every value is ready now
 #pragma unroll
-          for (int k2 = 0; k2 < K; ++k2) cur.xi[k2] = is_sent(cur.xi[k2]) ? T(0) : cur.xi[k2];
-          pend = false;
+      for (int k2 = 0; k2 < K; ++k2) x[k2] = lds_x_v(xa_s + cur.xo[k2], T(0));
+    } else {
+#pragma unroll
+      for (int k2 = 0; k2 < K; ++k2) {
+        const bool glb = cur.xo[k2] & 0x80000000u;
+        for (;;) {
+          x[k2] = glb ? ldg_x_v(xs + (cur.xo[k2] & 0x7fffffffu)) : lds_x_v(xa_s + cur.xo[k2], T(0));
+          if (!is_sent(x[k2])) break;
+          ++npolls;
+          if (++spins > kWatchdogSpins) {
+            watchdog_trip(st);
+            x[k2] = T(0);
+            break;
+          }
         }
       }
-    }
-    // ---- critical chain: own-strand x_j (written by this warp before the
-    // last __syncwarp: always ready, no test)
-    T x[K];
-#pragma unroll
-    for (int k2 = 0; k2 < K; ++k2)
-      x[k2] = (cur.w[k2] & (kWaveGLB | kWaveIMP)) ? cur.xi[k2] : lds_x_v(xa_s + (cur.w[k2] << SH), T(0));
-    // ---- prefetch the next group's operands in the shadow of the loads
-    int refill_slot = -1, refill_c = 0;
-    if (gidx + 1 < s_ng) {
-      if (++gi_n == g.GPC) {  // next group opens a new chunk: the current one
-        gi_n = 0;             // is consumed once this group is done
-        refill_slot = slot;
-        refill_c = c_n;
-        ++c_n;
-        if (++slot == g.NCH) {
-          slot = 0;
-          ph ^= 1u;
-        }
-        enter_chunk();
-      }
-      load_op(nxt);
     }
     T acc = cur.b;
 #pragma unroll
     for (int k2 = 0; k2 < K; ++k2) acc = fma(-cur.v[k2], x[k2], acc);
-    if (act) {
-      sts_x_v(xa_s + ((uint32_t)(s_own + ((uint32_t)(cur.row - s_row0) & xmask)) << SH), acc);
-      if (E > 0 && (cur.cnt & kWaveGF_PUSH)) {
+    return acc;
+  };
+  auto publish = [&](WaveOp<T, K, E>& cur, T acc) {
+    sts_x_v(xa_s + cur.so, acc);
 #pragma unroll
-        for (int e = 0; e < E; ++e)
-          if (cur.push[e] != 0xffffffffu)
-            st_cluster(mapa_shared(xa_s + ((cur.push[e] & 0xffffffu) << SH), cur.push[e] >> 24), acc);
+    for (int e = 0; e < E; ++e) wave_push(cur.push[e], xa_s, acc);
+    if (lane < (cur.cnt & kWaveCntMask)) stg_x_v(xs + cur.row, acc);
+  };
+
+  WaveOp<T, K, E> opA, opB;
+  int slot = 0;
+  uint32_t ph = 0;
+  const unsigned char* B = ring;
+  const T* bb = (const T*)bring;
+  if (s_nchunk > 0) {
+    mbar_wait(&full[0], 0);
+    load_op(B, bb, 0, opA);
+  }
+  for (int c = 0; c < s_nchunk; ++c) {
+#pragma unroll
+    for (int gi = 0; gi < GPC; ++gi) {
+      WaveOp<T, K, E>& cur = (gi & 1) ? opB : opA;
+      WaveOp<T, K, E>& nxt = (gi & 1) ? opA : opB;
+      if (gi + 1 < GPC) {
+        const T acc = solve_op(cur);
+        load_op(B, bb, gi + 1, nxt);  // in the shadow of the x loads / DFMAs
+        publish(cur, acc);
+      } else {  // last group of the chunk: open the next chunk, recycle this one
+        const T acc = solve_op(cur);
+        const int cur_slot = slot;
+        if (c + 1 < s_nchunk) {
+          if (++slot == g.NCH) {
+            slot = 0;
+            ph ^= 1u;
+          }
+          mbar_wait(&full[slot], ph);
+          B = ring + (size_t)slot * g.chunk_bytes;
+          bb = (const T*)(bring + (size_t)slot * g.bring_bytes);
+          load_op(B, bb, 0, nxt);
+        }
+        publish(cur, acc);
+        if (lane == 0 && c + g.NCH < s_nchunk) {
+          const int4 hdr = *(const int4*)(ring + (size_t)cur_slot * g.chunk_bytes);
+          issue_chunk(cur_slot, c + g.NCH, hdr.z, hdr.w);
+        }
       }
-      stg_x_v(xs + cur.row, acc);
+      warp_sync_all();
     }
-    if (refill_slot >= 0 && lane == 0 && refill_c + g.NCH < s_nchunk) {
-      // every operand of chunk refill_c is consumed: reuse its ring slot
-      const int4 hdr = *(const int4*)(ring + (size_t)refill_slot * g.chunk_bytes);
-      issue_chunk(refill_slot, refill_c + g.NCH, hdr.z, hdr.w);
-    }
-    __syncwarp();
   }
   if (tr && lane == 0) {
     tr[2] = clock64();
     tr[3] = npolls;
-    tr[4] = s_ng;
+    tr[4] = s_nchunk * GPC;
   }
   __syncthreads();
   cluster_sync_all();  // no CTA leaves while a peer may still push into it
