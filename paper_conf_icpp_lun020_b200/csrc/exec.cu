@@ -400,10 +400,11 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   S.wave_tau.clear();
   S.wave_strands.clear();
   S.wave_data.clear();
+  S.wave_crows.clear();
   auto& I = S.info;
   if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_PIPE) return;
   const int m = I.row1 - I.row0;
-  int C = 8, W = 4, GPC = 8, NCH = 4;
+  int C = 16, W = 4, GPC = 8, NCH = 4;
   if (const char* e = std::getenv("SPTRSV_WAVE")) {
     int a, b2, c, d;
     if (std::sscanf(e, "%d,%d,%d,%d", &a, &b2, &c, &d) == 4 && a >= 1 && a <= 16 && b2 >= 1 && b2 <= 8 &&
@@ -420,14 +421,48 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   for (int r = 0; r < m; ++r) K = std::max(K, S.rp[r + 1] - S.rp[r]);
   if (m < 1 || K < 1 || K > 8) return give_up();
   const int Kt = K <= 2 ? 2 : K <= 4 ? 4 : 8;
-  while (C > 1 && (int64_t)C * W * 256 > m) --C;  // at least ~256 rows per strand
-  const int NS = C * W;
-  // strands by rank of the original row index
+  // strands: contiguous runs of the original row index, cut so that no
+  // strand holds more than `cap` rows of one level (cap = 32: one group per
+  // level and strand).  A strand then needs one level step per level it
+  // spans, and a strand that starts late (its rows sit in late levels) is
+  // short: the critical path is ~ the number of levels, not the widest
+  // strand's row count (equal-row strands made the last strands of C2's
+  // anti-diagonal triangles 3-6 groups per level).  cap grows by 32 until
+  // the strands fit the cluster (C_max x W warps).
   std::vector<int32_t> order(m), strand(m);
   std::iota(order.begin(), order.end(), 0);
   std::stable_sort(order.begin(), order.end(),
                    [&](int a, int b2) { return p.lower_old[I.row0 + a] < p.lower_old[I.row0 + b2]; });
-  for (int q = 0; q < m; ++q) strand[order[q]] = (int)((int64_t)q * NS / m);
+  const int C_max = C;
+  int NS = 0;
+  {
+    std::vector<int32_t> lvcnt(std::max(1, I.nlevels) + 1, 0), touched;
+    for (int cap = 32;; cap += 32) {
+      NS = 0;
+      int cur = 0;
+      for (int q = 0; q < m; ++q) {
+        const int r = order[q];
+        const int lv = p.leaf_level[I.row0 + r];
+        if (q == 0 || lvcnt[lv] + 1 > cap) {  // open a new strand
+          for (int t : touched) lvcnt[t] = 0;
+          touched.clear();
+          cur = NS++;
+        }
+        if (lvcnt[lv]++ == 0) touched.push_back(lv);
+        strand[r] = cur;
+      }
+      for (int t : touched) lvcnt[t] = 0;
+      touched.clear();
+      if (NS <= C_max * W) break;
+    }
+  }
+  C = std::max(1, (NS + W - 1) / W);
+  if (const char* e = std::getenv("SPTRSV_WAVE_EQUAL")) {  // tuning: the old equal-row strands
+    NS = C_max * W;
+    C = C_max;
+    for (int q = 0; q < m; ++q) strand[order[q]] = (int)((int64_t)q * NS / m);
+  }
+  NS = C * W;  // trailing strands of the last CTA stay empty
   // rows of every strand in level order (= local row order); groups
   std::vector<std::vector<int32_t>> srows(NS);
   for (int r = 0; r < m; ++r) srows[strand[r]].push_back(r);
@@ -468,7 +503,7 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   int64_t icap = -1;
   for (;;) {
     bring = vb == 8 ? k::wave_bring_bytes<double>(GPC) : k::wave_bring_bytes<float>(GPC);
-    const int64_t rings = (int64_t)W * NCH * (k::wave_hdr_bytes(GPC) + (int64_t)GPC * gb2 + bring + 8);
+    const int64_t rings = (int64_t)W * NCH * (k::wave_hdr_bytes(GPC) + (int64_t)GPC * gb2 + bring + 16);
     const int64_t slots_avail = (232448 - 512 - rings) / (int64_t)vb;
     icap = (slots_avail - 2) / W - XW;
     if (icap >= 1024 || (GPC == 4 && NCH == 2)) break;
@@ -639,7 +674,7 @@ Error launch_wave_t(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, c
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(S.wave_C);
-  cfg.blockDim = dim3(32 * S.wave_W);
+  cfg.blockDim = dim3(32 * (S.wave_W + 1));  // + the TMA producer warp
   cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
   cudaLaunchAttribute at[1];
@@ -651,7 +686,7 @@ Error launch_wave_t(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, c
   cfg.numAttrs = 1;
   long long* tr = nullptr;
   if (p.trace) {  // debug: SPTRSV_TRACE=1, per-strand clock64 stamps
-    const size_t nt = (size_t)S.wave_C * S.wave_W * 8;
+    const size_t nt = (size_t)S.wave_C * S.wave_W * 1024;
     if (S.h_trace.size() < nt) S.h_trace.assign(nt, 0);
     if (!S.d_trace) CUDA_TRY(cudaMalloc(&S.d_trace, nt * 8));
     CUDA_TRY(cudaMemsetAsync(S.d_trace, 0, nt * 8, s));
@@ -875,7 +910,7 @@ void dump_trace(Plan& p, cudaStream_t s) {
     Segment& S = p.segs[si];
     if (!S.d_trace) continue;
     if (S.wave_K > 0) {  // raw per-strand stamps -> $SPTRSV_TRACE_DIR/wave_seg<i>.bin
-      const size_t nt = (size_t)S.wave_C * S.wave_W * 8;
+      const size_t nt = (size_t)S.wave_C * S.wave_W * 1024;
       cudaMemcpy(S.h_trace.data(), S.d_trace, nt * 8, cudaMemcpyDeviceToHost);
       const char* dir = std::getenv("SPTRSV_TRACE_DIR");
       std::string path = std::string(dir ? dir : ".") + "/wave_seg" + std::to_string(si) + ".bin";
@@ -1012,7 +1047,7 @@ Error upload(Plan& p, void* stream_v) {
   };
   size_t o_perm = take((size_t)2 * n * 4);  // perm (new->old) then iperm (old->new)
   size_t o_rdiag = take((size_t)n * vb);
-  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed, sd, sc, sv, sbk, ps, pd; };
+  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed, sd, sc, sv, sbk, ps, pd, pc; };
   std::vector<Offs> so(p.segs.size());
   p.trace = std::getenv("SPTRSV_TRACE") != nullptr;
   p.spmm = spmm_cfg();
@@ -1101,6 +1136,7 @@ Error upload(Plan& p, void* stream_v) {
     so[i].sbk = take(S.sn_blk.size());
     so[i].ps = take(S.wave_strands.size());
     so[i].pd = take(S.wave_data.size());
+    so[i].pc = take(S.wave_crows.size() * 4);
     if (S.info.kind == 0) S.ticket_slot = p.nticket++;
     if (S.info.kind == 0 && (S.info.impl == SPTRSV_IMPL_TRI_SYNCFREE || S.info.impl == SPTRSV_IMPL_TRI_SUPERNODE ||
                              (S.info.impl == SPTRSV_IMPL_TRI_PIPE && (S.wave_K == 0 || S.wave_global > 0))))
@@ -1166,6 +1202,8 @@ Error upload(Plan& p, void* stream_v) {
     std::memcpy(&h[so[i].pd], S.wave_data.data(), S.wave_data.size());
     S.d_wave_strands = (const void*)(A + so[i].ps);
     S.d_wave_data = (const char*)(A + so[i].pd);
+    std::memcpy(&h[so[i].pc], S.wave_crows.data(), S.wave_crows.size() * 4);
+    S.d_wave_crows = (const int32_t*)(A + so[i].pc);
   }
   p.d_perm = (const int32_t*)(A + o_perm);
   p.d_rdiag = (const void*)(A + o_rdiag);

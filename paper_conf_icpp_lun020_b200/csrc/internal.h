@@ -58,6 +58,8 @@ struct Segment {
   std::vector<int32_t> wave_tau;   // execution position q -> local row (the device row order of the triangle)
   std::vector<char> wave_strands;  // k::WaveStrand[C * W]
   std::vector<char> wave_data;     // chunk blocks
+  std::vector<int32_t> wave_crows; // {lo, hi} b' rows of every chunk (the producer warp's TMA windows)
+  const int32_t* d_wave_crows = nullptr;
   const void* d_wave_strands = nullptr;
   const char* d_wave_data = nullptr;
   // device-side square format: a CSR square whose rows are reordered by a

@@ -1255,7 +1255,7 @@ __host__ __device__ inline uint32_t wave_bring_bytes(int GPC) {
 template <typename T>
 __host__ __device__ inline uint32_t wave_smem_bytes(const WaveGeom& g) {
   return al16((uint32_t)g.xa_slots * (uint32_t)sizeof(T)) +
-         (uint32_t)(g.W * g.NCH) * (g.chunk_bytes + g.bring_bytes) + (uint32_t)(g.W * g.NCH) * 8u;
+         (uint32_t)(g.W * g.NCH) * (g.chunk_bytes + g.bring_bytes) + (uint32_t)(g.W * g.NCH) * 16u;
 }
 
 __device__ __forceinline__ uint32_t cluster_ctarank() {
@@ -1345,42 +1345,101 @@ __device__ __forceinline__ bool vote_any(bool p) {
 // padding groups (cnt 0: zero-slot operands, sink store, no global store, no
 // push) execute as no-ops instead of being branched around.  GLB: some group
 // polls xs in global memory (window / import overflow).
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+  uint32_t done;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+      : "=r"(done)
+      : "r"(smem_addr(bar)), "r"(parity)
+      : "memory");
+  return done != 0;
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
+}
+
+// Block = W consumer warps (one strand each) + one producer warp that keeps
+// every strand's ring of NCH chunks filled by TMA (full / empty mbarriers),
+// so a consumer never issues a copy: at a chunk end it only arrives on the
+// slot's empty barrier and waits on the next slot's full barrier.
 template <typename T, int K, int E, int GPC, bool GLB>
-__global__ void __launch_bounds__(256, 1)
-    tri_wave(const WaveStrand* __restrict__ strands, const char* __restrict__ data, const T* __restrict__ bw,
-             T* __restrict__ xs, WaveGeom g, SolveState st, long long* __restrict__ trace) {
+__global__ void __launch_bounds__(288, 1)
+    tri_wave(const WaveStrand* __restrict__ strands, const char* __restrict__ data, const T* __restrict__ bw, T* __restrict__ xs, WaveGeom g, SolveState st, long long* __restrict__ trace) {
   extern __shared__ __align__(128) unsigned char smem[];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const uint32_t rank = cluster_ctarank();
-  const WaveStrand* Sp = strands + rank * g.W + warp;
-  const int s_nchunk = Sp->nchunk;
-  const char* s_data = data + (size_t)Sp->off16 * 16;
-  long long* tr = trace ? trace + (size_t)(rank * g.W + warp) * 8 : nullptr;
-  if (tr && lane == 0) tr[0] = clock64();
   T* xa = (T*)smem;
   const uint32_t xa_s = smem_addr(smem);
-  unsigned char* ring = smem + al16((uint32_t)g.xa_slots * (uint32_t)sizeof(T));
-  unsigned char* bring = ring + (size_t)(g.W * g.NCH) * g.chunk_bytes;
-  uint64_t* full = (uint64_t*)(bring + (size_t)(g.W * g.NCH) * g.bring_bytes) + warp * g.NCH;
-  ring += (size_t)warp * g.NCH * g.chunk_bytes;
-  bring += (size_t)warp * g.NCH * g.bring_bytes;
+  unsigned char* ring0 = smem + al16((uint32_t)g.xa_slots * (uint32_t)sizeof(T));
+  unsigned char* bring0 = ring0 + (size_t)(g.W * g.NCH) * g.chunk_bytes;
+  uint64_t* full0 = (uint64_t*)(bring0 + (size_t)(g.W * g.NCH) * g.bring_bytes);
+  uint64_t* empty0 = full0 + g.W * g.NCH;
   // x area: slot 0 zero (padding dependencies), slot 1 sink (padding lanes'
   // stores), the rest the sentinel (import slots read "not ready" until pushed)
   for (int i = tid; i < g.xa_slots; i += blockDim.x) xa[i] = i < 2 ? T(0) : sent<T>();
-  if (lane == 0)
-    for (int c = 0; c < g.NCH; ++c) mbar_init(&full[c], 1);
+  if (tid == 0)
+    for (int c = 0; c < 2 * g.W * g.NCH; ++c) mbar_init(&full0[c], 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncthreads();
   cluster_sync_all();  // every import area is initialised before any push
 
-  auto issue_chunk = [&](int slot, int c, int lo, int hi) {
-    const Win wb = win(bw, (int64_t)lo, hi - lo);
-    mbar_expect_tx(&full[slot], g.chunk_bytes + wb.bytes);
-    tma_bulk_g2s(ring + (size_t)slot * g.chunk_bytes, s_data + (size_t)c * g.chunk_bytes, g.chunk_bytes, &full[slot]);
-    tma_bulk_g2s(bring + (size_t)slot * g.bring_bytes, wb.src, wb.bytes, &full[slot]);
-  };
-  if (lane == 0)
-    for (int c = 0; c < g.NCH && c < s_nchunk; ++c) issue_chunk(c, c, Sp->lo[c], Sp->hi[c]);
+  if (warp == g.W) {  // ---------------- producer warp: lane w feeds strand w
+    const int w = lane;
+    int nch = 0, c = 0, off16 = 0;
+    if (w < g.W) {
+      const WaveStrand* Sp = strands + rank * g.W + w;
+      nch = Sp->nchunk;
+      off16 = Sp->off16;
+    }
+    auto issue = [&](int cc, int lo, int hi) {
+      const int slot = cc % g.NCH;
+      const Win wb = win(bw, (int64_t)lo, hi - lo);
+      uint64_t* fb = &full0[w * g.NCH + slot];
+      mbar_expect_tx(fb, g.chunk_bytes + wb.bytes);
+      tma_bulk_g2s(ring0 + (size_t)(w * g.NCH + slot) * g.chunk_bytes,
+                   data + (size_t)off16 * 16 + (size_t)cc * g.chunk_bytes, g.chunk_bytes, fb);
+      tma_bulk_g2s(bring0 + (size_t)(w * g.NCH + slot) * g.bring_bytes, wb.src, wb.bytes, fb);
+    };
+    if (w < g.W) {
+      const WaveStrand* Sp = strands + rank * g.W + w;
+      for (; c < g.NCH && c < nch; ++c) issue(c, Sp->lo[c], Sp->hi[c]);
+    }
+    uint32_t idle = 0;
+    while (__any_sync(0xffffffffu, c < nch)) {
+      bool did = false;
+      if (c < nch) {
+        const int slot = c % g.NCH;
+        // chunk c reuses the slot of chunk c - NCH: wait for its release; the
+        // released block's header carries chunk c's b' row range
+        if (mbar_test(&empty0[w * g.NCH + slot], (uint32_t)(c / g.NCH - 1) & 1u)) {
+          const int4 hdr = *(const int4*)(ring0 + (size_t)(w * g.NCH + slot) * g.chunk_bytes);
+          issue(c, hdr.z, hdr.w);
+          ++c;
+          did = true;
+        }
+      }
+      if (!__any_sync(0xffffffffu, did)) {
+        __nanosleep(20);
+        if (++idle > (kWatchdogSpins >> 4)) {
+          if (lane == 0) watchdog_trip(st);
+          break;
+        }
+      }
+    }
+    __syncthreads();
+    cluster_sync_all();
+    return;
+  }
+
+  // ---------------- consumer warps
+  const WaveStrand* Sp = strands + rank * g.W + warp;
+  const int s_nchunk = Sp->nchunk;
+  long long* tr = trace ? trace + (size_t)(rank * g.W + warp) * 1024 : nullptr;
+  if (tr && lane == 0) tr[0] = clock64();
+  unsigned char* ring = ring0 + (size_t)warp * g.NCH * g.chunk_bytes;
+  unsigned char* bring = bring0 + (size_t)warp * g.NCH * g.bring_bytes;
+  uint64_t* full = full0 + warp * g.NCH;
+  uint64_t* empty = empty0 + warp * g.NCH;
   if (tr && lane == 0) tr[1] = clock64();
 
   uint32_t spins = 0, npolls = 0;
@@ -1468,13 +1527,21 @@ __global__ void __launch_bounds__(256, 1)
     for (int gi = 0; gi < GPC; ++gi) {
       WaveOp<T, K, E>& cur = (gi & 1) ? opB : opA;
       WaveOp<T, K, E>& nxt = (gi & 1) ? opA : opB;
+      if (tr && lane == 0 && c * GPC + gi < 1016) {
+        long long gt;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
+        tr[8 + c * GPC + gi] = gt;
+      }
       if (gi + 1 < GPC) {
         const T acc = solve_op(cur);
         load_op(B, bb, gi + 1, nxt);  // in the shadow of the x loads / DFMAs
         publish(cur, acc);
-      } else {  // last group of the chunk: open the next chunk, recycle this one
+      } else {  // last group of the chunk: publish first, then release this
+                // slot to the producer warp and open the next chunk
         const T acc = solve_op(cur);
-        const int cur_slot = slot;
+        publish(cur, acc);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[slot]);
         if (c + 1 < s_nchunk) {
           if (++slot == g.NCH) {
             slot = 0;
@@ -1484,11 +1551,6 @@ __global__ void __launch_bounds__(256, 1)
           B = ring + (size_t)slot * g.chunk_bytes;
           bb = (const T*)(bring + (size_t)slot * g.bring_bytes);
           load_op(B, bb, 0, nxt);
-        }
-        publish(cur, acc);
-        if (lane == 0 && c + g.NCH < s_nchunk) {
-          const int4 hdr = *(const int4*)(ring + (size_t)cur_slot * g.chunk_bytes);
-          issue_chunk(cur_slot, c + g.NCH, hdr.z, hdr.w);
         }
       }
       warp_sync_all();

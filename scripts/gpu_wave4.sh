@@ -2,7 +2,7 @@
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { tail -20 gpurun_out/build.log; exit 1; }
 timeout 300 python scripts/time_segs.py --config C2 --tag "default" 2>&1 | tail -1
-for geo in "8,8,8,4" "16,4,8,4" "16,2,8,4" "8,4,16,3"; do
+for geo in "8,4,8,4" "16,2,8,4" "16,4,8,3" "16,8,8,4"; do
   SPTRSV_WAVE=$geo timeout 300 python scripts/time_segs.py --config C2 --tag "geo=$geo" 2>&1 | tail -1
 done
 mkdir -p gpurun_out/tr

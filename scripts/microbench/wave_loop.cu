@@ -128,7 +128,9 @@ void run(int iters, long long* d, double* g, const char* name) {
   printf("%-48s F=%3d: %7.1f cycles/group\n", name, F, (double)h[F & 127] / iters);
 }
 
+int main_hop();
 int main() {
+  main_hop();
   long long* d;
   double* g;
   cudaMalloc(&d, 128 * 8);
@@ -148,5 +150,73 @@ int main() {
   run<97 + 256>(it, d, g, "+ operand loads + per-lane sentinel branch");
   run<97 + 256 + 4 + 16>(it, d, g, "+ operand loads + sentinel branch + STG + push");
   printf("status %s\n", cudaGetErrorString(cudaDeviceSynchronize()));
+  return 0;
+}
+
+// ---- hop latency: ping-pong of a value between two warps that poll their
+// own shared memory; the partner writes it there (same CTA: st.shared;
+// other CTA of the cluster: mapa + st.shared::cluster, weak or relaxed.cluster)
+template <int MODE>  // 0 same CTA STS, 1 DSMEM relaxed.cluster, 2 DSMEM weak, 3 DSMEM volatile
+__global__ void k_hop(int iters, long long* out) {
+  __shared__ double box[2];
+  uint32_t rank;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+  const int w = MODE == 0 ? threadIdx.x / 32 : (int)rank;  // player id
+  const int lane = threadIdx.x & 31;
+  if (threadIdx.x < 2) box[threadIdx.x] = -1.0;
+  __syncthreads();
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+  if (MODE != 0 && threadIdx.x >= 32) return;
+  const uint32_t mybox = (uint32_t)__cvta_generic_to_shared(&box[w]);
+  const uint32_t other = (uint32_t)__cvta_generic_to_shared(&box[1 - w]);
+  uint32_t remote;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(other), "r"(1 - rank));
+  long long t0 = clock64();
+  for (int i = 0; i < iters; ++i) {
+    if (w == 1 || i > 0) {  // wait for value i
+      double v;
+      do {
+        asm volatile("ld.volatile.shared.f64 %0, [%1];" : "=d"(v) : "r"(mybox));
+      } while (v != (double)(2 * i + (w == 1 ? 0 : -1)) && !(w == 0 && v == (double)(2 * i - 1)));
+    }
+    const double nv = (double)(2 * i + w);
+    if (lane == 0) {
+      if (MODE == 0) asm volatile("st.volatile.shared.f64 [%0], %1;" ::"r"(other), "d"(nv));
+      if (MODE == 1) asm volatile("st.relaxed.cluster.shared::cluster.f64 [%0], %1;" ::"r"(remote), "d"(nv) : "memory");
+      if (MODE == 2) asm volatile("st.shared::cluster.f64 [%0], %1;" ::"r"(remote), "d"(nv) : "memory");
+      if (MODE == 3) asm volatile("st.volatile.shared::cluster.f64 [%0], %1;" ::"r"(remote), "d"(nv) : "memory");
+    }
+    __syncwarp();
+  }
+  if (w == 0 && lane == 0) out[100 + MODE] = clock64() - t0;
+}
+
+template <int MODE>
+void run_hop(int iters, long long* d, const char* name) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(MODE == 0 ? 1 : 2);
+  cfg.blockDim = dim3(MODE == 0 ? 64 : 32);
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = MODE == 0 ? 1 : 2;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, k_hop<MODE>, iters, d);
+  cudaError_t e2 = cudaDeviceSynchronize();
+  long long h[128];
+  cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
+  printf("hop %-40s: %7.1f cycles per one-way hop (%s/%s)\n", name, (double)h[100 + MODE] / iters / 2,
+         cudaGetErrorString(e), cudaGetErrorString(e2));
+}
+
+int main_hop() {
+  long long* d;
+  cudaMalloc(&d, 128 * 8);
+  run_hop<0>(20000, d, "same CTA, st.volatile.shared");
+  run_hop<1>(20000, d, "DSMEM st.relaxed.cluster");
+  run_hop<2>(20000, d, "DSMEM st weak");
+  run_hop<3>(20000, d, "DSMEM st.volatile");
   return 0;
 }
