@@ -404,12 +404,12 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   auto& I = S.info;
   if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_PIPE) return;
   const int m = I.row1 - I.row0;
-  int C = 16, W = 4, GPC = 8, NCH = 4;
+  int C = 16, W = 2, GPC = 12, NCH = 4;
   if (const char* e = std::getenv("SPTRSV_WAVE")) {
     int a, b2, c, d;
     if (std::sscanf(e, "%d,%d,%d,%d", &a, &b2, &c, &d) == 4 && a >= 1 && a <= 16 && b2 >= 1 && b2 <= 8 &&
         c >= 1 && c <= 32 && d >= 2 && d <= 4) {
-      C = a; W = b2; GPC = c <= 4 ? 4 : 8; NCH = d;
+      C = a; W = b2; GPC = c <= 6 ? 6 : 12; NCH = d;
     }
   }
   auto give_up = [&]() {
@@ -506,9 +506,9 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
     const int64_t rings = (int64_t)W * NCH * (k::wave_hdr_bytes(GPC) + (int64_t)GPC * gb2 + bring + 16);
     const int64_t slots_avail = (232448 - 512 - rings) / (int64_t)vb;
     icap = (slots_avail - 2) / W - XW;
-    if (icap >= 1024 || (GPC == 4 && NCH == 2)) break;
+    if (icap >= 1024 || (GPC == 6 && NCH == 2)) break;
     if (NCH > 2) --NCH;
-    else { GPC = 4; NCH = 4; }
+    else { GPC = 6; NCH = 4; }
   }
   if (const char* e = std::getenv("SPTRSV_WAVE_ICAP")) icap = std::min<int64_t>(icap, std::max(0, std::atoi(e)));
   if (icap < 0) return give_up();
@@ -699,9 +699,9 @@ Error launch_wave_t(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, c
 template <typename T, int K, int E>
 Error launch_wave_e(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
   const bool glb = S.wave_global > 0;
-  if (S.wave_GPC == 4)
-    return glb ? launch_wave_t<T, K, E, 4, true>(p, S, bw, xs, st, s) : launch_wave_t<T, K, E, 4, false>(p, S, bw, xs, st, s);
-  return glb ? launch_wave_t<T, K, E, 8, true>(p, S, bw, xs, st, s) : launch_wave_t<T, K, E, 8, false>(p, S, bw, xs, st, s);
+  if (S.wave_GPC == 6)
+    return glb ? launch_wave_t<T, K, E, 6, true>(p, S, bw, xs, st, s) : launch_wave_t<T, K, E, 6, false>(p, S, bw, xs, st, s);
+  return glb ? launch_wave_t<T, K, E, 12, true>(p, S, bw, xs, st, s) : launch_wave_t<T, K, E, 12, false>(p, S, bw, xs, st, s);
 }
 
 template <typename T, int K>

@@ -1457,6 +1457,10 @@ __global__ void __launch_bounds__(288, 1)
     o.b = bb[gh.z + lane];
     o.row = gh.x + lane;
     o.cnt = gh.y;
+  };
+  // early poll of a group's dependencies (readiness test only): issued a
+  // whole group before the test, so the test never waits on the load
+  auto early_poll = [&](WaveOp<T, K, E>& o) {
     if (!GLB) {
 #pragma unroll
       for (int k2 = 0; k2 < K; ++k2) o.xe[k2] = lds_x_v(xa_s + o.xo[k2], T(0));
@@ -1466,10 +1470,16 @@ __global__ void __launch_bounds__(288, 1)
   auto solve_op = [&](WaveOp<T, K, E>& cur) -> T {
     T x[K];
     if (!GLB) {
+      // ---- level chain: the x_j loads go first (own-strand values were
+      // stored before the last __syncwarp); the readiness test uses the
+      // early poll and only sends the warp to the wait loop (then reloads)
+      // when a producer strand is behind
+#pragma unroll
+      for (int k2 = 0; k2 < K; ++k2) x[k2] = lds_x_v(xa_s + cur.xo[k2], T(0));
       bool pend = false;
 #pragma unroll
       for (int k2 = 0; k2 < K; ++k2) pend |= maybe_sent(cur.xe[k2]);
-      if (vote_any(pend)) {  // a producer strand is behind: wait for it
+      if (vote_any(pend)) {
         for (;;) {
           pend = false;
 #pragma unroll
@@ -1481,10 +1491,9 @@ __global__ void __launch_bounds__(288, 1)
             break;
           }
         }
-      }
-      // ---- level chain: every value is ready now
 #pragma unroll
-      for (int k2 = 0; k2 < K; ++k2) x[k2] = lds_x_v(xa_s + cur.xo[k2], T(0));
+        for (int k2 = 0; k2 < K; ++k2) x[k2] = lds_x_v(xa_s + cur.xo[k2], T(0));
+      }
     } else {
 #pragma unroll
       for (int k2 = 0; k2 < K; ++k2) {
@@ -1513,45 +1522,60 @@ __global__ void __launch_bounds__(288, 1)
     if (lane < (cur.cnt & kWaveCntMask)) stg_x_v(xs + cur.row, acc);
   };
 
-  WaveOp<T, K, E> opA, opB;
+  // three operand sets rotate over the groups (GPC % 3 == 0): group g solves
+  // from set g%3 while set (g+1)%3 gets its early poll and set (g+2)%3 its
+  // operands -- every load has a whole group of lead before its first use
+  WaveOp<T, K, E> op0, op1, op2;
   int slot = 0;
   uint32_t ph = 0;
   const unsigned char* B = ring;
   const T* bb = (const T*)bring;
+  const unsigned char* Bn = ring;
+  const T* bbn = (const T*)bring;
+  int slot_n = 0;
+  uint32_t ph_n = 0;
   if (s_nchunk > 0) {
     mbar_wait(&full[0], 0);
-    load_op(B, bb, 0, opA);
+    load_op(B, bb, 0, op0);
+    load_op(B, bb, 1, op1);
+    early_poll(op0);
   }
   for (int c = 0; c < s_nchunk; ++c) {
+    const bool more = c + 1 < s_nchunk;
 #pragma unroll
     for (int gi = 0; gi < GPC; ++gi) {
-      WaveOp<T, K, E>& cur = (gi & 1) ? opB : opA;
-      WaveOp<T, K, E>& nxt = (gi & 1) ? opA : opB;
+      WaveOp<T, K, E>& cur = gi % 3 == 0 ? op0 : gi % 3 == 1 ? op1 : op2;
+      WaveOp<T, K, E>& n1 = gi % 3 == 0 ? op1 : gi % 3 == 1 ? op2 : op0;
+      WaveOp<T, K, E>& n2 = gi % 3 == 0 ? op2 : gi % 3 == 1 ? op0 : op1;
+#ifdef SPTRSV_WAVE_TRACE
       if (tr && lane == 0 && c * GPC + gi < 1016) {
         long long gt;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
         tr[8 + c * GPC + gi] = gt;
       }
-      if (gi + 1 < GPC) {
-        const T acc = solve_op(cur);
-        load_op(B, bb, gi + 1, nxt);  // in the shadow of the x loads / DFMAs
-        publish(cur, acc);
-      } else {  // last group of the chunk: publish first, then release this
-                // slot to the producer warp and open the next chunk
-        const T acc = solve_op(cur);
-        publish(cur, acc);
+#endif
+      const T acc = solve_op(cur);
+      if (gi + 1 < GPC || more) early_poll(n1);
+      if (gi + 2 < GPC) {
+        load_op(B, bb, gi + 2, n2);
+      } else if (more) {
+        if (gi + 2 == GPC) {  // open the next chunk two groups ahead
+          slot_n = slot + 1 == g.NCH ? 0 : slot + 1;
+          ph_n = slot + 1 == g.NCH ? ph ^ 1u : ph;
+          mbar_wait(&full[slot_n], ph_n);
+          Bn = ring + (size_t)slot_n * g.chunk_bytes;
+          bbn = (const T*)(bring + (size_t)slot_n * g.bring_bytes);
+        }
+        load_op(Bn, bbn, gi + 2 - GPC, n2);
+      }
+      publish(cur, acc);
+      if (gi + 1 == GPC) {  // chunk consumed: release its slot to the producer warp
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[slot]);
-        if (c + 1 < s_nchunk) {
-          if (++slot == g.NCH) {
-            slot = 0;
-            ph ^= 1u;
-          }
-          mbar_wait(&full[slot], ph);
-          B = ring + (size_t)slot * g.chunk_bytes;
-          bb = (const T*)(bring + (size_t)slot * g.bring_bytes);
-          load_op(B, bb, 0, nxt);
-        }
+        slot = slot_n;
+        ph = ph_n;
+        B = Bn;
+        bb = bbn;
       }
       warp_sync_all();
     }
