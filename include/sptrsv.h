@@ -82,11 +82,14 @@ typedef enum {
   SPTRSV_IMPL_SQ_VECTOR = 5,     /* K6/K8: warp per row, CSR or DCSR                                */
   SPTRSV_IMPL_TRI_SUPERNODE = 6, /* B200: warp per fundamental supernode (<= 32 rows): dense GEMV of its
                                     shared external columns + register-resident dense triangle     */
-  SPTRSV_IMPL_TRI_PIPE = 7       /* B200: strand wavefront -- narrow-level triangle split by original row
+  SPTRSV_IMPL_TRI_PIPE = 7,      /* B200: strand wavefront -- narrow-level triangle split by original row
                                     index into C x W strands (one warp each, one thread-block cluster);
                                     no level barrier; cross-strand x pushed into the consumer's shared
                                     memory (DSMEM).  Replaced by TRI_CHAIN at upload when a row has > 8
                                     dependencies (or > 10% would be polled in global memory)          */
+  SPTRSV_IMPL_SQ_ADAPT = 8       /* B200: nnz-balanced row blocks (<= 32 rows, <= 256 entries) per warp,
+                                    products staged in shared memory, lane-per-row sums; long rows
+                                    alone (split into 1024-entry chunks with atomic partial sums)   */
 } sptrsv_impl_t;
 
 /* Which kernel implements each Alg 7 label. PAPER maps labels 1:1 onto the

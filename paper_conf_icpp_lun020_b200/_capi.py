@@ -23,7 +23,7 @@ SELECTORS = {"PAPER": 0, "B200": 1}
 KERNELS = ["COMPLETELY_PARALLEL", "LEVEL_SET", "SYNC_FREE", "NEAR_SERIAL",
            "SCALAR_CSR", "SCALAR_DCSR", "VECTOR_CSR", "VECTOR_DCSR"]
 FORMATS = ["DIAG", "CSR", "DCSR"]
-IMPLS = ["TRI_DIAG", "TRI_LEVELSET", "TRI_SYNCFREE", "TRI_CHAIN", "SQ_SCALAR", "SQ_VECTOR", "TRI_SUPERNODE", "TRI_PIPE"]
+IMPLS = ["TRI_DIAG", "TRI_LEVELSET", "TRI_SYNCFREE", "TRI_CHAIN", "SQ_SCALAR", "SQ_VECTOR", "TRI_SUPERNODE", "TRI_PIPE", "SQ_ADAPT"]
 ARRAY_IN_DEGREE, ARRAY_LEVEL_PTR, ARRAY_DCSR_ROWS = 0, 1, 2
 
 EXPORTS = ["sptrsv_opts_default", "sptrsv_analyse", "sptrsv_solve", "sptrsv_free", "sptrsv_plan_info",

@@ -14,8 +14,10 @@
 //   features + Alg 7    Sec 3.4 (L252-L296)
 #include <algorithm>
 #include <chrono>
+#include <cstdlib>
 #include <cstring>
 #include <functional>
+#include <mutex>
 #include <numeric>
 #include <thread>
 
@@ -39,73 +41,111 @@ void parallel_for(int64_t n, int threads, const std::function<void(int64_t, int6
   for (auto& x : th) x.join();
 }
 
+// The lower-triangular input the analysis works on.  LOWER input is read in
+// place (the caller's CSR outlives the blocking sptrsv_analyse call); UPPER
+// is materialised as J U J.
 struct LowerCSR {
   int32_t n = 0;
   std::vector<int64_t> rp;
-  std::vector<int32_t> ci;
-  std::vector<char> val;
+  const int32_t* ci = nullptr;
+  const char* val = nullptr;
+  dvec<int32_t> ci_own;
+  dvec<char> val_own;
 };
 
+// Row-local checks of one CSR row (the first failing check wins).
+Error validate_row(int32_t i, int64_t nnz, int32_t n, const int32_t* rp, const int32_t* ci, const char* val,
+                   size_t vb, sptrsv_fill_t fill) {
+  int64_t s = rp[i], e = rp[i + 1];
+  if (e < s || e > nnz) return {SPTRSV_ERROR_INVALID_VALUE, "row_ptr not monotone at row " + std::to_string(i)};
+  for (int64_t q = s; q < e; ++q) {
+    int32_t c = ci[q];
+    if (c < 0 || c >= n) return {SPTRSV_ERROR_INVALID_VALUE, "column index out of range in row " + std::to_string(i)};
+    if (q > s && c <= ci[q - 1]) return {SPTRSV_ERROR_UNSORTED, "columns not strictly increasing in row " + std::to_string(i)};
+  }
+  bool zero;
+  if (fill == SPTRSV_LOWER) {
+    if (e > s && ci[e - 1] > i) return {SPTRSV_ERROR_NOT_TRIANGULAR, "entry above the diagonal in row " + std::to_string(i)};
+    if (e == s || ci[e - 1] != i) return {SPTRSV_ERROR_ZERO_PIVOT, "missing diagonal in row " + std::to_string(i)};
+    const char* d = val + (size_t)(e - 1) * vb;
+    zero = vb == 8 ? (*(const double*)d == 0.0) : (*(const float*)d == 0.0f);
+  } else {
+    if (e > s && ci[s] < i) return {SPTRSV_ERROR_NOT_TRIANGULAR, "entry below the diagonal in row " + std::to_string(i)};
+    if (e == s || ci[s] != i) return {SPTRSV_ERROR_ZERO_PIVOT, "missing diagonal in row " + std::to_string(i)};
+    const char* d = val + (size_t)s * vb;
+    zero = vb == 8 ? (*(const double*)d == 0.0) : (*(const float*)d == 0.0f);
+  }
+  if (zero) return {SPTRSV_ERROR_ZERO_PIVOT, "zero diagonal in row " + std::to_string(i)};
+  return {SPTRSV_SUCCESS, ""};
+}
+
+// Rows are checked in parallel chunks; the error reported is the one of the
+// lowest failing row, exactly what a serial row-order scan reports.
 Error validate(int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, const char* val, size_t vb,
-               sptrsv_fill_t fill) {
+               sptrsv_fill_t fill, int threads) {
   if (rp[0] != 0) return {SPTRSV_ERROR_INVALID_VALUE, "row_ptr[0] != 0"};
   if ((int64_t)rp[n] != nnz) return {SPTRSV_ERROR_INVALID_VALUE, "nnz != row_ptr[n]"};
-  for (int32_t i = 0; i < n; ++i) {
-    int64_t s = rp[i], e = rp[i + 1];
-    if (e < s || e > nnz) return {SPTRSV_ERROR_INVALID_VALUE, "row_ptr not monotone at row " + std::to_string(i)};
-    for (int64_t q = s; q < e; ++q) {
-      int32_t c = ci[q];
-      if (c < 0 || c >= n) return {SPTRSV_ERROR_INVALID_VALUE, "column index out of range in row " + std::to_string(i)};
-      if (q > s && c <= ci[q - 1]) return {SPTRSV_ERROR_UNSORTED, "columns not strictly increasing in row " + std::to_string(i)};
+  // a monotone row_ptr is checked first (n reads) so every chunk may index
+  // its rows safely; a violation is reported by a serial scan up to it
+  for (int32_t i = 0; i < n; ++i)
+    if (rp[i + 1] < rp[i] || rp[i + 1] > nnz) {
+      for (int32_t j = 0; j <= i; ++j) {
+        Error e = validate_row(j, nnz, n, rp, ci, val, vb, fill);
+        if (e.status) return e;
+      }
     }
-    bool zero;
-    if (fill == SPTRSV_LOWER) {
-      if (e > s && ci[e - 1] > i) return {SPTRSV_ERROR_NOT_TRIANGULAR, "entry above the diagonal in row " + std::to_string(i)};
-      if (e == s || ci[e - 1] != i) return {SPTRSV_ERROR_ZERO_PIVOT, "missing diagonal in row " + std::to_string(i)};
-      const char* d = val + (size_t)(e - 1) * vb;
-      zero = vb == 8 ? (*(const double*)d == 0.0) : (*(const float*)d == 0.0f);
-    } else {
-      if (e > s && ci[s] < i) return {SPTRSV_ERROR_NOT_TRIANGULAR, "entry below the diagonal in row " + std::to_string(i)};
-      if (e == s || ci[s] != i) return {SPTRSV_ERROR_ZERO_PIVOT, "missing diagonal in row " + std::to_string(i)};
-      const char* d = val + (size_t)s * vb;
-      zero = vb == 8 ? (*(const double*)d == 0.0) : (*(const float*)d == 0.0f);
+  std::mutex mu;
+  int32_t best = -1;
+  Error best_e{SPTRSV_SUCCESS, ""};
+  parallel_for(n, threads, [&](int64_t a, int64_t b) {
+    for (int64_t i = a; i < b; ++i) {
+      Error e = validate_row((int32_t)i, nnz, n, rp, ci, val, vb, fill);
+      if (e.status) {
+        std::lock_guard<std::mutex> g(mu);
+        if (best < 0 || i < best) {
+          best = (int32_t)i;
+          best_e = e;
+        }
+        return;
+      }
     }
-    if (zero) return {SPTRSV_ERROR_ZERO_PIVOT, "zero diagonal in row " + std::to_string(i)};
-  }
-  return {SPTRSV_SUCCESS, ""};
+  });
+  return best_e;
 }
 
 // Lower CSR of the input; UPPER is mapped to J U J (i -> n-1-i, reading R19):
 // row n-1-i of the result is row i of U read backwards, so its columns are
 // ascending and the diagonal (first in U's row) becomes last.
-LowerCSR to_lower(int32_t n, const int32_t* rp, const int32_t* ci, const char* val, size_t vb,
-                  sptrsv_fill_t fill) {
-  LowerCSR L;
+void to_lower(LowerCSR& L, int32_t n, const int32_t* rp, const int32_t* ci, const char* val, size_t vb,
+              sptrsv_fill_t fill, int threads) {
   L.n = n;
   int64_t nnz = rp[n];
   L.rp.resize((size_t)n + 1);
-  L.ci.resize((size_t)nnz);
-  L.val.resize((size_t)nnz * vb);
   if (fill == SPTRSV_LOWER) {
     for (int32_t i = 0; i <= n; ++i) L.rp[i] = rp[i];
-    std::memcpy(L.ci.data(), ci, (size_t)nnz * 4);
-    std::memcpy(L.val.data(), val, (size_t)nnz * vb);
-    return L;
+    L.ci = ci;
+    L.val = val;
+    return;
   }
+  L.ci_own.resize((size_t)nnz);
+  L.val_own.resize((size_t)nnz * vb);
   L.rp[0] = 0;
   for (int32_t r = 0; r < n; ++r) {
     int32_t i = n - 1 - r;
     L.rp[r + 1] = L.rp[r] + (rp[i + 1] - rp[i]);
   }
-  for (int32_t r = 0; r < n; ++r) {
-    int32_t i = n - 1 - r;
-    int64_t o = L.rp[r];
-    for (int64_t q = (int64_t)rp[i + 1] - 1; q >= rp[i]; --q, ++o) {
-      L.ci[o] = n - 1 - ci[q];
-      std::memcpy(&L.val[(size_t)o * vb], val + (size_t)q * vb, vb);
+  parallel_for(n, threads, [&](int64_t a, int64_t b) {
+    for (int64_t r = a; r < b; ++r) {
+      int32_t i = n - 1 - (int32_t)r;
+      int64_t o = L.rp[r];
+      for (int64_t q = (int64_t)rp[i + 1] - 1; q >= rp[i]; --q, ++o) {
+        L.ci_own[o] = n - 1 - ci[q];
+        std::memcpy(&L.val_own[(size_t)o * vb], val + (size_t)q * vb, vb);
+      }
     }
-  }
-  return L;
+  });
+  L.ci = L.ci_own.data();
+  L.val = L.val_own.data();
 }
 
 // Reading R2: largest d with d == 0 or floor(n / 2^d) >= T.
@@ -129,7 +169,7 @@ int32_t clamp_depth(int64_t n, int32_t d) {
 // share one list of external columns).  Returns the number of pieces.
 constexpr int32_t kSnMax = 32;
 
-int64_t supernode_pieces(int32_t n, const std::vector<int64_t>& rp, const std::vector<int32_t>& ci,
+int64_t supernode_pieces(int32_t n, const std::vector<int64_t>& rp, const int32_t* ci,
                          std::vector<int32_t>* starts) {
   int64_t np = 0;
   int32_t start = 0;
@@ -139,7 +179,7 @@ int64_t supernode_pieces(int32_t n, const std::vector<int64_t>& rp, const std::v
       const int64_t a0 = rp[r - 1], l0 = rp[r] - 1 - a0;  // off-diagonals of r-1
       const int64_t a1 = rp[r], l1 = rp[r + 1] - 1 - a1;  // off-diagonals of r
       join = l1 == l0 + 1 && ci[a1 + l1 - 1] == r - 1 &&
-             std::equal(ci.begin() + a0, ci.begin() + a0 + l0, ci.begin() + a1);
+             std::equal(ci + a0, ci + a0 + l0, ci + a1);
     }
     if (!join) {
       start = r;
@@ -168,20 +208,32 @@ struct Reorderer {
   // dependencies inside the triangle count, reading R5), then a stable
   // counting sort of its rows by level (ties keep the current order, R4).
   // Writes the (sorted) levels into leaf_level[lo,hi); returns nlevels.
-  int32_t node_reorder(int32_t lo, int32_t hi) {
+  int32_t node_reorder(int32_t lo, int32_t hi, bool identity = false) {
     int32_t m = hi - lo;
     if (m == 0) return 0;
     std::vector<int32_t> lev((size_t)m);
     int32_t nl = 0;
-    for (int32_t r = lo; r < hi; ++r) {
-      int32_t o = perm[r];
-      int32_t lv = 0;
-      for (int64_t q = L.rp[o], e = L.rp[o + 1] - 1; q < e; ++q) {  // off-diagonals
-        int32_t c = old2new[L.ci[q]];
-        if (c >= lo) lv = std::max(lv, lev[c - lo] + 1);
+    if (identity) {  // perm is still the identity (the root): no old2new lookups
+      for (int32_t r = lo; r < hi; ++r) {
+        int32_t lv = 0;
+        for (int64_t q = L.rp[r], e = L.rp[r + 1] - 1; q < e; ++q) {
+          int32_t c = L.ci[q];
+          if (c >= lo) lv = std::max(lv, lev[c - lo] + 1);
+        }
+        lev[r - lo] = lv;
+        nl = std::max(nl, lv + 1);
       }
-      lev[r - lo] = lv;
-      nl = std::max(nl, lv + 1);
+    } else {
+      for (int32_t r = lo; r < hi; ++r) {
+        int32_t o = perm[r];
+        int32_t lv = 0;
+        for (int64_t q = L.rp[o], e = L.rp[o + 1] - 1; q < e; ++q) {  // off-diagonals
+          int32_t c = old2new[L.ci[q]];
+          if (c >= lo) lv = std::max(lv, lev[c - lo] + 1);
+        }
+        lev[r - lo] = lv;
+        nl = std::max(nl, lv + 1);
+      }
     }
     if (reorder) {
       std::vector<int32_t> cnt((size_t)nl + 1, 0);
@@ -193,7 +245,10 @@ struct Reorderer {
         perm[lo + k] = np[k];
         old2new[np[k]] = lo + k;
       }
-      std::sort(lev.begin(), lev.end());
+      // the sorted levels straight from the counts (cnt[l] is now the end of
+      // level l's range)
+      for (int32_t l = 0, k = 0; l < nl; ++l)
+        for (; k < cnt[l]; ++k) lev[k] = l;
     }
     std::copy(lev.begin(), lev.end(), leaf_level.begin() + lo);
     return nl;
@@ -224,9 +279,13 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
   int threads = p.opts.threads > 0 ? p.opts.threads : (int)std::max(1u, std::thread::hardware_concurrency());
   threads = std::min(threads, 64);
 
-  Error e = validate(n, nnz, row_ptr, col_idx, val, vb, p.fill);
+  PhaseClock clk;
+  Error e = validate(n, nnz, row_ptr, col_idx, val, vb, p.fill, threads);
   if (e.status) return e;
-  LowerCSR L = to_lower(n, row_ptr, col_idx, val, vb, p.fill);
+  clk.lap("validate");
+  LowerCSR L;
+  to_lower(L, n, row_ptr, col_idx, val, vb, p.fill, threads);
+  clk.lap("to_lower");
   p.n = n;
   p.nnz = nnz;
 
@@ -253,17 +312,33 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
   std::vector<std::pair<int32_t, int32_t>> nodes = {{0, n}};
   for (int32_t d = 0; d <= p.depth && n > 0; ++d) {
     std::vector<int32_t> nl(nodes.size());
-    if (nodes.size() == 1 || threads == 1) {
-      for (size_t k = 0; k < nodes.size(); ++k) nl[k] = R.node_reorder(nodes[k].first, nodes[k].second);
+    // A top child [lo, mid) needs no work: its rows depend only on rows
+    // < mid, so their levels inside [lo, mid) are the parent's (already in
+    // leaf_level, and already sorted when reordering) and its stable level
+    // sort is the identity (reading R3's invariant).  Only bottom children
+    // (and the root) are analysed, in parallel.
+    std::vector<size_t> work;
+    for (size_t k = 0; k < nodes.size(); ++k) {
+      if (d > 0 && k % 2 == 0) {
+        int32_t mx = -1;
+        for (int32_t r = nodes[k].first; r < nodes[k].second; ++r) mx = std::max(mx, R.leaf_level[r]);
+        nl[k] = mx + 1;
+      } else {
+        work.push_back(k);
+      }
+    }
+    if (work.size() == 1 || threads == 1) {
+      for (size_t k : work) nl[k] = R.node_reorder(nodes[k].first, nodes[k].second, d == 0);
     } else {
       std::vector<std::thread> th;
-      int T = std::min<int>(threads, (int)nodes.size());
+      int T = std::min<int>(threads, (int)work.size());
       for (int t = 0; t < T; ++t)
         th.emplace_back([&, t] {
-          for (size_t k = t; k < nodes.size(); k += T) nl[k] = R.node_reorder(nodes[k].first, nodes[k].second);
+          for (size_t w = t; w < work.size(); w += T) nl[work[w]] = R.node_reorder(nodes[work[w]].first, nodes[work[w]].second);
         });
       for (auto& x : th) x.join();
     }
+    if (clk.on) clk.lap(("  reorder depth " + std::to_string(d)).c_str());
     if (d == p.depth) {
       leaf_nl = nl;
       break;
@@ -277,6 +352,7 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
     nodes.swap(next);
   }
 
+  clk.lap("levels + reorder");
   // ---- final P L P^T, columns sorted (reading R6) ----
   p.p_rp.assign((size_t)n + 1, 0);
   for (int32_t r = 0; r < n; ++r) {
@@ -290,13 +366,27 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
     for (int64_t r = a; r < b; ++r) {
       int32_t o = R.perm[r];
       int64_t s = L.rp[o], len = L.rp[o + 1] - s;
-      tmp.resize((size_t)len);
-      for (int64_t k = 0; k < len; ++k) tmp[k] = {R.old2new[L.ci[s + k]], s + k};
-      std::sort(tmp.begin(), tmp.end());
       int64_t d0 = p.p_rp[r];
+      // map the columns; rows whose mapped columns stay ascending (all of
+      // them without reordering, most of them with it) need no sort
+      bool sorted = true;
+      int32_t prev = -1;
+      for (int64_t k = 0; k < len; ++k) {
+        const int32_t c = R.old2new[L.ci[s + k]];
+        p.p_ci[d0 + k] = c;
+        sorted &= c > prev;
+        prev = c;
+      }
+      if (sorted) {
+        std::memcpy(&p.p_val[(size_t)d0 * vb], L.val + (size_t)s * vb, (size_t)len * vb);
+        continue;
+      }
+      tmp.resize((size_t)len);
+      for (int64_t k = 0; k < len; ++k) tmp[k] = {p.p_ci[d0 + k], s + k};
+      std::sort(tmp.begin(), tmp.end());
       for (int64_t k = 0; k < len; ++k) {
         p.p_ci[d0 + k] = tmp[k].first;
-        std::memcpy(&p.p_val[(size_t)(d0 + k) * vb], &L.val[(size_t)tmp[k].second * vb], vb);
+        std::memcpy(&p.p_val[(size_t)(d0 + k) * vb], L.val + (size_t)tmp[k].second * vb, vb);
       }
     }
   });
@@ -318,6 +408,7 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
   p.leaf_level = R.leaf_level;
   p.lower_old = R.perm;
 
+  clk.lap("P L P^T");
   // ---- segment geometry in execution order ----
   struct Geo { int32_t kind, r0, r1, c0, c1, leaf; };
   std::vector<Geo> geo;
@@ -353,7 +444,7 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
 
   // ---- extract blocks, features, Alg 7 ----
   p.segs.resize(geo.size());
-  auto build_seg = [&](size_t si) {
+  auto build_seg = [&](size_t si, int inner) {
     const Geo& g = geo[si];
     Segment& S = p.segs[si];
     sptrsv_seg_info_t& I = S.info;
@@ -361,17 +452,19 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
     I.row0 = g.r0; I.row1 = g.r1; I.col0 = g.c0; I.col1 = g.c1;
     int32_t m = g.r1 - g.r0;
     S.rp.assign((size_t)m + 1, 0);
-    std::vector<int64_t> lo_idx((size_t)m), hi_idx((size_t)m);
-    for (int32_t k = 0; k < m; ++k) {
-      int32_t r = g.r0 + k;
-      const int32_t* rb = p.p_ci.data() + p.p_rp[r];
-      const int32_t* re = p.p_ci.data() + p.p_rp[r + 1];
-      int32_t cend = g.kind == 0 ? r : g.c1;  // TRI: off-diagonals only
-      const int32_t* a = std::lower_bound(rb, re, g.c0);
-      const int32_t* b = std::lower_bound(a, re, cend);
-      lo_idx[k] = a - p.p_ci.data();
-      hi_idx[k] = b - p.p_ci.data();
-    }
+    dvec<int64_t> lo_idx((size_t)m), hi_idx((size_t)m);
+    parallel_for(m, inner, [&](int64_t ka, int64_t kb) {
+      for (int64_t k = ka; k < kb; ++k) {
+        int32_t r = g.r0 + (int32_t)k;
+        const int32_t* rb = p.p_ci.data() + p.p_rp[r];
+        const int32_t* re = p.p_ci.data() + p.p_rp[r + 1];
+        int32_t cend = g.kind == 0 ? r : g.c1;  // TRI: off-diagonals only
+        const int32_t* a = std::lower_bound(rb, re, g.c0);
+        const int32_t* b = std::lower_bound(a, re, cend);
+        lo_idx[k] = a - p.p_ci.data();
+        hi_idx[k] = b - p.p_ci.data();
+      }
+    });
     int64_t tot = 0, empty = 0;
     for (int32_t k = 0; k < m; ++k) {
       int64_t c = hi_idx[k] - lo_idx[k];
@@ -398,15 +491,20 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
       S.nzr = m;
       {  // fundamental-supernode pieces of the triangle (its own entries only)
         S.sn_ptr.clear();
-        int32_t start = 0;
-        for (int32_t k = 0; k < m; ++k) {
-          bool join = false;
-          if (k > start && k - start < kSnMax) {
+        // whether row k may extend row k-1's piece depends on those two rows
+        // only (parallel); the 32-row cut is a serial pass
+        std::vector<char> canj((size_t)m, 0);
+        parallel_for(m, inner, [&](int64_t ka, int64_t kb) {
+          for (int64_t k = std::max<int64_t>(ka, 1); k < kb; ++k) {
             const int64_t a0 = lo_idx[k - 1], l0 = hi_idx[k - 1] - a0;
             const int64_t a1 = lo_idx[k], l1 = hi_idx[k] - a1;
-            join = l1 == l0 + 1 && p.p_ci[a1 + l1 - 1] == g.r0 + k - 1 &&
-                   std::equal(p.p_ci.begin() + a0, p.p_ci.begin() + a0 + l0, p.p_ci.begin() + a1);
+            canj[k] = l1 == l0 + 1 && p.p_ci[a1 + l1 - 1] == g.r0 + k - 1 &&
+                      std::equal(p.p_ci.begin() + a0, p.p_ci.begin() + a0 + l0, p.p_ci.begin() + a1);
           }
+        });
+        int32_t start = 0;
+        for (int32_t k = 0; k < m; ++k) {
+          const bool join = k > start && k - start < kSnMax && canj[k];
           if (!join) {
             start = k;
             S.sn_ptr.push_back(k);
@@ -434,20 +532,36 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
     } else {
       S.nzr = m;
     }
-    int64_t o = 0;
-    int32_t jr = 0;
-    for (int32_t k = 0; k < m; ++k) {
-      int64_t a = lo_idx[k], b = hi_idx[k];
-      if (dcsr) {
-        if (b == a) continue;
-        S.rows[jr] = g.r0 + k;
+    // row pointers (serial prefix), then the entries in parallel: every
+    // stored row is scaled by 1/d_i (triangles: l_ij/d_i, squares: a_ij/d_i;
+    // permute-in scales b the same way), so the solve evaluates
+    // x_i = b_i/d_i - sum_j (l_ij/d_i) x_j with no division on the chain
+    std::vector<int32_t> slot;  // DCSR: stored-row index of local row k
+    {
+      int64_t o = 0;
+      int32_t jr = 0;
+      if (dcsr) slot.assign((size_t)m, -1);
+      for (int32_t k = 0; k < m; ++k) {
+        int64_t c = hi_idx[k] - lo_idx[k];
+        if (dcsr) {
+          if (c == 0) continue;
+          S.rows[jr] = g.r0 + k;
+          slot[k] = jr;
+          o += c;
+          S.rp[++jr] = (int32_t)o;
+        } else {
+          o += c;
+          S.rp[k + 1] = (int32_t)o;
+        }
       }
-      std::memcpy(&S.ci[o], &p.p_ci[a], (size_t)(b - a) * 4);
-      {
-        // every stored row is scaled by 1/d_i (triangles: l_ij/d_i, squares:
-        // a_ij/d_i; permute-in scales b the same way), so the solve evaluates
-        // x_i = b_i/d_i - sum_j (l_ij/d_i) x_j with no division on the chain
-        const int32_t r = g.r0 + k;
+    }
+    parallel_for(m, inner, [&](int64_t ka, int64_t kb) {
+      for (int64_t k = ka; k < kb; ++k) {
+        int64_t a = lo_idx[k], b = hi_idx[k];
+        if (b == a) continue;
+        const int64_t o = dcsr ? S.rp[slot[k]] : S.rp[k];
+        std::memcpy(&S.ci[o], &p.p_ci[a], (size_t)(b - a) * 4);
+        const int32_t r = g.r0 + (int32_t)k;
         if (vb == 8) {
           double d = *(const double*)&p.diag_new[(size_t)r * 8];
           for (int64_t q = a; q < b; ++q) {
@@ -462,25 +576,24 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
           }
         }
       }
-      o += b - a;
-      if (dcsr)
-        S.rp[++jr] = (int32_t)o;
-      else
-        S.rp[k + 1] = (int32_t)o;
-    }
+    });
   };
-  if (threads > 1 && geo.size() > 1) {
+  // few segments: one after the other, each with every thread on its rows;
+  // many: one thread per segment
+  if (threads > 1 && (int)geo.size() >= threads) {
     std::vector<std::thread> th;
-    int T = std::min<int>(threads, (int)geo.size());
+    int T = threads;
     for (int t = 0; t < T; ++t)
       th.emplace_back([&, t] {
-        for (size_t k = t; k < geo.size(); k += T) build_seg(k);
+        for (size_t k = t; k < geo.size(); k += T) build_seg(k, 1);
       });
     for (auto& x : th) x.join();
   } else {
-    for (size_t k = 0; k < geo.size(); ++k) build_seg(k);
+    for (size_t k = 0; k < geo.size(); ++k) build_seg(k, threads);
   }
+  clk.lap("segments + Alg 7");
   choose_impls(p);
+  clk.lap("choose_impls");
   return {SPTRSV_SUCCESS, ""};
 }
 
@@ -536,7 +649,11 @@ void choose_impls(Plan& p) {
     } else {
       int impl = (I.kernel == SPTRSV_K_VECTOR_CSR || I.kernel == SPTRSV_K_VECTOR_DCSR) ? SPTRSV_IMPL_SQ_VECTOR
                                                                                       : SPTRSV_IMPL_SQ_SCALAR;
-      if (p.opts.force_sq_impl == SPTRSV_IMPL_SQ_SCALAR || p.opts.force_sq_impl == SPTRSV_IMPL_SQ_VECTOR)
+      // B200: every square streams through the nnz-balanced row-block kernel
+      // (the Alg 7 label still fixes the format, CSR or DCSR)
+      if (p.opts.selector == SPTRSV_SELECT_B200 && std::getenv("SPTRSV_NO_SQ_ADAPT") == nullptr) impl = SPTRSV_IMPL_SQ_ADAPT;
+      if (p.opts.force_sq_impl == SPTRSV_IMPL_SQ_SCALAR || p.opts.force_sq_impl == SPTRSV_IMPL_SQ_VECTOR ||
+          p.opts.force_sq_impl == SPTRSV_IMPL_SQ_ADAPT)
         impl = p.opts.force_sq_impl;
       I.impl = impl;
     }

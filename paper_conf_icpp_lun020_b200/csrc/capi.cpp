@@ -258,12 +258,20 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_matrix(sptrsv_plan_t plan, int64_t* ro
 namespace {
 struct Fnv {
   uint64_t h = 1469598103934665603ull;
+  // FNV-1a over 64-bit words (then the byte tail): deterministic on any
+  // machine, ~8x fewer multiplies than the byte-wise form on 1 GB plans
   void add(const void* p, size_t bytes) {
     const unsigned char* c = (const unsigned char*)p;
-    for (size_t i = 0; i < bytes; ++i) h = (h ^ c[i]) * 1099511628211ull;
+    size_t i = 0;
+    for (; i + 8 <= bytes; i += 8) {
+      uint64_t w;
+      std::memcpy(&w, c + i, 8);
+      h = (h ^ w) * 1099511628211ull;
+    }
+    for (; i < bytes; ++i) h = (h ^ c[i]) * 1099511628211ull;
   }
-  template <typename V>
-  void vec(const std::vector<V>& v) {
+  template <typename V, typename A>
+  void vec(const std::vector<V, A>& v) {
     uint64_t s = v.size();
     add(&s, 8);
     if (!v.empty()) add(v.data(), v.size() * sizeof(V));

@@ -8,6 +8,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <string>
+#include <mutex>
 #include <unordered_map>
 #include <array>
 
@@ -368,22 +369,24 @@ void build_supernodes(Segment& S, size_t vb) {
     nb += (size_t)w * (w - 1) / 2;
   }
   S.sn_cols.resize(nc);
-  S.sn_vals.assign(std::max<size_t>(nv, 1) * vb, 0);
-  S.sn_blk.assign(std::max<size_t>(nb, 1) * vb, 0);
-  for (int J = 0; J < np; ++J) {
-    const k::SnDesc& d = desc[J];
-    const int a = S.sn_ptr[J];
-    std::memcpy(&S.sn_cols[d.coff], &S.ci[S.rp[a]], (size_t)d.ne * 4);
-    for (int t = 0; t < d.w; ++t) {
-      const int base = S.rp[a + t];
-      for (int q = 0; q < d.ne; ++q)
-        std::memcpy(&S.sn_vals[((size_t)d.voff + (size_t)q * d.w + t) * vb], &S.val[(size_t)(base + q) * vb], vb);
-      for (int c = 0; c < t; ++c) {
-        const size_t off = (size_t)d.boff + (size_t)c * (d.w - 1) - (size_t)c * (c - 1) / 2 + (t - c - 1);
-        std::memcpy(&S.sn_blk[off * vb], &S.val[(size_t)(base + d.ne + c) * vb], vb);
+  S.sn_vals.resize(std::max<size_t>(nv, 1) * vb);  // every byte is written below
+  S.sn_blk.resize(std::max<size_t>(nb, 1) * vb);
+  par_for(np, 0, [&](int64_t J0, int64_t J1) {
+    for (int64_t J = J0; J < J1; ++J) {
+      const k::SnDesc& d = desc[J];
+      const int a = S.sn_ptr[J];
+      std::memcpy(&S.sn_cols[d.coff], &S.ci[S.rp[a]], (size_t)d.ne * 4);
+      for (int t = 0; t < d.w; ++t) {
+        const int base = S.rp[a + t];
+        for (int q = 0; q < d.ne; ++q)
+          std::memcpy(&S.sn_vals[((size_t)d.voff + (size_t)q * d.w + t) * vb], &S.val[(size_t)(base + q) * vb], vb);
+        for (int c = 0; c < t; ++c) {
+          const size_t off = (size_t)d.boff + (size_t)c * (d.w - 1) - (size_t)c * (c - 1) / 2 + (t - c - 1);
+          std::memcpy(&S.sn_blk[off * vb], &S.val[(size_t)(base + d.ne + c) * vb], vb);
+        }
       }
     }
-  }
+  }, 512);
   S.sn_desc.resize((size_t)np * sizeof(k::SnDesc));
   std::memcpy(S.sn_desc.data(), desc.data(), S.sn_desc.size());
 }
@@ -732,7 +735,15 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
     if (I.kind == 1) {  // square: b -= A x
       if (S.dev_nzr > 0 && I.nnz > 0) {
         const bool dcsr = S.dev_dcsr;
-        if (nrhs == 1) {
+        if (nrhs == 1 && I.impl == SPTRSV_IMPL_SQ_ADAPT) {
+          const int nitem = (int)(S.sq_items.size() / 4);
+          const auto* items = (const k::SqItem*)S.d_sq_items;
+          unsigned g = cdiv(nitem, 8);
+          if (dcsr)
+            k::sq_adapt_1<T, true><<<g, 256, 0, s>>>(nitem, I.row0, items, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
+          else
+            k::sq_adapt_1<T, false><<<g, 256, 0, s>>>(nitem, I.row0, items, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
+        } else if (nrhs == 1) {
           if (I.impl == SPTRSV_IMPL_SQ_VECTOR) {
             unsigned g = cdiv((int64_t)S.dev_nzr * 32, 256);
             if (dcsr)
@@ -994,8 +1005,7 @@ Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs
     int64_t stride = layout == SPTRSV_ROW_MAJOR ? ldb : 1;
     k::perm_in_1<T><<<std::max(1u, cdiv(n, 256)), 256, 0, s>>>(n, p.d_perm, rd, b, stride, bw, xs, fill, st);
   } else if (layout == SPTRSV_COL_MAJOR) {
-    dim3 g(std::max(1u, cdiv(n, 32)), cdiv(nrhs, 32));
-    k::perm_in_cm<T><<<g, dim3(32, 8), 0, s>>>(n, nrhs, iperm, rd, b, ldb, bw, xs, fill, st);
+    k::perm_in_cm<T><<<std::max(1u, cdiv(n, 32)), 256, 0, s>>>(n, nrhs, iperm, rd, b, ldb, bw, xs, fill, st);
   } else {
     k::perm_in_rm<T><<<std::max(1u, cdiv((int64_t)n * nrhs, 256)), 256, 0, s>>>(n, nrhs, p.d_perm, rd, b, ldb, bw,
                                                                                  xs, fill, st);
@@ -1009,8 +1019,7 @@ Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs
     int64_t stride = layout == SPTRSV_ROW_MAJOR ? ldx : 1;
     k::perm_out_1<T><<<std::max(1u, cdiv(n, 256)), 256, 0, s>>>(n, p.d_perm, xs, x, stride);
   } else if (layout == SPTRSV_COL_MAJOR) {
-    dim3 g(std::max(1u, cdiv(n, 32)), cdiv(nrhs, 32));
-    k::perm_out_cm<T><<<g, dim3(32, 8), 0, s>>>(n, nrhs, iperm, xs, x, ldx);
+    k::perm_out_cm<T><<<std::max(1u, cdiv(n, 32)), 256, 0, s>>>(n, nrhs, iperm, xs, x, ldx);
   } else {
     k::perm_out_rm<T><<<std::max(1u, cdiv((int64_t)n * nrhs, 256)), 256, 0, s>>>(n, nrhs, p.d_perm, xs, x, ldx);
   }
@@ -1034,10 +1043,89 @@ bool is_device_ptr(const void* ptr) {
 
 }  // namespace
 
+// Work items of the row-block square kernel (k::sq_adapt_1): greedy runs of
+// <= 32 consecutive stored rows with <= kSqNB entries; a longer row is an
+// item of its own, cut into kSqLW-entry chunks (flagged: atomic update) when
+// longer than kSqLW.
+void build_sq_items(Segment& S) {
+  S.sq_items.clear();
+  const auto& I = S.info;
+  if (I.kind != 1 || I.impl != SPTRSV_IMPL_SQ_ADAPT || S.nzr == 0) return;
+  const int nzr = S.nzr;
+  const std::vector<int32_t>& rp = S.rp;
+  auto push = [&](int t0, int t1, int p0, int p1, bool split) {
+    S.sq_items.push_back(t0);
+    S.sq_items.push_back(split ? (int32_t)((uint32_t)t1 | 0x80000000u) : t1);
+    S.sq_items.push_back(p0);
+    S.sq_items.push_back(p1);
+  };
+  int t = 0;
+  while (t < nzr) {
+    const int len = rp[t + 1] - rp[t];
+    if (len > k::kSqNB) {
+      if (len <= k::kSqLW) {
+        push(t, t + 1, rp[t], rp[t + 1], false);
+      } else {
+        for (int p0 = rp[t]; p0 < rp[t + 1]; p0 += k::kSqLW)
+          push(t, t + 1, p0, std::min(p0 + k::kSqLW, rp[t + 1]), true);
+      }
+      ++t;
+      continue;
+    }
+    const int start = t;
+    int tot = 0;
+    while (t < nzr && t - start < 32 && tot + (rp[t + 1] - rp[t]) <= k::kSqNB) {
+      tot += rp[t + 1] - rp[t];
+      ++t;
+    }
+    push(start, t, rp[start], rp[t], false);
+  }
+}
+
+// Host -> device upload of the plan through pinned staging: pageable
+// cudaMemcpy runs at a fraction of PCIe / C2C bandwidth, so large pieces are
+// copied (in parallel) into one of two pinned 32 MB buffers, each sent with
+// an async copy while the other is being filled.  Small pieces go directly.
+struct PinnedStager {
+  static constexpr size_t kBuf = size_t(32) << 20;
+  char* buf[2] = {nullptr, nullptr};
+  cudaEvent_t ev[2] = {nullptr, nullptr};
+  int cur = 0;
+  bool ok = false;
+  cudaStream_t s = nullptr;
+  PinnedStager() {
+    ok = cudaHostAlloc((void**)&buf[0], kBuf, cudaHostAllocDefault) == cudaSuccess &&
+         cudaHostAlloc((void**)&buf[1], kBuf, cudaHostAllocDefault) == cudaSuccess &&
+         cudaEventCreateWithFlags(&ev[0], cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&ev[1], cudaEventDisableTiming) == cudaSuccess;
+    if (!ok) cudaGetLastError();
+  }
+  cudaError_t put(char* dst, const void* src, size_t bytes) {
+    if (!bytes) return cudaSuccess;
+    if (!ok || bytes < (size_t(1) << 20)) return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, s);
+    const char* sp = (const char*)src;
+    for (size_t o = 0; o < bytes; o += kBuf) {
+      const size_t nb = std::min(kBuf, bytes - o);
+      cudaError_t e = cudaEventSynchronize(ev[cur]);  // the buffer's previous copy is done
+      if (e != cudaSuccess) return e;
+      char* b = buf[cur];
+      par_for((int64_t)nb, 0, [&](int64_t a, int64_t z) { std::memcpy(b + a, sp + o + a, (size_t)(z - a)); },
+              int64_t(4) << 20);
+      e = cudaMemcpyAsync(dst + o, b, nb, cudaMemcpyHostToDevice, s);
+      if (e != cudaSuccess) return e;
+      e = cudaEventRecord(ev[cur], s);
+      if (e != cudaSuccess) return e;
+      cur ^= 1;
+    }
+    return cudaSuccess;
+  }
+};
+
 Error upload(Plan& p, void* stream_v) {
   cudaStream_t s = (cudaStream_t)stream_v;
   const size_t vb = p.vbytes;
   const int n = p.n;
+  PhaseClock clk;
   // ---- arena layout (one allocation, segments in execution order, L229) ----
   size_t off = 0;
   auto take = [&](size_t bytes) {
@@ -1047,7 +1135,7 @@ Error upload(Plan& p, void* stream_v) {
   };
   size_t o_perm = take((size_t)2 * n * 4);  // perm (new->old) then iperm (old->new)
   size_t o_rdiag = take((size_t)n * vb);
-  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed, sd, sc, sv, sbk, ps, pd, pc; };
+  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed, sd, sc, sv, sbk, ps, pd, pc, sq; };
   std::vector<Offs> so(p.segs.size());
   p.trace = std::getenv("SPTRSV_TRACE") != nullptr;
   p.spmm = spmm_cfg();
@@ -1060,6 +1148,7 @@ Error upload(Plan& p, void* stream_v) {
   p.needs_sentinel = false;
   p.needs_flags = false;
   for (size_t i = 0; i < p.segs.size(); ++i) build_wave(p, p.segs[i], vb);  // may switch a segment to CHAIN
+  clk.lap("upload: build_wave");
   // execution order of the rows on the device: identity except inside wave
   // triangles (strand-major, group-major); sigma: new (plan) index -> device row
   std::vector<int32_t> sigma;
@@ -1072,8 +1161,16 @@ Error upload(Plan& p, void* stream_v) {
       for (size_t q2 = 0; q2 < S.wave_tau.size(); ++q2) sigma[S.info.row0 + S.wave_tau[q2]] = S.info.row0 + (int)q2;
     }
   auto sg = [&](int32_t k2) { return sigma.empty() ? k2 : sigma[k2]; };
-  // device copies of the segment CSR in device row order
-  struct Dev { std::vector<int32_t> rp, ci, rows; std::vector<char> val; };
+  // device images of the segment CSR in device row order: views of the
+  // segment's own arrays, or owned re-ordered copies where sigma moves rows
+  struct Dev {
+    std::vector<int32_t> rp_o, rows_o;
+    dvec<int32_t> ci_o;
+    dvec<char> val_o;
+    const int32_t *rp = nullptr, *ci = nullptr, *rows = nullptr;
+    const char* val = nullptr;
+    size_t nrp = 0, nci = 0, nrows = 0, nval = 0;
+  };
   std::vector<Dev> dv(p.segs.size());
   for (size_t i = 0; i < p.segs.size(); ++i) {
     Segment& S = p.segs[i];
@@ -1081,40 +1178,53 @@ Error upload(Plan& p, void* stream_v) {
     const auto& I = S.info;
     if (I.kind == 0 && S.wave_K > 0) {  // rows permuted by wave_tau
       const int m = I.row1 - I.row0;
-      D.rp.assign(m + 1, 0);
-      D.ci.reserve(S.ci.size());
-      D.val.reserve(S.val.size());
+      D.rp_o.assign(m + 1, 0);
+      D.ci_o.reserve(S.ci.size());
+      D.val_o.reserve(S.val.size());
       for (int q2 = 0; q2 < m; ++q2) {
         const int r = S.wave_tau[q2];
-        for (int e = S.rp[r]; e < S.rp[r + 1]; ++e) D.ci.push_back(sg(S.ci[e]));
-        D.val.insert(D.val.end(), S.val.begin() + (size_t)S.rp[r] * vb, S.val.begin() + (size_t)S.rp[r + 1] * vb);
-        D.rp[q2 + 1] = (int32_t)D.ci.size();
+        for (int e = S.rp[r]; e < S.rp[r + 1]; ++e) D.ci_o.push_back(sg(S.ci[e]));
+        D.val_o.insert(D.val_o.end(), S.val.begin() + (size_t)S.rp[r] * vb, S.val.begin() + (size_t)S.rp[r + 1] * vb);
+        D.rp_o[q2 + 1] = (int32_t)D.ci_o.size();
       }
+      D.rp = D.rp_o.data(); D.nrp = D.rp_o.size();
+      D.ci = D.ci_o.data(); D.nci = D.ci_o.size();
+      D.val = D.val_o.data(); D.nval = D.val_o.size();
     } else {
-      D.rp = S.rp;
-      D.ci = S.ci;
-      if (!sigma.empty())
-        for (auto& c : D.ci) c = sigma[c];
-      D.val = S.val;
+      D.rp = S.rp.data(); D.nrp = S.rp.size();
+      D.val = S.val.data(); D.nval = S.val.size();
+      if (!sigma.empty()) {
+        D.ci_o.resize(S.ci.size());
+        for (size_t q2 = 0; q2 < S.ci.size(); ++q2) D.ci_o[q2] = sigma[S.ci[q2]];
+        D.ci = D.ci_o.data();
+      } else {
+        D.ci = S.ci.data();
+      }
+      D.nci = S.ci.size();
     }
     S.dev_dcsr = I.kind == 1 && I.format == SPTRSV_FMT_DCSR;
     S.dev_nzr = S.nzr;
+    D.rows = S.rows.data();
+    D.nrows = S.rows.size();
     if (I.kind == 1) {
       if (S.dev_dcsr) {
-        D.rows = S.rows;
-        for (auto& r : D.rows) r = sg(r);
+        if (!sigma.empty()) {
+          D.rows_o = S.rows;
+          for (auto& r : D.rows_o) r = sg(r);
+          D.rows = D.rows_o.data();
+        }
       } else {
         bool moved = false;
         for (int r = I.row0; r < I.row1 && !sigma.empty() && !moved; ++r) moved = sigma[r] != r;
         if (moved) {  // CSR rows reordered: upload as DCSR with every row listed
           S.dev_dcsr = true;
-          D.rows.resize(I.row1 - I.row0);
-          for (int r = I.row0; r < I.row1; ++r) D.rows[r - I.row0] = sigma[r];
+          D.rows_o.resize(I.row1 - I.row0);
+          for (int r = I.row0; r < I.row1; ++r) D.rows_o[r - I.row0] = sigma[r];
+          D.rows = D.rows_o.data();
+          D.nrows = D.rows_o.size();
           S.dev_nzr = I.row1 - I.row0;
         }
       }
-    } else {
-      D.rows = S.rows;
     }
   }
   for (size_t i = 0; i < p.segs.size(); ++i) {
@@ -1122,12 +1232,13 @@ Error upload(Plan& p, void* stream_v) {
     build_chain_stages(S, cg);
     build_chain_ell(S, vb);
     build_supernodes(S, vb);
+    build_sq_items(S);
     so[i].er = take(S.ell_recs.size() * 4);
     so[i].ed = take(S.ell_data.size());
-    so[i].rp = take(dv[i].rp.size() * 4);
-    so[i].ci = take(dv[i].ci.size() * 4);
-    so[i].val = take(dv[i].val.size());
-    so[i].rows = take(dv[i].rows.size() * 4);
+    so[i].rp = take(dv[i].nrp * 4);
+    so[i].ci = take(dv[i].nci * 4);
+    so[i].val = take(dv[i].nval);
+    so[i].rows = take(dv[i].nrows * 4);
     so[i].lp = take(S.level_ptr.size() * 4);
     so[i].st = take(S.chain_recs.size() * 4);
     so[i].sd = take(S.sn_desc.size());
@@ -1137,6 +1248,7 @@ Error upload(Plan& p, void* stream_v) {
     so[i].ps = take(S.wave_strands.size());
     so[i].pd = take(S.wave_data.size());
     so[i].pc = take(S.wave_crows.size() * 4);
+    so[i].sq = take(S.sq_items.size() * 4);
     if (S.info.kind == 0) S.ticket_slot = p.nticket++;
     if (S.info.kind == 0 && (S.info.impl == SPTRSV_IMPL_TRI_SYNCFREE || S.info.impl == SPTRSV_IMPL_TRI_SUPERNODE ||
                              (S.info.impl == SPTRSV_IMPL_TRI_PIPE && (S.wave_K == 0 || S.wave_global > 0))))
@@ -1147,6 +1259,7 @@ Error upload(Plan& p, void* stream_v) {
   }
   size_t o_tickets = take((size_t)std::max(1, p.nticket) * 4);
   p.arena_bytes = off;
+  clk.lap("upload: chain/ell/supernode");
 
   int dev;
   CUDA_TRY(cudaGetDevice(&dev));
@@ -1155,8 +1268,10 @@ Error upload(Plan& p, void* stream_v) {
     cudaGetLastError();
     return {SPTRSV_ERROR_ALLOC, "plan arena allocation failed (" + std::to_string(off) + " bytes)"};
   }
-  // host staging of the whole arena, then one copy
-  std::vector<char> h(off, 0);
+  clk.lap("upload: cudaMalloc");
+  // perm / iperm / 1/d are composed on the host (sigma), every segment array
+  // is copied straight from its host vector (no staging image of the arena)
+  std::vector<char> h(o_rdiag + (size_t)n * vb, 0);
   // p.perm is in ORIGINAL indexing (UPPER: composed with J); the device
   // gathers b[perm_dev[k]] into device row k and scatters x back
   {
@@ -1171,44 +1286,56 @@ Error upload(Plan& p, void* stream_v) {
     }
   }
   char* A = (char*)p.arena;
+  CUDA_TRY(cudaMemsetAsync(A, 0, off, s));  // padding and tickets
+  CUDA_TRY(cudaMemcpyAsync(A, h.data(), h.size(), cudaMemcpyHostToDevice, s));
+  // one stager per process (pinned buffers are costly to allocate), used
+  // by one upload at a time
+  static std::mutex stager_mu;
+  static PinnedStager* stager = nullptr;
+  std::lock_guard<std::mutex> stager_lock(stager_mu);
+  if (!stager) stager = new PinnedStager();
+  stager->s = s;
+  auto put = [&](size_t o, const void* src, size_t bytes) -> cudaError_t { return stager->put(A + o, src, bytes); };
   for (size_t i = 0; i < p.segs.size(); ++i) {
     Segment& S = p.segs[i];
     const Dev& D = dv[i];
-    std::memcpy(&h[so[i].rp], D.rp.data(), D.rp.size() * 4);
-    std::memcpy(&h[so[i].ci], D.ci.data(), D.ci.size() * 4);
-    std::memcpy(&h[so[i].val], D.val.data(), D.val.size());
-    std::memcpy(&h[so[i].rows], D.rows.data(), D.rows.size() * 4);
-    std::memcpy(&h[so[i].lp], S.level_ptr.data(), S.level_ptr.size() * 4);
-    std::memcpy(&h[so[i].st], S.chain_recs.data(), S.chain_recs.size() * 4);
+    CUDA_TRY(put(so[i].rp, D.rp, D.nrp * 4));
+    CUDA_TRY(put(so[i].ci, D.ci, D.nci * 4));
+    CUDA_TRY(put(so[i].val, D.val, D.nval));
+    CUDA_TRY(put(so[i].rows, D.rows, D.nrows * 4));
+    CUDA_TRY(put(so[i].lp, S.level_ptr.data(), S.level_ptr.size() * 4));
+    CUDA_TRY(put(so[i].st, S.chain_recs.data(), S.chain_recs.size() * 4));
     S.d_rp = (const int32_t*)(A + so[i].rp);
     S.d_ci = (const int32_t*)(A + so[i].ci);
     S.d_val = (const void*)(A + so[i].val);
     S.d_rows = (const int32_t*)(A + so[i].rows);
     S.d_level_ptr = (const int32_t*)(A + so[i].lp);
     S.d_chain_recs = (const int32_t*)(A + so[i].st);
-    std::memcpy(&h[so[i].er], S.ell_recs.data(), S.ell_recs.size() * 4);
-    std::memcpy(&h[so[i].ed], S.ell_data.data(), S.ell_data.size());
+    CUDA_TRY(put(so[i].er, S.ell_recs.data(), S.ell_recs.size() * 4));
+    CUDA_TRY(put(so[i].ed, S.ell_data.data(), S.ell_data.size()));
     S.d_ell_recs = (const int32_t*)(A + so[i].er);
     S.d_ell_data = (const char*)(A + so[i].ed);
-    std::memcpy(&h[so[i].sd], S.sn_desc.data(), S.sn_desc.size());
-    std::memcpy(&h[so[i].sc], S.sn_cols.data(), S.sn_cols.size() * 4);
-    std::memcpy(&h[so[i].sv], S.sn_vals.data(), S.sn_vals.size());
-    std::memcpy(&h[so[i].sbk], S.sn_blk.data(), S.sn_blk.size());
+    CUDA_TRY(put(so[i].sd, S.sn_desc.data(), S.sn_desc.size()));
+    CUDA_TRY(put(so[i].sc, S.sn_cols.data(), S.sn_cols.size() * 4));
+    CUDA_TRY(put(so[i].sv, S.sn_vals.data(), S.sn_vals.size()));
+    CUDA_TRY(put(so[i].sbk, S.sn_blk.data(), S.sn_blk.size()));
     S.d_sn_desc = (const void*)(A + so[i].sd);
     S.d_sn_cols = (const int32_t*)(A + so[i].sc);
     S.d_sn_vals = (const void*)(A + so[i].sv);
     S.d_sn_blk = (const void*)(A + so[i].sbk);
-    std::memcpy(&h[so[i].ps], S.wave_strands.data(), S.wave_strands.size());
-    std::memcpy(&h[so[i].pd], S.wave_data.data(), S.wave_data.size());
+    CUDA_TRY(put(so[i].ps, S.wave_strands.data(), S.wave_strands.size()));
+    CUDA_TRY(put(so[i].pd, S.wave_data.data(), S.wave_data.size()));
     S.d_wave_strands = (const void*)(A + so[i].ps);
     S.d_wave_data = (const char*)(A + so[i].pd);
-    std::memcpy(&h[so[i].pc], S.wave_crows.data(), S.wave_crows.size() * 4);
+    CUDA_TRY(put(so[i].pc, S.wave_crows.data(), S.wave_crows.size() * 4));
     S.d_wave_crows = (const int32_t*)(A + so[i].pc);
+    CUDA_TRY(put(so[i].sq, S.sq_items.data(), S.sq_items.size() * 4));
+    S.d_sq_items = (const int32_t*)(A + so[i].sq);
   }
   p.d_perm = (const int32_t*)(A + o_perm);
   p.d_rdiag = (const void*)(A + o_rdiag);
   p.d_tickets = (uint32_t*)(A + o_tickets);
-  CUDA_TRY(cudaMemcpyAsync(p.arena, h.data(), off, cudaMemcpyHostToDevice, s));
+  clk.lap("upload: H2D copies issued");
   // mapped host word for the spin-wait watchdog
   if (cudaHostAlloc((void**)&p.h_error, sizeof(int32_t), cudaHostAllocMapped) == cudaSuccess) {
     *p.h_error = 0;
@@ -1219,6 +1346,7 @@ Error upload(Plan& p, void* stream_v) {
     p.d_error = nullptr;
   }
   CUDA_TRY(cudaStreamSynchronize(s));
+  clk.lap("upload: H2D complete");
   p.launches_per_solve = count_launches(p);
   return {SPTRSV_SUCCESS, ""};
 }

@@ -2,7 +2,14 @@
 // Not part of the ABI; see include/sptrsv.h.
 #pragma once
 
+#include <algorithm>
+#include <chrono>
 #include <cstdint>
+#include <functional>
+#include <thread>
+#include <cstdio>
+#include <cstdlib>
+#include <memory>
 #include <string>
 #include <vector>
 
@@ -18,6 +25,57 @@ struct Error {
 
 void set_last_error(const std::string& msg);
 
+// Allocator whose resize() leaves new elements default-initialised (i.e.
+// unwritten for scalars): the big index/value arrays of the analysis are
+// then first touched by the threads that fill them, in parallel, instead of
+// being zero-filled serially by resize().
+template <class T>
+struct DefaultInit : std::allocator<T> {
+  template <class U>
+  struct rebind { using other = DefaultInit<U>; };
+  DefaultInit() = default;
+  template <class U>
+  DefaultInit(const DefaultInit<U>&) noexcept {}
+  template <class U>
+  void construct(U* p) noexcept { ::new ((void*)p) U; }
+  template <class U, class... A>
+  void construct(U* p, A&&... a) { ::new ((void*)p) U(std::forward<A>(a)...); }
+};
+template <class T>
+using dvec = std::vector<T, DefaultInit<T>>;
+
+// Run f(lo, hi) over [0, n) split into contiguous chunks on `threads`
+// threads (threads <= 0: hardware concurrency, capped at 64); small ranges
+// run inline.
+inline void par_for(int64_t n, int threads, const std::function<void(int64_t, int64_t)>& f,
+                    int64_t grain = 65536) {
+  if (threads <= 0) threads = (int)std::min(64u, std::max(1u, std::thread::hardware_concurrency()));
+  if (threads <= 1 || n < grain) {
+    f(0, n);
+    return;
+  }
+  std::vector<std::thread> th;
+  for (int t = 0; t < threads; ++t) {
+    int64_t a = n * t / threads, b = n * (t + 1) / threads;
+    th.emplace_back([=, &f] { f(a, b); });
+  }
+  for (auto& x : th) x.join();
+}
+
+// Phase stopwatch of the preprocessing (SPTRSV_ANALYSE_TRACE=1 prints every
+// lap to stderr); costs one clock read per phase otherwise.
+struct PhaseClock {
+  bool on = std::getenv("SPTRSV_ANALYSE_TRACE") != nullptr;
+  std::chrono::steady_clock::time_point t = std::chrono::steady_clock::now();
+  void lap(const char* what) {
+    if (!on) return;
+    auto now = std::chrono::steady_clock::now();
+    std::fprintf(stderr, "[sptrsv analyse] %-28s %9.2f ms\n", what,
+                 std::chrono::duration<double, std::milli>(now - t).count());
+    t = now;
+  }
+};
+
 // One block of the reordered matrix P L P^T in execution order (Fig. 3(d),
 // PAPER.md:L229/L235): a triangle (solved) or a rectangle (b -= A x).
 struct Segment {
@@ -28,8 +86,8 @@ struct Segment {
   // CSR rows are local (0..m-1 for CSR, 0..nzr-1 for DCSR); columns are GLOBAL
   // permuted indices so kernels index the permuted vector directly.
   std::vector<int32_t> rp;         // CSR/DCSR row pointer (local offsets)
-  std::vector<int32_t> ci;         // global permuted column index
-  std::vector<char> val;           // dtype values
+  dvec<int32_t> ci;                // global permuted column index
+  dvec<char> val;                  // dtype values
   std::vector<int32_t> rows;       // DCSR: global permuted row of every stored row
   std::vector<int32_t> level_ptr;  // TRI: nlevels+1 local row offsets
   std::vector<int32_t> in_degree;  // TRI: off-diagonal count per local row
@@ -45,7 +103,8 @@ struct Segment {
   // supernodal kernel (nrhs == 1): piece descriptors, shared external
   // column lists, dense external values (column-major, ld = width) and the
   // packed strictly-lower diagonal blocks
-  std::vector<char> sn_desc, sn_vals, sn_blk;
+  std::vector<char> sn_desc;
+  dvec<char> sn_vals, sn_blk;
   std::vector<int32_t> sn_cols;
   const void* d_sn_desc = nullptr;
   const int32_t* d_sn_cols = nullptr;
@@ -66,6 +125,9 @@ struct Segment {
   // wave triangle is uploaded as DCSR with explicit (execution-order) rows
   bool dev_dcsr = false;
   int32_t dev_nzr = 0;
+  // row-block square kernel (k::sq_adapt_1, nrhs == 1): k::SqItem[] as 4 ints
+  std::vector<int32_t> sq_items;
+  const int32_t* d_sq_items = nullptr;
   // TMA-staged chain kernel (nrhs == 1): 8-int stage records (k::StageRec),
   // empty = not staged
   std::vector<int32_t> chain_recs;
@@ -116,8 +178,8 @@ struct Plan {
   std::vector<char> rdiag_new;      // 1 / diagonal in new order (dtype), what kernels read
   // P L P^T kept on the host for introspection (sptrsv_plan_matrix)
   std::vector<int64_t> p_rp;
-  std::vector<int32_t> p_ci;
-  std::vector<char> p_val;
+  dvec<int32_t> p_ci;
+  dvec<char> p_val;
 
   // ----- device -----
   int device = -1;

@@ -110,44 +110,98 @@ __global__ void perm_out_1(int n, const int* __restrict__ perm, const T* __restr
   if (k < n) x[(int64_t)perm[k] * stride] = xs[k];
 }
 
-// Column-major B (n x nrhs, ldb) -> row-major bw: a 32x32 tile transposed in
-// shared memory; reads are coalesced along original rows i, writes are 32
-// contiguous RHS values of the permuted row iperm[i].
+// Column-major B (n x nrhs, ldb) -> row-major bw.  A block owns 32 original
+// rows i and walks ALL the RHS columns in 32 x 32 tiles transposed through
+// shared memory: reads are coalesced along i (256 B per column), writes are
+// 256 B pieces of the permuted rows iperm[i], and each 4 KB (512-RHS) row is
+// completed by one block within a few microseconds (DRAM-page friendly, no
+// partial sectors left in L2).  The next tile's loads are in flight while
+// the current tile is stored.
 template <typename T>
-__global__ void perm_in_cm(int n, int nrhs, const int* __restrict__ iperm, const T* __restrict__ rd,
-                           const T* __restrict__ b, int64_t ldb, T* __restrict__ bw, T* __restrict__ xs,
-                           int fill_sent, SolveState st) {
+__global__ void __launch_bounds__(256) perm_in_cm(int n, int nrhs, const int* __restrict__ iperm,
+                                                  const T* __restrict__ rd, const T* __restrict__ b, int64_t ldb,
+                                                  T* __restrict__ bw, T* __restrict__ xs, int fill_sent,
+                                                  SolveState st) {
   __shared__ T tile[32][33];
-  if (blockIdx.x == 0 && blockIdx.y == 0) reset_tickets(st, threadIdx.y * 32 + threadIdx.x, 256);
-  int i0 = blockIdx.x * 32, c0 = blockIdx.y * 32;
-  for (int cc = threadIdx.y; cc < 32; cc += 8) {
-    int i = i0 + threadIdx.x, c = c0 + cc;
-    if (i < n && c < nrhs) tile[cc][threadIdx.x] = b[i + (int64_t)c * ldb];
+  __shared__ int ks[32];
+  __shared__ T rs[32];
+  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+  if (blockIdx.x == 0) reset_tickets(st, threadIdx.x, 256);
+  const int i0 = blockIdx.x * 32, i = i0 + tx;
+  const bool iv = i < n;
+  if (threadIdx.x < 32) {
+    const int k = iv ? iperm[i] : 0;
+    ks[tx] = k;
+    rs[tx] = iv ? rd[k] : T(0);
   }
-  __syncthreads();
-  for (int ii = threadIdx.y; ii < 32; ii += 8) {
-    int i = i0 + ii, c = c0 + threadIdx.x;
-    if (i < n && c < nrhs) {
-      int k = iperm[i];
-      bw[(int64_t)k * nrhs + c] = tile[threadIdx.x][ii] * rd[k];
-      if (fill_sent) xs[(int64_t)k * nrhs + c] = sent<T>();
+  T v[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const int c = ty + 8 * j;
+    v[j] = (iv && c < nrhs) ? ldg_nc(b + i + (int64_t)c * ldb) : T(0);
+  }
+  for (int c0 = 0; c0 < nrhs; c0 += 32) {
+    __syncthreads();  // the previous tile has been read out
+#pragma unroll
+    for (int j = 0; j < 4; ++j) tile[ty + 8 * j][tx] = v[j];
+    __syncthreads();
+    if (c0 + 32 < nrhs) {
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int c = c0 + 32 + ty + 8 * j;
+        v[j] = (iv && c < nrhs) ? ldg_nc(b + i + (int64_t)c * ldb) : T(0);
+      }
+    }
+    const int c = c0 + tx;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int ii = ty + 8 * j;
+      if (i0 + ii < n && c < nrhs) {
+        const int64_t o = (int64_t)ks[ii] * nrhs + c;
+        bw[o] = tile[tx][ii] * rs[ii];
+        if (fill_sent) xs[o] = sent<T>();
+      }
     }
   }
 }
 
+// x = P^T xs for column-major X: the mirror of perm_in_cm (a block gathers
+// 256 B pieces of 32 permuted rows, writes 32 consecutive rows per column).
 template <typename T>
-__global__ void perm_out_cm(int n, int nrhs, const int* __restrict__ iperm, const T* __restrict__ xs,
-                            T* __restrict__ x, int64_t ldx) {
+__global__ void __launch_bounds__(256) perm_out_cm(int n, int nrhs, const int* __restrict__ iperm,
+                                                   const T* __restrict__ xs, T* __restrict__ x, int64_t ldx) {
   __shared__ T tile[32][33];
-  int i0 = blockIdx.x * 32, c0 = blockIdx.y * 32;
-  for (int ii = threadIdx.y; ii < 32; ii += 8) {
-    int i = i0 + ii, c = c0 + threadIdx.x;
-    if (i < n && c < nrhs) tile[threadIdx.x][ii] = xs[(int64_t)iperm[i] * nrhs + c];
-  }
+  __shared__ int ks[32];
+  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+  const int i0 = blockIdx.x * 32;
+  if (threadIdx.x < 32) ks[tx] = i0 + tx < n ? iperm[i0 + tx] : 0;
   __syncthreads();
-  for (int cc = threadIdx.y; cc < 32; cc += 8) {
-    int i = i0 + threadIdx.x, c = c0 + cc;
-    if (i < n && c < nrhs) x[i + (int64_t)c * ldx] = tile[cc][threadIdx.x];
+  T v[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const int ii = ty + 8 * j;
+    v[j] = (i0 + ii < n && tx < nrhs) ? ldg_nc(xs + (int64_t)ks[ii] * nrhs + tx) : T(0);
+  }
+  const int i = i0 + tx;
+  for (int c0 = 0; c0 < nrhs; c0 += 32) {
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < 4; ++j) tile[ty + 8 * j][tx] = v[j];
+    __syncthreads();
+    if (c0 + 32 < nrhs) {
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int ii = ty + 8 * j, c = c0 + 32 + tx;
+        v[j] = (i0 + ii < n && c < nrhs) ? ldg_nc(xs + (int64_t)ks[ii] * nrhs + c) : T(0);
+      }
+    }
+    if (i < n) {
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int c = c0 + ty + 8 * j;
+        if (c < nrhs) x[i + (int64_t)c * ldx] = tile[tx][ty + 8 * j];
+      }
+    }
   }
 }
 
@@ -213,6 +267,93 @@ __global__ void sq_vector_1(int nzr, int r0, const int* __restrict__ rows, const
   if (lane == 0) {
     int r = DCSR ? rows[wid] : r0 + wid;
     bw[r] -= s;
+  }
+}
+
+// B200 square update (nrhs == 1, selector B200): nnz-balanced ROW BLOCKS.
+// The upload cuts the stored rows into work items of <= 32 consecutive rows
+// holding <= kSqNB entries together (a row longer than kSqNB is an item of
+// its own, cut into kSqLW-entry chunks when longer still), one warp each.
+// A block streams its entries coalesced -- every lane issues all its
+// (ci, val) loads, then all its x gathers, before the first use, so
+// kSqNB / 32 independent gathers per lane are in flight -- into shared
+// memory as products; then lane t sums row t0 + t from shared memory and
+// updates b'.  Rows of any length mix in one launch with full lanes (the
+// paper's scalar / vector kernels leave lanes idle on short rows and
+// serialise long ones, L249-L250).  A row cut into several chunks adds its
+// partial sums with atomics (summation order then varies, reading R22).
+constexpr int kSqNB = 256, kSqLW = 1024;
+struct SqItem {
+  int t0, t1;  // stored rows [t0, t1); bit 31 of t1: chunk of a split row (atomic update)
+  int p0, p1;  // entries [p0, p1)
+};
+
+template <typename T, bool DCSR>
+__global__ void __launch_bounds__(256) sq_adapt_1(int nitem, int r0, const SqItem* __restrict__ items,
+                                                  const int* __restrict__ rows, const int* __restrict__ rp,
+                                                  const int* __restrict__ ci, const T* __restrict__ val,
+                                                  const T* __restrict__ xs, T* __restrict__ bw) {
+  __shared__ T prod[8][kSqNB];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int w = blockIdx.x * 8 + warp;
+  if (w >= nitem) return;
+  const int4 it = __ldg((const int4*)(items + w));
+  const int t0 = it.x, t1 = it.y & 0x7fffffff, a = it.z, e = it.w;
+  if (it.y < 0 || e - a > kSqNB) {  // one long row, or a chunk of a split one (any length)
+    T s[4] = {0, 0, 0, 0};
+    for (int p = a + lane; p < e; p += 128) {
+      int j[4];
+      T v[4], x[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (p + 32 * u < e) {
+          j[u] = ldg_nc(ci + p + 32 * u);
+          v[u] = ldg_nc(val + p + 32 * u);
+        }
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (p + 32 * u < e) x[u] = ldg_nc(xs + j[u]);
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (p + 32 * u < e) s[u] += v[u] * x[u];
+    }
+    const T sum = warp_sum((s[0] + s[1]) + (s[2] + s[3]));
+    if (lane == 0) {
+      const int r = DCSR ? rows[t0] : r0 + t0;
+      if (it.y < 0)
+        atomicAdd(bw + r, -sum);
+      else
+        bw[r] -= sum;
+    }
+    return;
+  }
+  T* pr = prod[warp];
+  int j[kSqNB / 32];
+  T v[kSqNB / 32], x[kSqNB / 32];
+#pragma unroll
+  for (int u = 0; u < kSqNB / 32; ++u) {
+    const int p = a + 32 * u + lane;
+    if (p < e) {
+      j[u] = ldg_nc(ci + p);
+      v[u] = ldg_nc(val + p);
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < kSqNB / 32; ++u)
+    if (a + 32 * u + lane < e) x[u] = ldg_nc(xs + j[u]);
+#pragma unroll
+  for (int u = 0; u < kSqNB / 32; ++u)
+    if (a + 32 * u + lane < e) pr[32 * u + lane] = v[u] * x[u];
+  __syncwarp();
+  const int t = t0 + lane;
+  if (t < t1) {
+    const int q0 = rp[t] - a, q1 = rp[t + 1] - a;
+    if (q1 > q0) {
+      T sum = 0;
+      for (int q = q0; q < q1; ++q) sum += pr[q];
+      const int r = DCSR ? rows[t] : r0 + t;
+      bw[r] -= sum;
+    }
   }
 }
 

@@ -59,7 +59,7 @@ def test_small_configs_default(gpu, name, selector):
 
 @pytest.mark.parametrize("name", CONFIGS)
 @pytest.mark.parametrize("tri", ["TRI_LEVELSET", "TRI_SYNCFREE", "TRI_CHAIN", "TRI_SUPERNODE", "TRI_PIPE"])
-@pytest.mark.parametrize("sq", ["SQ_SCALAR", "SQ_VECTOR"])
+@pytest.mark.parametrize("sq", ["SQ_SCALAR", "SQ_VECTOR", "SQ_ADAPT"])
 def test_forced_kernels(gpu, name, tri, sq):
     M, b = g.gen_config(name, small=True, nrhs=1)
     if tri == "TRI_LEVELSET" and name in ("C2",):
@@ -274,3 +274,21 @@ def test_wave_is_the_c2_default(gpu):
     _check64(M, b[:1], x)
     x3, _ = _solve(M, b, depth=1)
     _check64(M, b, x3)
+
+
+@pytest.mark.parametrize("depth", [1, 3])
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+@pytest.mark.parametrize("reorder", [False, True])
+def test_square_row_blocks(gpu, depth, dtype, reorder):
+    """The B200 row-block square kernel on rows of every length class:
+    empty, short, 257-1024 entries (one warp alone) and > 1024 entries (split
+    into chunks with atomic partial sums)."""
+    M = g.shape_long_rows()
+    b = g.gen_rhs(M.n, 1)
+    x, plan = _solve(M, b, dtype=dtype, depth=depth, reorder=reorder, force_sq_impl="SQ_ADAPT")
+    sqs = [s for s in plan.segments() if s["kind"] == "SQ"]
+    assert sqs and all(s["impl"] == "SQ_ADAPT" for s in sqs)
+    if dtype == torch.float64:
+        _check64(M, b, x)
+    else:
+        assert on.rel_err(x, on.solve(M, b)) <= TOL32

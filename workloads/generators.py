@@ -376,6 +376,29 @@ def shape_random_small(n: int, density: float, seed: int) -> Matrix:
     return _assemble(n, r[keep], c[keep], rng, f"random_{n}_{density}")
 
 
+def shape_long_rows(n: int = 6000, seed: int = 11) -> Matrix:
+    """Rows of every length class of the row-block square kernel: empty,
+    short (1-20), medium (257-1024 entries: one warp alone) and very long
+    (> 1024: split into chunks), scattered over the lower half."""
+    rng = _rng(seed)
+    rows, cols = [], []
+    for i in range(1, n):
+        u = rng.random()
+        if i < n // 2 or u < 0.2:
+            k = min(i, int(rng.integers(0, 4)))
+        elif u < 0.9:
+            k = min(i, int(rng.integers(1, 21)))
+        elif u < 0.97:
+            k = min(i, int(rng.integers(257, 1025)))
+        else:
+            k = min(i, int(rng.integers(1025, 2900)))
+        if k:
+            c = rng.choice(i, size=k, replace=False)
+            rows.append(np.full(k, i))
+            cols.append(c)
+    return _assemble(n, np.concatenate(rows), np.concatenate(cols), rng, "long_rows")
+
+
 def to_upper(L: Matrix) -> Matrix:
     """U = J L J (index reversal i -> n-1-i): an upper-triangular CSR whose
     diagonal is the FIRST entry of its row.  Pure re-indexing."""
