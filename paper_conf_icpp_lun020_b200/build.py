@@ -20,6 +20,8 @@ NVCC = os.environ.get("NVCC", shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc"
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-fvisibility=hidden,-O3",
           "-I", INCLUDE, "-I", CSRC]
+# extra nvcc flags for instrumented builds (e.g. -DSPTRSV_WAVE_TRACE); never set by the driver
+COMMON += os.environ.get("SPTRSV_NVCC_FLAGS", "").split()
 
 
 def _stale(out: str, deps: list[str]) -> bool:

@@ -407,12 +407,12 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   auto& I = S.info;
   if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_PIPE) return;
   const int m = I.row1 - I.row0;
-  int C = 16, W = 2, GPC = 12, NCH = 4;
+  int C = 16, W = 2, GPC = k::kWaveGpcBig, NCH = 4;
   if (const char* e = std::getenv("SPTRSV_WAVE")) {
     int a, b2, c, d;
     if (std::sscanf(e, "%d,%d,%d,%d", &a, &b2, &c, &d) == 4 && a >= 1 && a <= 16 && b2 >= 1 && b2 <= 8 &&
         c >= 1 && c <= 32 && d >= 2 && d <= 4) {
-      C = a; W = b2; GPC = c <= 6 ? 6 : 12; NCH = d;
+      C = a; W = b2; GPC = c <= 6 ? 6 : k::kWaveGpcBig; NCH = d;
     }
   }
   auto give_up = [&]() {
@@ -571,7 +571,37 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   }
   const uint32_t gbytes = vb == 8 ? k::wave_group_bytes<double>(Kt, E) : k::wave_group_bytes<float>(Kt, E);
   const uint32_t hbytes = k::wave_hdr_bytes(GPC);
-  const uint32_t cbytes = hbytes + (uint32_t)GPC * gbytes;
+  // first-use import list per chunk (what chunk_wait polls): its length
+  std::vector<std::vector<std::vector<uint32_t>>> clist(NS);
+  int max_ci = 0;
+  {
+    const uint32_t VB0 = (uint32_t)vb;
+    for (int s2 = 0; s2 < NS; ++s2) {
+      std::vector<char> seen(nimp[s2], 0);
+      const auto& Gs = groups[s2];
+      const auto& R = srows[s2];
+      const int nch = (int)((Gs.size() + GPC - 1) / GPC);
+      clist[s2].resize(nch);
+      for (int c = 0; c < nch; ++c) {
+        for (int g2 = c * GPC; g2 < std::min<int>((int)Gs.size(), (c + 1) * GPC); ++g2)
+          for (int l = 0; l < Gs[g2].second; ++l) {
+            const int r = R[Gs[g2].first + l];
+            for (int e = S.rp[r]; e < S.rp[r + 1]; ++e)
+              if (dep[e].kind == 1 && !seen[dep[e].b]) {
+                seen[dep[e].b] = 1;
+                clist[s2][c].push_back((uint32_t)(imp_base[s2] + dep[e].b) * VB0);
+              }
+          }
+        max_ci = std::max<int>(max_ci, (int)clist[s2][c].size());
+      }
+    }
+  }
+  const int ipl = (max_ci + 31) / 32;
+  const uint32_t cbytes = hbytes + (uint32_t)GPC * gbytes + (uint32_t)ipl * 128u;
+  {  // the import lists must still fit next to the x area (else: the chain kernel)
+    const int64_t need = (int64_t)k::al16((uint32_t)xa * (uint32_t)vb) + (int64_t)W * NCH * (cbytes + bring + 16);
+    if (need > 232448) return give_up();
+  }
   // chunks
   std::vector<k::WaveStrand> sr(NS);
   std::vector<int32_t> nchunk(NS);
@@ -598,6 +628,8 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
     W2.nchunk = nchunk[s2];
     W2.ngroups = (int)groups[s2].size();
     W2.row0 = r0 + s_start[s2];
+    W2.imp_lo = (uint32_t)imp_base[s2] * VB;
+    W2.imp_hi = (uint32_t)(imp_base[s2] + nimp[s2]) * VB;
     const auto& Gs = groups[s2];
     const auto& R = srows[s2];
     auto chunk_rows = [&](int c, int& lo, int& hi) {
@@ -642,6 +674,8 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
         }
         gh[1] = Gs[g].second | flags;
       }
+      uint32_t* il = (uint32_t*)(B + hbytes + (size_t)GPC * gbytes);
+      for (size_t i = 0; i < clist[s2][c].size(); ++i) il[i] = clist[s2][c][i];  // rest: 0 = the zero slot
     }
     off += (size_t)nchunk[s2] * cbytes;
   }
@@ -660,13 +694,15 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   S.wave_chunk_bytes = cbytes;
   S.wave_bring_bytes = bring;
   S.wave_group_bytes = gbytes;
+  S.wave_ipl = ipl;
   S.wave_global = nglobal;
 }
 
 template <typename T, int K, int E, int GPC, bool GLB>
 Error launch_wave_t(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
   k::WaveGeom g{S.wave_W,           S.wave_GPC,         S.wave_NCH,         S.wave_xa,
-                S.wave_chunk_bytes, S.wave_bring_bytes, S.wave_group_bytes, k::wave_hdr_bytes(S.wave_GPC)};
+                S.wave_chunk_bytes, S.wave_bring_bytes, S.wave_group_bytes, k::wave_hdr_bytes(S.wave_GPC),
+                S.wave_ipl};
   const uint32_t smem = k::wave_smem_bytes<T>(g);
   auto kern = k::tri_wave<T, K, E, GPC, GLB>;
   static uint32_t attr_bytes = 0;  // per template instance
@@ -704,7 +740,8 @@ Error launch_wave_e(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, c
   const bool glb = S.wave_global > 0;
   if (S.wave_GPC == 6)
     return glb ? launch_wave_t<T, K, E, 6, true>(p, S, bw, xs, st, s) : launch_wave_t<T, K, E, 6, false>(p, S, bw, xs, st, s);
-  return glb ? launch_wave_t<T, K, E, 12, true>(p, S, bw, xs, st, s) : launch_wave_t<T, K, E, 12, false>(p, S, bw, xs, st, s);
+  return glb ? launch_wave_t<T, K, E, k::kWaveGpcBig, true>(p, S, bw, xs, st, s)
+             : launch_wave_t<T, K, E, k::kWaveGpcBig, false>(p, S, bw, xs, st, s);
 }
 
 template <typename T, int K>

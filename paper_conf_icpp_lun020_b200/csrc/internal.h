@@ -113,6 +113,7 @@ struct Segment {
   // strand wavefront over a cluster (k::tri_wave, nrhs == 1); wave_K == 0: not built
   int wave_K = 0, wave_E = 0, wave_C = 0, wave_W = 0, wave_GPC = 0, wave_NCH = 0, wave_XW = 0, wave_xa = 0;
   uint32_t wave_chunk_bytes = 0, wave_bring_bytes = 0, wave_group_bytes = 0;
+  int wave_ipl = 0;                // words per lane of a chunk's first-use import list
   int64_t wave_global = 0;         // dependencies polled in global memory (needs the xs sentinel)
   std::vector<int32_t> wave_tau;   // execution position q -> local row (the device row order of the triangle)
   std::vector<char> wave_strands;  // k::WaveStrand[C * W]

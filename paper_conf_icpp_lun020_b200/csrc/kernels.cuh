@@ -1376,10 +1376,13 @@ constexpr int kWaveGF_GLOBAL = 1 << 30, kWaveGF_PUSH = 1 << 29, kWaveCntMask = (
 struct WaveStrand {
   int off16, nchunk, ngroups, row0;  // row0: first execution-order row of the strand
   int lo[4], hi[4];                  // b' row ranges of chunks 0..3 (the prologue loads)
+  uint32_t imp_lo, imp_hi;           // byte range of the strand's import slots in its CTA's x area
+  int pad[2];
 };
 struct WaveGeom {
   int W, GPC, NCH, xa_slots;  // warps per CTA, groups per chunk, ring depth, x area slots per CTA
   uint32_t chunk_bytes, bring_bytes, group_bytes, hdr_bytes;
+  int imp_per_lane;           // words per lane of a chunk's first-use import list (after its groups)
 };
 
 template <typename T>
@@ -1418,6 +1421,19 @@ __device__ __forceinline__ double lds_x_v(uint32_t a, double) {
 __device__ __forceinline__ float lds_x_v(uint32_t a, float) {
   float v;
   asm volatile("ld.volatile.shared.f32 %0, [%1];" : "=f"(v) : "r"(a));
+  return v;
+}
+// the level-chain x load: a "memory" clobber pins it ahead of the operand
+// prefetch that follows it in program order (the prefetch LDS then queue
+// behind it in the MIO pipe instead of delaying it)
+__device__ __forceinline__ double lds_x_first(uint32_t a, double) {
+  double v;
+  asm volatile("ld.volatile.shared.f64 %0, [%1];" : "=d"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ float lds_x_first(uint32_t a, float) {
+  float v;
+  asm volatile("ld.volatile.shared.f32 %0, [%1];" : "=f"(v) : "r"(a) : "memory");
   return v;
 }
 __device__ __forceinline__ void sts_x_v(uint32_t a, double v) {
@@ -1466,7 +1482,6 @@ struct WaveOp {
   uint32_t xo[K], so;
   uint32_t push[E > 0 ? E : 1];
   T v[K];
-  T xe[K];  // early poll of the dependencies (readiness test only)
   T b;
   int row, cnt;  // cnt with the group flags
 };
@@ -1503,6 +1518,17 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 // every strand's ring of NCH chunks filled by TMA (full / empty mbarriers),
 // so a consumer never issues a copy: at a chunk end it only arrives on the
 // slot's empty barrier and waits on the next slot's full barrier.
+#ifndef SPTRSV_WAVE_EXP
+#define SPTRSV_WAVE_EXP 0  // instrumented builds drop parts of the loop to time them (tuning only)
+#endif
+#ifndef SPTRSV_WAVE_WAIT_NS
+#define SPTRSV_WAVE_WAIT_NS 64
+#endif
+constexpr unsigned kWaveWaitNs = SPTRSV_WAVE_WAIT_NS;
+#ifndef SPTRSV_WAVE_GPC_BIG
+#define SPTRSV_WAVE_GPC_BIG 12
+#endif
+constexpr int kWaveGpcBig = SPTRSV_WAVE_GPC_BIG;  // groups per chunk (multiple of 3); 6 when smem is short
 template <typename T, int K, int E, int GPC, bool GLB>
 __global__ void __launch_bounds__(288, 1)
     tri_wave(const WaveStrand* __restrict__ strands, const char* __restrict__ data, const T* __restrict__ bw, T* __restrict__ xs, WaveGeom g, SolveState st, long long* __restrict__ trace) {
@@ -1599,43 +1625,21 @@ __global__ void __launch_bounds__(288, 1)
     o.row = gh.x + lane;
     o.cnt = gh.y;
   };
-  // early poll of a group's dependencies (readiness test only): issued a
-  // whole group before the test, so the test never waits on the load
-  auto early_poll = [&](WaveOp<T, K, E>& o) {
-    if (!GLB) {
-#pragma unroll
-      for (int k2 = 0; k2 < K; ++k2) o.xe[k2] = lds_x_v(xa_s + o.xo[k2], T(0));
-    }
-  };
   // the level-chain part of one group (cur resident)
-  auto solve_op = [&](WaveOp<T, K, E>& cur) -> T {
+  auto solve_op = [&](WaveOp<T, K, E>& cur, auto&& mid) -> T {
     T x[K];
     if (!GLB) {
-      // ---- level chain: the x_j loads go first (own-strand values were
-      // stored before the last __syncwarp); the readiness test uses the
-      // early poll and only sends the warp to the wait loop (then reloads)
-      // when a producer strand is behind
+      // ---- level chain: the x_j loads go first, then the next groups'
+      // operand prefetch (mid), which overlaps the load latency.  No
+      // readiness test here: own-strand values were stored by this warp
+      // before the last __syncwarp and every import of the chunk passed
+      // chunk_wait at the chunk's start, so the chain is branch-free
+      // (LDS x_j -> 2 DFMA -> STS x_i)
 #pragma unroll
-      for (int k2 = 0; k2 < K; ++k2) x[k2] = lds_x_v(xa_s + cur.xo[k2], T(0));
-      bool pend = false;
-#pragma unroll
-      for (int k2 = 0; k2 < K; ++k2) pend |= maybe_sent(cur.xe[k2]);
-      if (vote_any(pend)) {
-        for (;;) {
-          pend = false;
-#pragma unroll
-          for (int k2 = 0; k2 < K; ++k2) pend |= is_sent(lds_x_v(xa_s + cur.xo[k2], T(0)));
-          if (!vote_any(pend)) break;
-          ++npolls;
-          if (++spins > kWatchdogSpins) {
-            watchdog_trip(st);
-            break;
-          }
-        }
-#pragma unroll
-        for (int k2 = 0; k2 < K; ++k2) x[k2] = lds_x_v(xa_s + cur.xo[k2], T(0));
-      }
+      for (int k2 = 0; k2 < K; ++k2) x[k2] = lds_x_first(xa_s + cur.xo[k2], T(0));
+      mid();
     } else {
+      mid();
 #pragma unroll
       for (int k2 = 0; k2 < K; ++k2) {
         const bool glb = cur.xo[k2] & 0x80000000u;
@@ -1658,9 +1662,11 @@ __global__ void __launch_bounds__(288, 1)
   };
   auto publish = [&](WaveOp<T, K, E>& cur, T acc) {
     sts_x_v(xa_s + cur.so, acc);
+    if (!(SPTRSV_WAVE_EXP & 4)) {
 #pragma unroll
-    for (int e = 0; e < E; ++e) wave_push(cur.push[e], xa_s, acc);
-    if (lane < (cur.cnt & kWaveCntMask)) stg_x_v(xs + cur.row, acc);
+      for (int e = 0; e < E; ++e) wave_push(cur.push[e], xa_s, acc);
+    }
+    if (!(SPTRSV_WAVE_EXP & 2) && lane < (cur.cnt & kWaveCntMask)) stg_x_v(xs + cur.row, acc);
   };
 
   // three operand sets rotate over the groups (GPC % 3 == 0): group g solves
@@ -1675,11 +1681,37 @@ __global__ void __launch_bounds__(288, 1)
   const T* bbn = (const T*)bring;
   int slot_n = 0;
   uint32_t ph_n = 0;
+  // readiness of a whole chunk: every import slot its groups read must hold
+  // a pushed value (not the sentinel) before the chunk starts.  Imports flow
+  // only from lower strands, which never wait on this one, so the strand
+  // simply runs a chunk behind its producers; one vote per chunk replaces
+  // a branch per group on the level chain
+  const uint32_t imp_lo = Sp->imp_lo, imp_hi = Sp->imp_hi;
+  // The chunk block ends with the byte offsets of the imports the chunk
+  // uses first (padding: the zero slot), imp_per_lane words per lane.
+  auto chunk_wait = [&](const unsigned char* Bc) {
+    const uint32_t* il = (const uint32_t*)(Bc + g.hdr_bytes + (uint32_t)GPC * g.group_bytes);
+    uint32_t xo0 = 0;
+    if (!GLB && g.imp_per_lane > 0) xo0 = il[lane];
+    for (; !GLB && imp_lo != imp_hi;) {
+      bool pend = is_sent(lds_x_v(xa_s + xo0, T(0)));
+      for (int i = 1; i < g.imp_per_lane; ++i) pend |= is_sent(lds_x_v(xa_s + il[i * 32 + lane], T(0)));
+      if (!vote_any(pend)) break;
+      ++npolls;
+      // back off: a spinning warp's polls compete for the SM's shared-memory
+      // pipe with the CTA-mate strand that is doing real work
+      __nanosleep(kWaveWaitNs);
+      if (++spins > kWatchdogSpins) {
+        watchdog_trip(st);
+        break;
+      }
+    }
+  };
   if (s_nchunk > 0) {
     mbar_wait(&full[0], 0);
     load_op(B, bb, 0, op0);
     load_op(B, bb, 1, op1);
-    early_poll(op0);
+    chunk_wait(B);
   }
   for (int c = 0; c < s_nchunk; ++c) {
     const bool more = c + 1 < s_nchunk;
@@ -1695,20 +1727,20 @@ __global__ void __launch_bounds__(288, 1)
         tr[8 + c * GPC + gi] = gt;
       }
 #endif
-      const T acc = solve_op(cur);
-      if (gi + 1 < GPC || more) early_poll(n1);
-      if (gi + 2 < GPC) {
-        load_op(B, bb, gi + 2, n2);
-      } else if (more) {
-        if (gi + 2 == GPC) {  // open the next chunk two groups ahead
-          slot_n = slot + 1 == g.NCH ? 0 : slot + 1;
-          ph_n = slot + 1 == g.NCH ? ph ^ 1u : ph;
-          mbar_wait(&full[slot_n], ph_n);
-          Bn = ring + (size_t)slot_n * g.chunk_bytes;
-          bbn = (const T*)(bring + (size_t)slot_n * g.bring_bytes);
+      const T acc = solve_op(cur, [&]() {
+        if (gi + 2 < GPC) {
+          load_op(B, bb, gi + 2, n2);
+        } else if (more) {
+          if (gi + 2 == GPC) {  // open the next chunk two groups ahead
+            slot_n = slot + 1 == g.NCH ? 0 : slot + 1;
+            ph_n = slot + 1 == g.NCH ? ph ^ 1u : ph;
+            mbar_wait(&full[slot_n], ph_n);
+            Bn = ring + (size_t)slot_n * g.chunk_bytes;
+            bbn = (const T*)(bring + (size_t)slot_n * g.bring_bytes);
+          }
+          load_op(Bn, bbn, gi + 2 - GPC, n2);
         }
-        load_op(Bn, bbn, gi + 2 - GPC, n2);
-      }
+      });
       publish(cur, acc);
       if (gi + 1 == GPC) {  // chunk consumed: release its slot to the producer warp
         __syncwarp();
@@ -1717,8 +1749,9 @@ __global__ void __launch_bounds__(288, 1)
         ph = ph_n;
         B = Bn;
         bb = bbn;
+        if (more) chunk_wait(B);
       }
-      warp_sync_all();
+      if (!(SPTRSV_WAVE_EXP & 16)) warp_sync_all();
     }
   }
   if (tr && lane == 0) {
