@@ -1362,16 +1362,16 @@ __global__ void __launch_bounds__(1024, 1)
 // The loop (one warp = one strand) keeps only this on the level chain:
 //   __syncwarp -> LDS x_j -> 2 x DFMA -> STS x_i
 // (single-warp microbenchmark: ~51 cycles, scripts/microbench/wave_loop.cu).
-// Everything else is off it: the next group's operands are loaded during the
-// current group, and so is a first poll of its dependencies -- the readiness
-// test of other-strand values (import slots start as the sentinel) is made on
-// that early poll, so no branch waits on a fresh load (the microbenchmark
-// measured +65..90 cycles per group for any test of a just-loaded x).  The
-// value loaded at use time is always ready: own-strand values were stored by
-// this warp before the last __syncwarp, imports passed the early test (an
-// import slot is written once).  An early poll that still sees the sentinel
-// (producer strand behind; or, in a strand's first XW rows, an own slot not
-// yet written) sends the warp to the wait loop.
+// Everything else is off it: the operands of group g+2 are loaded while
+// group g waits for its x loads, and there is NO readiness test per group
+// (the microbenchmark and the SPTRSV_WAVE_EXP ablation measured ~63 cycles
+// per group for any vote + branch, wherever it sits).  Instead a strand
+// checks readiness once per chunk: the chunk block ends with the import
+// slots its groups use for the first time, and chunk_wait polls them (one
+// LDS per lane) until none is the sentinel.  Own-strand values were stored
+// by this warp before the last __syncwarp; an import slot is written once,
+// so a slot that passed its first-use chunk stays valid.  The price is a
+// lag of one chunk (GPC levels) per strand boundary of the wavefront.
 constexpr int kWaveGF_GLOBAL = 1 << 30, kWaveGF_PUSH = 1 << 29, kWaveCntMask = (1 << 29) - 1;
 struct WaveStrand {
   int off16, nchunk, ngroups, row0;  // row0: first execution-order row of the strand

@@ -130,6 +130,26 @@ def test_deterministic_across_thread_counts():
         assert np.array_equal(x, y)
 
 
+@pytest.mark.parametrize("uplo", ["L", "U"])
+def test_deterministic_across_thread_counts_large(uplo):
+    """n above the parallel grain (65,536 rows): the parallel validation,
+    J U J mapping, P L P^T, bottom-child reorders and segment extraction (per
+    segment with few threads, per row with many) give the same plan, bit for
+    bit, as one thread -- the replicated multi-GPU plan relies on it."""
+    M = g.c5_random_multirhs(n=150_001)
+    if uplo == "U":
+        M = g.to_upper(M)
+    plans = [_analyse(M, depth=3, threads=t) for t in (1, 5, 16)]
+    h = [p.hash() for p in plans]
+    assert h[0] == h[1] == h[2]
+    for p in plans[1:]:
+        assert np.array_equal(plans[0].perm(), p.perm())
+        assert plans[0].segments() == p.segments()
+        for x, y in zip(plans[0].matrix(), p.matrix()):
+            assert np.array_equal(x, y)
+    _compare(M, plans[1], st.analyse(M, depth=3))
+
+
 # ------------------------------------------------------------ validation
 def _expect(status, rp, ci, val, fill="L", **kw):
     with pytest.raises(sp.SptrsvError) as e:
@@ -153,6 +173,25 @@ def test_validation_error_names_row():
     with pytest.raises(sp.SptrsvError) as e:
         sp.sptrsv_analyse(np.array([0, 1, 2, 4]), np.array([0, 1, 0, 1]), np.ones(4), host_only=True)
     assert "row 2" in str(e.value)
+
+
+@pytest.mark.parametrize("threads", [1, 16])
+def test_validation_reports_lowest_bad_row_in_parallel(threads):
+    """Rows are validated in parallel chunks; the error is still the one a
+    serial row-order scan meets first (the lowest bad row)."""
+    M = g.c5_random_multirhs(n=150_001)
+    ci, val = M.col_idx.copy(), M.val.copy()
+    r_zero, r_unsorted = 120_003, 100_001  # zero pivot late, unsorted earlier
+    val[M.row_ptr[r_zero + 1] - 1] = 0.0
+    a = M.row_ptr[r_unsorted]
+    ci[a], ci[a + 1] = ci[a + 1], ci[a]
+    with pytest.raises(sp.SptrsvError) as e:
+        sp.sptrsv_analyse(M.row_ptr, ci, val, host_only=True, threads=threads)
+    assert e.value.status_name == "UNSORTED" and f"row {r_unsorted}" in str(e.value)
+    ci2 = M.col_idx.copy()
+    with pytest.raises(sp.SptrsvError) as e:
+        sp.sptrsv_analyse(M.row_ptr, ci2, val, host_only=True, threads=threads)
+    assert e.value.status_name == "ZERO_PIVOT" and f"row {r_zero}" in str(e.value)
 
 
 def test_float32_plan_structure_matches_float64():
