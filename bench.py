@@ -327,13 +327,23 @@ def main():
     # ---------------- roofline of the dominant kernel
     peak, peak_kind = load_peaks()
     seg_mean = seg_acc / args.steps  # [perm-in, seg..., perm-out]
-    names = ["permute_in"] + [f"seg{i}:{s['impl']}" for i, s in enumerate(segs)] + ["permute_out"]
+    def run_impl(sg):
+        """The kernel family that actually runs the segment at this nrhs: the
+        plan's impl for one RHS; with many RHS squares run the SpMM (sq_multi)
+        and the supernodal / wave triangles the multi-RHS sync-free kernel."""
+        if nrhs == 1:
+            return sg["impl"]
+        if sg["kind"] == "SQ":
+            return "SQ_SPMM"
+        return {"TRI_SUPERNODE": "TRI_SYNCFREE", "TRI_PIPE": "TRI_SYNCFREE"}.get(sg["impl"], sg["impl"])
+
+    names = ["permute_in"] + [f"seg{i}:{run_impl(s)}" for i, s in enumerate(segs)] + ["permute_out"]
     dom = int(np.argmax(seg_mean))
     dep = None
     if 1 <= dom <= len(segs):
         dseg = segs[dom - 1]
         dbytes = seg_alg_bytes(dseg, nrhs, vb)
-        dimpl = dseg["impl"]
+        dimpl = run_impl(dseg)
         if dseg["kind"] == "TRI" and dseg["nlevels"] > 1:
             ns_lvl = seg_mean[dom] * 1e6 / dseg["nlevels"]
             dep = {"nlevels": dseg["nlevels"], "ns_per_level": ns_lvl}
@@ -408,7 +418,9 @@ def main():
     e2e = {"value": flops_job / e2e_t / 1e9, "unit": "GFLOPS", "h2d_bytes_per_step": h2d,
            "d2h_bytes_per_step": d2h, "ms_per_step": e2e_t * 1e3,
            "path": "dist_solve (NCCL scatter/gather) from pinned host B on rank 0" if sharded
-           else "sptrsv_solve with pinned host b/x (H2D + solve + D2H inside the call)"}
+           else ("sptrsv_solve with pinned host b/x (column blocks: H2D / solve / D2H overlapped on three "
+                 "streams inside the call)" if nrhs >= 32 else
+                 "sptrsv_solve with pinned host b/x (H2D + solve + D2H inside the call)")}
 
     # ---------------- parity of the timed result (sampled for multi-RHS)
     parity = None

@@ -13,10 +13,12 @@
 //                       execution order, diagonal separate, CSR or DCSR
 //   features + Alg 7    Sec 3.4 (L252-L296)
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cstdlib>
 #include <cstring>
 #include <functional>
+#include <memory>
 #include <mutex>
 #include <numeric>
 #include <thread>
@@ -208,12 +210,64 @@ struct Reorderer {
   // dependencies inside the triangle count, reading R5), then a stable
   // counting sort of its rows by level (ties keep the current order, R4).
   // Writes the (sorted) levels into leaf_level[lo,hi); returns nlevels.
-  int32_t node_reorder(int32_t lo, int32_t hi, bool identity = false) {
+  // Levels of rows [lo, hi) by threads working on consecutive row chunks
+  // in claim order: a dependency in an earlier chunk that is still being
+  // swept is waited for (its level slot holds -1 until written), and the
+  // lowest unfinished chunk never waits, so the sweep cannot deadlock.  The
+  // levels are the serial sweep's exactly (each is 1 + the max over its
+  // dependencies, however the work is split).
+  int32_t levels_parallel(int32_t lo, int32_t hi, bool identity, int threads, std::vector<int32_t>& lev) {
+    const int32_t m = hi - lo;
+    constexpr int32_t CH = 2048;
+    const int32_t nch = (m + CH - 1) / CH;
+    std::unique_ptr<std::atomic<int32_t>[]> al(new std::atomic<int32_t>[(size_t)m]);
+    par_for(m, threads, [&](int64_t a, int64_t b) {
+      for (int64_t k = a; k < b; ++k) al[k].store(-1, std::memory_order_relaxed);
+    });
+    std::atomic<int32_t> next{0};
+    std::vector<int32_t> tmax((size_t)threads, 0);
+    std::vector<std::thread> th;
+    for (int t = 0; t < threads; ++t)
+      th.emplace_back([&, t] {
+        int32_t mx = 0;
+        for (int32_t ch; (ch = next.fetch_add(1, std::memory_order_relaxed)) < nch;) {
+          const int32_t r1 = lo + std::min(m, (ch + 1) * CH);
+          for (int32_t r = lo + ch * CH; r < r1; ++r) {
+            const int32_t o = identity ? r : perm[r];
+            int32_t lv = 0;
+            for (int64_t q = L.rp[o], e = L.rp[o + 1] - 1; q < e; ++q) {
+              const int32_t c = identity ? L.ci[q] : old2new[L.ci[q]];
+              if (c < lo) continue;
+              int32_t v = al[c - lo].load(std::memory_order_acquire);
+              while (v < 0) {
+#if defined(__x86_64__) || defined(__i386__)
+                __builtin_ia32_pause();
+#endif
+                v = al[c - lo].load(std::memory_order_acquire);
+              }
+              lv = std::max(lv, v + 1);
+            }
+            al[r - lo].store(lv, std::memory_order_release);
+            mx = std::max(mx, lv + 1);
+          }
+        }
+        tmax[t] = mx;
+      });
+    for (auto& x : th) x.join();
+    par_for(m, threads, [&](int64_t a, int64_t b) {
+      for (int64_t k = a; k < b; ++k) lev[k] = al[k].load(std::memory_order_relaxed);
+    });
+    return *std::max_element(tmax.begin(), tmax.end());
+  }
+
+  int32_t node_reorder(int32_t lo, int32_t hi, bool identity = false, int inner = 1) {
     int32_t m = hi - lo;
     if (m == 0) return 0;
     std::vector<int32_t> lev((size_t)m);
     int32_t nl = 0;
-    if (identity) {  // perm is still the identity (the root): no old2new lookups
+    if (inner > 1 && m >= 65536) {
+      nl = levels_parallel(lo, hi, identity, inner, lev);
+    } else if (identity) {  // perm is still the identity (the root): no old2new lookups
       for (int32_t r = lo; r < hi; ++r) {
         int32_t lv = 0;
         for (int64_t q = L.rp[r], e = L.rp[r + 1] - 1; q < e; ++q) {
@@ -327,8 +381,9 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
         work.push_back(k);
       }
     }
-    if (work.size() == 1 || threads == 1) {
-      for (size_t k : work) nl[k] = R.node_reorder(nodes[k].first, nodes[k].second, d == 0);
+    if (work.size() * 4 <= (size_t)threads || threads == 1) {
+      // few nodes: one after the other, each swept by all threads
+      for (size_t k : work) nl[k] = R.node_reorder(nodes[k].first, nodes[k].second, d == 0, threads);
     } else {
       std::vector<std::thread> th;
       int T = std::min<int>(threads, (int)work.size());

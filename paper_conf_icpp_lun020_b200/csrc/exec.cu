@@ -78,7 +78,13 @@ void dispatch_multi_un(int nrhs, const SpmmCfg& c, F&& f) {
 inline unsigned cdiv(int64_t a, int64_t b) { return (unsigned)((a + b - 1) / b); }
 
 // long rows -> a warp per component (L247 "a thread or a 32-thread warp")
-inline bool tri_use_warp(const Segment& S) { return S.info.nnz_per_row > 8; }
+inline bool tri_use_warp(const Segment& S) {
+  static const int thr = [] {
+    const char* e = std::getenv("SPTRSV_SF_WARP_NPR");  // tuning: nnz/row above which a warp owns a row
+    return e ? std::atoi(e) : 8;
+  }();
+  return S.info.nnz_per_row > thr;
+}
 
 // Shared-memory geometry of the TMA-staged chain kernel (227 KB per CTA).
 // Overridable for tuning with SPTRSV_CHAIN_GEOM="NST,RMAX,EMAX,XW,LMAX".
@@ -1388,6 +1394,82 @@ Error upload(Plan& p, void* stream_v) {
   return {SPTRSV_SUCCESS, ""};
 }
 
+// End-to-end solve from HOST buffers with many column-major right-hand
+// sides: the columns are cut into blocks of cb; block k's host->device copy
+// (stream h2d), its solve (the caller's stream) and its device->host copy
+// (stream d2h) overlap the neighbouring blocks', over two staging buffers
+// per direction.  PCIe runs both directions at once, so the call costs about
+// one direction's transfer instead of transfer-in + solve + transfer-out.
+Error solve_host_pipelined(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t nrhs,
+                           cudaStream_t s) {
+  const size_t vb = p.vbytes;
+  const int nblk = std::min(8, std::max(2, nrhs / 16));
+  const int cb = (nrhs + nblk - 1) / nblk;
+  const size_t blk_bytes = (size_t)p.n * cb * vb;
+  if (2 * blk_bytes > p.ws.stage_bytes) {
+    if (p.ws.stage_b) cudaFree(p.ws.stage_b);
+    if (p.ws.stage_x) cudaFree(p.ws.stage_x);
+    p.ws.stage_b = p.ws.stage_x = nullptr;
+    p.ws.stage_bytes = 0;
+    if (cudaMalloc(&p.ws.stage_b, 2 * blk_bytes) != cudaSuccess ||
+        cudaMalloc(&p.ws.stage_x, 2 * blk_bytes) != cudaSuccess) {
+      cudaGetLastError();
+      return {SPTRSV_ERROR_ALLOC, "staging allocation failed"};
+    }
+    p.ws.stage_bytes = 2 * blk_bytes;
+  }
+  if (!p.ws.h2d) {
+    cudaStream_t a, c;
+    CUDA_TRY(cudaStreamCreateWithFlags(&a, cudaStreamNonBlocking));
+    CUDA_TRY(cudaStreamCreateWithFlags(&c, cudaStreamNonBlocking));
+    p.ws.h2d = (void*)a;
+    p.ws.d2h = (void*)c;
+    for (auto& e : p.ws.ev) {
+      cudaEvent_t ev;
+      CUDA_TRY(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+      e = (void*)ev;
+    }
+  }
+  cudaStream_t h2d = (cudaStream_t)p.ws.h2d, d2h = (cudaStream_t)p.ws.d2h;
+  cudaEvent_t* ev = (cudaEvent_t*)p.ws.ev;  // in[0..1], comp[2..3], out[4..5]
+  // the copy streams start after whatever the caller queued on s
+  CUDA_TRY(cudaEventRecord(ev[2], s));
+  CUDA_TRY(cudaEventRecord(ev[3], s));
+  CUDA_TRY(cudaEventRecord(ev[4], s));
+  CUDA_TRY(cudaEventRecord(ev[5], s));
+  const size_t width = (size_t)p.n * vb;
+  for (int k = 0; k * cb < nrhs; ++k) {
+    const int c0 = k * cb, nc = std::min(cb, nrhs - c0), u = k & 1;
+    char* sb = (char*)p.ws.stage_b + u * blk_bytes;
+    char* sx = (char*)p.ws.stage_x + u * blk_bytes;
+    // in: stage_b[u] is free once the solve of block k-2 finished
+    CUDA_TRY(cudaStreamWaitEvent(h2d, ev[2 + u], 0));
+    CUDA_TRY(cudaMemcpy2DAsync(sb, width, (const char*)b + (size_t)c0 * ldb * vb, (size_t)ldb * vb, width, nc,
+                               cudaMemcpyHostToDevice, h2d));
+    CUDA_TRY(cudaEventRecord(ev[u], h2d));
+    // solve: needs block k in, and stage_x[u] drained by block k-2's copy out
+    CUDA_TRY(cudaStreamWaitEvent(s, ev[u], 0));
+    CUDA_TRY(cudaStreamWaitEvent(s, ev[4 + u], 0));
+    Error e = p.dtype == SPTRSV_R64F
+                  ? solve_device<double>(p, (const double*)sb, p.n, (double*)sx, p.n, nc, SPTRSV_COL_MAJOR, s)
+                  : solve_device<float>(p, (const float*)sb, p.n, (float*)sx, p.n, nc, SPTRSV_COL_MAJOR, s);
+    if (e.status) return e;
+    CUDA_TRY(cudaEventRecord(ev[2 + u], s));
+    // out
+    CUDA_TRY(cudaStreamWaitEvent(d2h, ev[2 + u], 0));
+    CUDA_TRY(cudaMemcpy2DAsync((char*)x + (size_t)c0 * ldx * vb, (size_t)ldx * vb, sx, width, width, nc,
+                               cudaMemcpyDeviceToHost, d2h));
+    CUDA_TRY(cudaEventRecord(ev[4 + u], d2h));
+  }
+  CUDA_TRY(cudaStreamSynchronize(d2h));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  if (p.h_error && *(volatile int32_t*)p.h_error) {
+    *(volatile int32_t*)p.h_error = 0;
+    return {SPTRSV_ERROR_DEADLOCK, "spin-wait watchdog tripped"};
+  }
+  return {SPTRSV_SUCCESS, ""};
+}
+
 Error solve(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t nrhs, sptrsv_layout_t layout,
             void* stream_v) {
   cudaStream_t s = (cudaStream_t)stream_v;
@@ -1408,6 +1490,9 @@ Error solve(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t n
       return solve_device<double>(p, (const double*)b, ldb, (double*)x, ldx, nrhs, layout, s);
     return solve_device<float>(p, (const float*)b, ldb, (float*)x, ldx, nrhs, layout, s);
   }
+  // host buffers, many column-major RHS: pipelined by column blocks
+  if (layout == SPTRSV_COL_MAJOR && nrhs >= 32 && std::getenv("SPTRSV_NO_PIPELINE") == nullptr)
+    return solve_host_pipelined(p, b, ldb, x, ldx, nrhs, s);
   // host buffers: stage through the device (end-to-end path), then sync
   size_t need = (size_t)p.n * nrhs * vb;
   if (need > p.ws.stage_bytes) {
@@ -1455,6 +1540,10 @@ void release(Plan& p) {
   if (p.ws.stage_b) cudaFree(p.ws.stage_b);
   if (p.ws.stage_x) cudaFree(p.ws.stage_x);
   if (p.ws.flags) cudaFree(p.ws.flags);
+  if (p.ws.h2d) cudaStreamDestroy((cudaStream_t)p.ws.h2d);
+  if (p.ws.d2h) cudaStreamDestroy((cudaStream_t)p.ws.d2h);
+  for (void* e : p.ws.ev)
+    if (e) cudaEventDestroy((cudaEvent_t)e);
   if (p.h_error) cudaFreeHost(p.h_error);
   for (auto& S : p.segs)
     if (S.d_trace) cudaFree(S.d_trace);

@@ -151,6 +151,10 @@ struct Workspace {
   void* stage_x = nullptr;
   size_t stage_bytes = 0;
   void* flags = nullptr;    // nrhs > 1 sync-free: per-row ready flags (n x u32), epoch-valued
+  // pipelined host path (exec.cu solve_host_pipelined): copy streams + events
+  void* h2d = nullptr;      // cudaStream_t
+  void* d2h = nullptr;
+  void* ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};  // in[2], comp[2], out[2]
 };
 
 // SpMM lane geometry for nrhs > 1 (exec.cu: dispatch_multi_un)

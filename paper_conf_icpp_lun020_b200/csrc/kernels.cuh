@@ -282,7 +282,10 @@ __global__ void sq_vector_1(int nzr, int r0, const int* __restrict__ rows, const
 // paper's scalar / vector kernels leave lanes idle on short rows and
 // serialise long ones, L249-L250).  A row cut into several chunks adds its
 // partial sums with atomics (summation order then varies, reading R22).
-constexpr int kSqNB = 256, kSqLW = 1024;
+#ifndef SPTRSV_SQ_NB
+#define SPTRSV_SQ_NB 256  // entries per row block (tuning builds may change it)
+#endif
+constexpr int kSqNB = SPTRSV_SQ_NB, kSqLW = 1024;
 struct SqItem {
   int t0, t1;  // stored rows [t0, t1); bit 31 of t1: chunk of a split row (atomic update)
   int p0, p1;  // entries [p0, p1)
@@ -754,8 +757,11 @@ struct SnDesc {
   long long voff, boff;        // offsets (elements) of V_J and of the packed T_J
 };
 
+#ifndef SPTRSV_SN_MINB
+#define SPTRSV_SN_MINB 1  // min resident CTAs per SM requested from ptxas (tuning builds)
+#endif
 template <typename T>
-__global__ void __launch_bounds__(256) tri_supernode(int npieces, const SnDesc* __restrict__ desc,
+__global__ void __launch_bounds__(256, SPTRSV_SN_MINB) tri_supernode(int npieces, const SnDesc* __restrict__ desc,
                                                      const int* __restrict__ cols, const T* __restrict__ V,
                                                      const T* __restrict__ Tb, const T* __restrict__ bw,
                                                      T* __restrict__ xs, SolveState st, int slot) {

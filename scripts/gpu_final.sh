@@ -26,6 +26,17 @@ for c in ${NCU_CONFIGS:-C2 C3 C4 C5}; do
     C2) K=tri_wave; S=2;; C3) K=tri_syncfree; S=0;; C4) K=tri_supernode; S=0;; C5) K=sq_multi; S=1;;
   esac
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:$K -s $S -c 1 -o $O/prof_$c -f python scripts/prof_solve.py --config $c --reps 2 $nr > $O/ncu_$c.log 2>&1; echo "ncu full $c rc=$?"
+  # summarise on the box (gpurun brings back <= 64 MiB): launch list, full-set
+  # summary, DRAM bytes per launch; the .ncu-rep stays only if small
+  IMPL=$c:$(python - "$c" <<'PY'
+import sys
+print({"C2": "TRI_PIPE", "C3": "TRI_SYNCFREE", "C4": "TRI_SUPERNODE", "C5": "SQ_SPMM"}[sys.argv[1]])
+PY
+)
+  python scripts/ncu_summary.py --launches $O/launches_$c.csv --rep $O/prof_$c.ncu-rep --out $O/${TAG:-r01}_${c}_final --impl $IMPL --json $O/ncu_summary_part.json > /dev/null 2>&1; echo "summary $c rc=$?"
+  ncu -i $O/prof_$c.ncu-rep --page source --csv --print-source sass > $O/src_$c.csv 2>/dev/null
+  python scripts/sass_hot.py $O/src_$c.csv > $O/${TAG:-r01}_${c}_final_sass_hot.md 2>/dev/null; rm -f $O/src_$c.csv
+  [ $(stat -c %s $O/prof_$c.ncu-rep 2>/dev/null || echo 0) -gt 12000000 ] && rm -f $O/prof_$c.ncu-rep
 done
 fi
 ls $O

@@ -117,6 +117,8 @@ def main():
     ap.add_argument("--out", required=True)
     ap.add_argument("--impl", default=None, help="bench impl name the captured kernel implements")
     ap.add_argument("--title", default="")
+    ap.add_argument("--json", default=os.path.join(ROOT, "profiles", "ncu_summary.json"),
+                    help="summary json the captured kernel's DRAM bytes are merged into")
     a = ap.parse_args()
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     if a.launches:
@@ -132,7 +134,7 @@ def main():
                     f"(`--set full --clock-control none --import-source on`).\n\n")
             f.write(txt + "\n")
         if a.impl and recs:
-            p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+            p = a.json
             d = json.load(open(p)) if os.path.exists(p) else {}
             d.setdefault("dram_bytes_per_launch", {})[a.impl] = recs[0]["dram_bytes"]
             d.setdefault("source", {})[a.impl] = os.path.basename(a.out) + "_ncu.md"

@@ -166,6 +166,29 @@ def test_host_pointers(gpu):
     _check64(M, b, Xp.T.numpy())
 
 
+@pytest.mark.parametrize("nrhs", [32, 37, 133])
+@pytest.mark.parametrize("pinned", [True, False])
+def test_host_pointers_pipelined(gpu, nrhs, pinned):
+    """Host buffers with >= 32 column-major RHS go through the column-block
+    pipeline (copy in / solve / copy out overlapped on three streams), with
+    ragged last blocks and ld > n."""
+    M, b = g.gen_config("C5", small=True, nrhs=nrhs)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, depth=2)
+    n = M.n
+    big = torch.zeros((nrhs, n + 5), dtype=torch.float64)
+    big[:, :n] = torch.from_numpy(b)
+    if pinned:
+        big = big.pin_memory()
+    B = big[:, :n].T  # (n, nrhs) column-major, ld = n + 5
+    X = torch.full((nrhs, n + 3), float("nan"), dtype=torch.float64)
+    if pinned:
+        X = X.pin_memory()
+    Xv = X[:, :n].T
+    sp.sptrsv_solve(plan, B, Xv)
+    _check64(M, b, X[:, :n].numpy())
+    assert torch.isnan(X[:, n:]).all()  # the ld padding is untouched
+
+
 @pytest.mark.parametrize("shape", ["diag", "chain", "dense", "arrow", "n1", "fig1"])
 def test_adversarial(gpu, shape):
     M = {"diag": lambda: g.shape_diagonal(10000), "chain": lambda: g.shape_bidiagonal(100_000),

@@ -15,6 +15,8 @@ Nothing here solves, levels, reorders or blocks anything.
 from __future__ import annotations
 
 import dataclasses
+import os
+
 import numpy as np
 
 SEED_BASE = 20200817
@@ -301,11 +303,28 @@ SMALL = {
 }
 
 
+def _build_cached(name: str, small: bool, build) -> Matrix:
+    """build(), or its copy under $SPTRSV_GEN_CACHE (opt-in, for tuning
+    scripts that regenerate the same full-size matrix many times)."""
+    d = os.environ.get("SPTRSV_GEN_CACHE")
+    if not d:
+        return build()
+    path = os.path.join(d, f"{name}{'_small' if small else ''}.npz")
+    if os.path.exists(path):
+        z = np.load(path)
+        return Matrix(n=int(z["n"]), row_ptr=z["row_ptr"], col_idx=z["col_idx"], val=z["val"], name=str(z["name"]))
+    L = build()
+    os.makedirs(d, exist_ok=True)
+    np.savez(path + ".tmp.npz", n=L.n, row_ptr=L.row_ptr, col_idx=L.col_idx, val=L.val, name=L.name)
+    os.replace(path + ".tmp.npz", path)
+    return L
+
+
 def gen_config(name: str, small: bool = False, nrhs: int | None = None, dtype=np.float64):
     """Return (Matrix, b) for a config; b has numpy shape (nrhs, n)."""
     k = int(name[1:])
     build, default_nrhs = (SMALL if small else CONFIGS)[name]
-    L = build()
+    L = _build_cached(name, small, build)
     if dtype != np.float64:
         L = L.astype(dtype)
     nr = default_nrhs if nrhs is None else nrhs
