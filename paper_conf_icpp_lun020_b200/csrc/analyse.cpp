@@ -381,8 +381,10 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
         work.push_back(k);
       }
     }
-    if (work.size() * 4 <= (size_t)threads || threads == 1) {
-      // few nodes: one after the other, each swept by all threads
+    if (work.size() == 1 || threads == 1) {
+      // a lone node (the root, the first bottom child): swept by all threads
+      // (measured: on C3's layered DAG two or more bottom nodes go faster
+      // one thread each than one after the other swept in parallel)
       for (size_t k : work) nl[k] = R.node_reorder(nodes[k].first, nodes[k].second, d == 0, threads);
     } else {
       std::vector<std::thread> th;

@@ -131,6 +131,9 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_analyse(int32_t n, int64_t nnz, const int32
   } else {
     p.sm_count = o.sm_count > 0 ? o.sm_count : 148;
   }
+  if (std::getenv("SPTRSV_ANALYSE_TRACE"))
+    std::fprintf(stderr, "[sptrsv analyse] %-28s %9.2f ms\n", "capi: device + input checks",
+                 std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
   Error e = analyse_host(p, n, nnz, (const int32_t*)rp_h, (const int32_t*)ci_h, val_h);
   if (e.status) {
     delete P;

@@ -587,23 +587,27 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
       const auto& Gs = groups[s2];
       const auto& R = srows[s2];
       const int nch = (int)((Gs.size() + GPC - 1) / GPC);
-      clist[s2].resize(nch);
-      for (int c = 0; c < nch; ++c) {
-        for (int g2 = c * GPC; g2 < std::min<int>((int)Gs.size(), (c + 1) * GPC); ++g2)
-          for (int l = 0; l < Gs[g2].second; ++l) {
-            const int r = R[Gs[g2].first + l];
-            for (int e = S.rp[r]; e < S.rp[r + 1]; ++e)
-              if (dep[e].kind == 1 && !seen[dep[e].b]) {
-                seen[dep[e].b] = 1;
-                clist[s2][c].push_back((uint32_t)(imp_base[s2] + dep[e].b) * VB0);
-              }
-          }
-        max_ci = std::max<int>(max_ci, (int)clist[s2][c].size());
-      }
+      // one list per quarter (k::kWaveQ parts) of the chunk's groups
+      clist[s2].resize((size_t)nch * k::kWaveQ);
+      for (int c = 0; c < nch; ++c)
+        for (int q = 0; q < k::kWaveQ; ++q) {
+          auto& L = clist[s2][(size_t)c * k::kWaveQ + q];
+          const int ga = c * GPC + q * GPC / k::kWaveQ, gb = c * GPC + (q + 1) * GPC / k::kWaveQ;
+          for (int g2 = ga; g2 < std::min<int>((int)Gs.size(), gb); ++g2)
+            for (int l = 0; l < Gs[g2].second; ++l) {
+              const int r = R[Gs[g2].first + l];
+              for (int e = S.rp[r]; e < S.rp[r + 1]; ++e)
+                if (dep[e].kind == 1 && !seen[dep[e].b]) {
+                  seen[dep[e].b] = 1;
+                  L.push_back((uint32_t)(imp_base[s2] + dep[e].b) * VB0);
+                }
+            }
+          max_ci = std::max<int>(max_ci, (int)L.size());
+        }
     }
   }
   const int ipl = (max_ci + 31) / 32;
-  const uint32_t cbytes = hbytes + (uint32_t)GPC * gbytes + (uint32_t)ipl * 128u;
+  const uint32_t cbytes = hbytes + (uint32_t)GPC * gbytes + (uint32_t)(ipl * k::kWaveQ) * 128u;
   {  // the import lists must still fit next to the x area (else: the chain kernel)
     const int64_t need = (int64_t)k::al16((uint32_t)xa * (uint32_t)vb) + (int64_t)W * NCH * (cbytes + bring + 16);
     if (need > 232448) return give_up();
@@ -680,8 +684,11 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
         }
         gh[1] = Gs[g].second | flags;
       }
-      uint32_t* il = (uint32_t*)(B + hbytes + (size_t)GPC * gbytes);
-      for (size_t i = 0; i < clist[s2][c].size(); ++i) il[i] = clist[s2][c][i];  // rest: 0 = the zero slot
+      for (int q = 0; q < k::kWaveQ; ++q) {  // rest of each list: 0 = the zero slot
+        uint32_t* il = (uint32_t*)(B + hbytes + (size_t)GPC * gbytes + (size_t)q * ipl * 128);
+        const auto& L = clist[s2][(size_t)c * k::kWaveQ + q];
+        for (size_t i = 0; i < L.size(); ++i) il[i] = L[i];
+      }
     }
     off += (size_t)nchunk[s2] * cbytes;
   }
@@ -1164,6 +1171,40 @@ struct PinnedStager {
   }
 };
 
+// Pool of mapped pinned host words for the plans' spin-wait watchdogs: one
+// 4 KB page per 1024 plans, allocated on demand, never returned to the driver.
+namespace {
+std::mutex wd_mu;
+std::vector<std::pair<int32_t*, int32_t*>> wd_free;  // (host, device) of free words
+}  // namespace
+bool watchdog_word_acquire(int32_t** h, int32_t** d) {
+  std::lock_guard<std::mutex> g(wd_mu);
+  if (wd_free.empty()) {
+    int32_t* page = nullptr;
+    int32_t* dpage = nullptr;
+    if (cudaHostAlloc((void**)&page, 4096, cudaHostAllocMapped) != cudaSuccess ||
+        cudaHostGetDevicePointer((void**)&dpage, page, 0) != cudaSuccess) {
+      cudaGetLastError();
+      return false;
+    }
+    for (int i = 1023; i >= 0; --i) wd_free.push_back({page + i, dpage + i});
+  }
+  *h = wd_free.back().first;
+  *d = wd_free.back().second;
+  wd_free.pop_back();
+  return true;
+}
+void watchdog_word_release(int32_t* h) {
+  std::lock_guard<std::mutex> g(wd_mu);
+  // the device alias of a mapped host word is fixed: recover it
+  int32_t* d = nullptr;
+  if (cudaHostGetDevicePointer((void**)&d, h, 0) != cudaSuccess) {
+    cudaGetLastError();
+    return;
+  }
+  wd_free.push_back({h, d});
+}
+
 Error upload(Plan& p, void* stream_v) {
   cudaStream_t s = (cudaStream_t)stream_v;
   const size_t vb = p.vbytes;
@@ -1379,14 +1420,13 @@ Error upload(Plan& p, void* stream_v) {
   p.d_rdiag = (const void*)(A + o_rdiag);
   p.d_tickets = (uint32_t*)(A + o_tickets);
   clk.lap("upload: H2D copies issued");
-  // mapped host word for the spin-wait watchdog
-  if (cudaHostAlloc((void**)&p.h_error, sizeof(int32_t), cudaHostAllocMapped) == cudaSuccess) {
-    *p.h_error = 0;
-    CUDA_TRY(cudaHostGetDevicePointer((void**)&p.d_error, p.h_error, 0));
-  } else {
-    cudaGetLastError();
+  // mapped host word for the spin-wait watchdog, from a process-wide pool
+  // (cudaHostAlloc costs milliseconds per call)
+  if (!watchdog_word_acquire(&p.h_error, &p.d_error)) {
     p.h_error = nullptr;
     p.d_error = nullptr;
+  } else {
+    *p.h_error = 0;
   }
   CUDA_TRY(cudaStreamSynchronize(s));
   clk.lap("upload: H2D complete");
@@ -1544,7 +1584,7 @@ void release(Plan& p) {
   if (p.ws.d2h) cudaStreamDestroy((cudaStream_t)p.ws.d2h);
   for (void* e : p.ws.ev)
     if (e) cudaEventDestroy((cudaEvent_t)e);
-  if (p.h_error) cudaFreeHost(p.h_error);
+  if (p.h_error) watchdog_word_release(p.h_error);
   for (auto& S : p.segs)
     if (S.d_trace) cudaFree(S.d_trace);
   for (void* e : p.events) cudaEventDestroy((cudaEvent_t)e);
@@ -1573,11 +1613,10 @@ Error seg_times(Plan& p, float* ms, int32_t cap, int32_t* count) {
 Error device_info(int* sm_count, int* major, int* minor) {
   int dev;
   CUDA_TRY(cudaGetDevice(&dev));
-  cudaDeviceProp pr;
-  CUDA_TRY(cudaGetDeviceProperties(&pr, dev));
-  *sm_count = pr.multiProcessorCount;
-  *major = pr.major;
-  *minor = pr.minor;
+  // attribute queries (cudaGetDeviceProperties costs milliseconds per call)
+  CUDA_TRY(cudaDeviceGetAttribute(sm_count, cudaDevAttrMultiProcessorCount, dev));
+  CUDA_TRY(cudaDeviceGetAttribute(major, cudaDevAttrComputeCapabilityMajor, dev));
+  CUDA_TRY(cudaDeviceGetAttribute(minor, cudaDevAttrComputeCapabilityMinor, dev));
   return {SPTRSV_SUCCESS, ""};
 }
 

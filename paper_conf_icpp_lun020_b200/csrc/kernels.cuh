@@ -758,7 +758,7 @@ struct SnDesc {
 };
 
 #ifndef SPTRSV_SN_MINB
-#define SPTRSV_SN_MINB 1  // min resident CTAs per SM requested from ptxas (tuning builds)
+#define SPTRSV_SN_MINB 2  // min resident CTAs per SM requested from ptxas (C4: 2 measured best of 1-3)
 #endif
 template <typename T>
 __global__ void __launch_bounds__(256, SPTRSV_SN_MINB) tri_supernode(int npieces, const SnDesc* __restrict__ desc,
@@ -1535,6 +1535,10 @@ constexpr unsigned kWaveWaitNs = SPTRSV_WAVE_WAIT_NS;
 #define SPTRSV_WAVE_GPC_BIG 12
 #endif
 constexpr int kWaveGpcBig = SPTRSV_WAVE_GPC_BIG;  // groups per chunk (multiple of 3); 6 when smem is short
+#ifndef SPTRSV_WAVE_Q
+#define SPTRSV_WAVE_Q 1  // measured on C2: 1 0.2586 ms, 2 0.2597, 3 0.2668
+#endif
+constexpr int kWaveQ = SPTRSV_WAVE_Q;  // import checks per chunk (divides 6)
 template <typename T, int K, int E, int GPC, bool GLB>
 __global__ void __launch_bounds__(288, 1)
     tri_wave(const WaveStrand* __restrict__ strands, const char* __restrict__ data, const T* __restrict__ bw, T* __restrict__ xs, WaveGeom g, SolveState st, long long* __restrict__ trace) {
@@ -1695,8 +1699,9 @@ __global__ void __launch_bounds__(288, 1)
   const uint32_t imp_lo = Sp->imp_lo, imp_hi = Sp->imp_hi;
   // The chunk block ends with the byte offsets of the imports the chunk
   // uses first (padding: the zero slot), imp_per_lane words per lane.
-  auto chunk_wait = [&](const unsigned char* Bc) {
-    const uint32_t* il = (const uint32_t*)(Bc + g.hdr_bytes + (uint32_t)GPC * g.group_bytes);
+  auto chunk_wait = [&](const unsigned char* Bc, int q) {
+    const uint32_t* il = (const uint32_t*)(Bc + g.hdr_bytes + (uint32_t)GPC * g.group_bytes +
+                                           (uint32_t)(q * g.imp_per_lane) * 128u);
     uint32_t xo0 = 0;
     if (!GLB && g.imp_per_lane > 0) xo0 = il[lane];
     for (; !GLB && imp_lo != imp_hi;) {
@@ -1717,7 +1722,7 @@ __global__ void __launch_bounds__(288, 1)
     mbar_wait(&full[0], 0);
     load_op(B, bb, 0, op0);
     load_op(B, bb, 1, op1);
-    chunk_wait(B);
+    chunk_wait(B, 0);
   }
   for (int c = 0; c < s_nchunk; ++c) {
     const bool more = c + 1 < s_nchunk;
@@ -1726,6 +1731,10 @@ __global__ void __launch_bounds__(288, 1)
       WaveOp<T, K, E>& cur = gi % 3 == 0 ? op0 : gi % 3 == 1 ? op1 : op2;
       WaveOp<T, K, E>& n1 = gi % 3 == 0 ? op1 : gi % 3 == 1 ? op2 : op0;
       WaveOp<T, K, E>& n2 = gi % 3 == 0 ? op2 : gi % 3 == 1 ? op0 : op1;
+      // imports of the next part of the chunk (the first part was checked
+      // when the chunk was opened): GPC / kWaveQ levels of lag per strand
+      // boundary instead of GPC, one vote per part
+      if (gi > 0 && gi % (GPC / kWaveQ) == 0) chunk_wait(B, gi / (GPC / kWaveQ));
 #ifdef SPTRSV_WAVE_TRACE
       if (tr && lane == 0 && c * GPC + gi < 1016) {
         long long gt;
@@ -1755,7 +1764,7 @@ __global__ void __launch_bounds__(288, 1)
         ph = ph_n;
         B = Bn;
         bb = bbn;
-        if (more) chunk_wait(B);
+        if (more) chunk_wait(B, 0);
       }
       if (!(SPTRSV_WAVE_EXP & 16)) warp_sync_all();
     }
