@@ -99,7 +99,10 @@ typedef enum { SPTRSV_SELECT_PAPER = 0, SPTRSV_SELECT_B200 = 1 } sptrsv_selector
 
 typedef struct {
   int32_t variant;          /* sptrsv_variant_t, default REC                                   */
-  int32_t depth;            /* -1 = the paper's rule (L299); >= 0 forces a uniform depth       */
+  int32_t depth;            /* -1 = the paper's rule (L299) -- under selector B200 with
+                               min_block_rows 0, a root whose levels are all <= 2048 rows with
+                               1..8 dependencies per row stays one triangle (R30);
+                               >= 0 forces a uniform depth                                     */
   int64_t min_block_rows;   /* depth-rule threshold; 0 = 20 * SMs * 128 (378,880 on 148 SMs)   */
   int32_t reorder;          /* 0 = level-set reordering of every triangle (L231), 1 = none,
                                2 = auto (default): none when the input is supernodal (mean width of
@@ -172,6 +175,9 @@ typedef struct {
   int32_t launches_per_solve; /* kernel launches of one nrhs=1 solve (graph nodes)          */
   double analyse_ms;          /* host wall time of sptrsv_analyse, upload included          */
   int64_t device_bytes;       /* device memory owned by the plan (arena, excl. workspace)  */
+  int32_t depth_rule;         /* 0 = the paper's rule (L299), 1 = B200 retune (a root with
+                                 only narrow levels stays whole: DESIGN.md R30), 2 = caller's */
+  int32_t reserved_info;
 } sptrsv_plan_info_t;
 
 typedef struct {

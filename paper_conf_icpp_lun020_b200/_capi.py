@@ -45,7 +45,8 @@ class PlanInfo(ctypes.Structure):
                 ("reorder", ctypes.c_int32), ("selector", ctypes.c_int32), ("nnz", ctypes.c_int64),
                 ("min_block_rows", ctypes.c_int64), ("sm_count", ctypes.c_int32),
                 ("launches_per_solve", ctypes.c_int32), ("analyse_ms", ctypes.c_double),
-                ("device_bytes", ctypes.c_int64)]
+                ("device_bytes", ctypes.c_int64), ("depth_rule", ctypes.c_int32),
+                ("reserved_info", ctypes.c_int32)]
 
 
 class SegInfo(ctypes.Structure):

@@ -396,6 +396,30 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
       for (auto& x : th) x.join();
     }
     if (clk.on) clk.lap(("  reorder depth " + std::to_string(d)).c_str());
+    // Depth retune under the B200 selector (reading R30): a
+    // root triangle whose levels are all narrow (<= 2048 rows) and whose rows
+    // have 1..8 dependencies is solved whole by the strand wavefront, which
+    // pipelines the level chain across the cluster; the paper's split
+    // (L299) would only add a square and drain and refill the wavefront at
+    // the kernel boundary (C2: 0.260 -> 0.215 ms).  Only when the caller left
+    // both depth and min_block_rows to the library and level reordering is on.
+    if (d == 0 && p.depth > 0 && p.opts.depth < 0 && p.opts.min_block_rows == 0 &&
+        p.opts.selector == SPTRSV_SELECT_B200 && p.reorder_eff == 0 && n >= 4096 &&
+        std::getenv("SPTRSV_NO_DEPTH_RETUNE") == nullptr) {
+      std::vector<int32_t> wid((size_t)nl[0] + 1, 0);
+      int32_t wmax = 0;
+      for (int32_t r = 0; r < n; ++r) wmax = std::max(wmax, ++wid[R.leaf_level[r]]);
+      int64_t kmin = INT64_MAX, kmax = 0;
+      for (int32_t r = 0; r < n; ++r) {
+        const int64_t k = L.rp[r + 1] - L.rp[r] - 1;
+        kmin = std::min(kmin, k);
+        kmax = std::max(kmax, k);
+      }
+      if (wmax <= 2048 && kmax >= 1 && kmax <= 8) {
+        p.depth = 0;
+        p.depth_retuned = 1;
+      }
+    }
     if (d == p.depth) {
       leaf_nl = nl;
       break;

@@ -195,6 +195,8 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_info(sptrsv_plan_t plan, sptrsv_plan_i
   out->sm_count = p.sm_count;
   out->launches_per_solve = p.launches_per_solve;
   out->analyse_ms = p.analyse_ms;
+  out->depth_rule = p.opts.depth >= 0 ? 2 : p.depth_retuned;
+  out->reserved_info = 0;
   out->device_bytes = (int64_t)p.arena_bytes;
   return SPTRSV_SUCCESS;
 }

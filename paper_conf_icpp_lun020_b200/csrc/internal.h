@@ -173,6 +173,7 @@ struct Plan {
   int64_t min_block_rows = 0;
   double analyse_ms = 0.0;
   int32_t reorder_eff = 0;  // reorder actually applied (0 level, 1 none)
+  int32_t depth_retuned = 0;  // 1: the B200 selector overrode the paper's depth rule (R30)
   size_t vbytes = 8;
 
   std::vector<Segment> segs;

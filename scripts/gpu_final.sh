@@ -1,8 +1,8 @@
 #!/bin/bash
 # Round-end measurement: smoke, GPU suite, bench of every config (with the
 # oracle baseline), ncu launch lists and one full capture per config.
-mkdir -p gpurun_out/final
 O=gpurun_out/${OUTDIR:-final}
+mkdir -p $O
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,driver_version --format=csv > $O/gpu.txt 2>&1
 nproc > $O/nproc.txt
 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?"; tail -1 $O/smoke.log

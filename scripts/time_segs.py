@@ -12,9 +12,10 @@ ap.add_argument("--config", default="C2")
 ap.add_argument("--reps", type=int, default=20)
 ap.add_argument("--nrhs", type=int, default=None)
 ap.add_argument("--tag", default="")
+ap.add_argument("--depth", type=int, default=-1)
 a = ap.parse_args()
 M, b = g.gen_config(a.config, nrhs=a.nrhs or 1)
-plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val)
+plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, depth=a.depth)
 B = torch.from_numpy(b).cuda().T
 if B.shape[1] == 1:
     B = B[:, 0].contiguous()

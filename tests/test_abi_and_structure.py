@@ -109,6 +109,28 @@ def test_structure_parity_c2_full_size():
     assert plan.info()["depth"] == 1
 
 
+def test_b200_depth_retune_keeps_narrow_root_whole():
+    """Reading R30: with the library's defaults (selector B200, depth and
+    min_block_rows unset) C2's root -- every level <= 1,000 rows, <= 2
+    dependencies per row -- stays one triangle (the wavefront solves it
+    whole); the structure is then the oracle's at depth 0.  An explicit
+    min_block_rows (or depth) restores the paper's rule; so does PAPER."""
+    M, _ = g.gen_config("C2")
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, host_only=True)
+    info = plan.info()
+    assert info["depth"] == 0 and info["depth_rule"] == 1
+    assert [s["impl"] for s in plan.segments()] == ["TRI_PIPE"]
+    _compare(M, plan, st.analyse(M, depth=0))
+    paper = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, host_only=True, selector="PAPER")
+    assert paper.info()["depth"] == 1 and paper.info()["depth_rule"] == 0
+    forced = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, host_only=True, depth=1)
+    assert forced.info()["depth_rule"] == 2
+    # a wide-level root keeps the paper's depth (C5 shape, 150K rows, T small)
+    M5 = g.c5_random_multirhs(n=150_001)
+    p5 = sp.sptrsv_analyse(M5.row_ptr, M5.col_idx, M5.val, host_only=True)
+    assert p5.info()["depth_rule"] == 0
+
+
 @pytest.mark.parametrize("shape", ["diag", "chain", "dense", "arrow", "fig1", "n1", "n2", "empty"])
 def test_structure_parity_adversarial(shape):
     M = {"diag": lambda: g.shape_diagonal(1000), "chain": lambda: g.shape_bidiagonal(3000),

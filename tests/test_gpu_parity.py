@@ -315,3 +315,15 @@ def test_square_row_blocks(gpu, depth, dtype, reorder):
         _check64(M, b, x)
     else:
         assert on.rel_err(x, on.solve(M, b)) <= TOL32
+
+
+def test_full_size_c2_default_plan(gpu):
+    """BASELINE configs[1] at full size with the library defaults: the B200
+    depth retune (R30) keeps the 1,999-level root whole and the strand
+    wavefront solves it; every component matches the oracle."""
+    M, b = g.gen_config("C2", nrhs=1)
+    x, plan = _solve(M, b)
+    info = plan.info()
+    assert info["depth"] == 0 and info["depth_rule"] == 1
+    assert [s["impl"] for s in plan.segments()] == ["TRI_PIPE"]
+    _check64(M, b, x)
