@@ -114,7 +114,13 @@ typedef struct {
   int32_t sm_count;         /* 0 = query the device (148 assumed when host_only)               */
   int32_t threads;          /* host threads for the analysis; 0 = hardware concurrency         */
   int32_t device;           /* CUDA device ordinal the plan lives on; -1 = the current device  */
-  int32_t reserved[8];
+  int32_t transpose;        /* 0 = the plan solves A x = b (default); 1 = it solves A^T x = b
+                               for the given A (the preconditioner's transposed sweep, L33/L35;
+                               SURVEY 8(f) f-4).  The given fill is validated as usual; the
+                               system solved has the other fill (sptrsv_plan_info reports it).
+                               The transpose is built on the host during the analysis; the solve
+                               path is the one of an analysed A^T (R31).             */
+  int32_t reserved[7];
 } sptrsv_opts_t;
 
 /* Fill *o with the defaults above. */

@@ -175,8 +175,10 @@ def sptrsv_analyse(row_ptr, col_idx, val, n: int | None = None, fill: str = "L",
                    depth: int = -1, min_block_rows: int = 0, reorder="auto", selector: str = "B200",
                    force_tri_impl: str | None = None, force_sq_impl: str | None = None,
                    host_only: bool = False, sm_count: int = 0, threads: int = 0, stream=None,
-                   device: int | None = None) -> Plan:
+                   device: int | None = None, transpose: bool = False) -> Plan:
     """Preprocess a CSR lower (fill='L') or upper (fill='U') triangular matrix.
+
+    transpose=True: the plan solves A^T x = b for the given A (R31).
 
     reorder: True = level-set reordering of every triangle (the paper, L231),
     False = none, "auto" = none for supernodal inputs, else level (R29).
@@ -203,6 +205,7 @@ def sptrsv_analyse(row_ptr, col_idx, val, n: int | None = None, fill: str = "L",
     o.sm_count = sm_count
     o.threads = threads
     o.device = -1
+    o.transpose = 1 if transpose else 0
     if not host_only:
         import torch
         if torch.cuda.is_available():

@@ -36,7 +36,8 @@ class Opts(ctypes.Structure):
     _fields_ = [("variant", ctypes.c_int32), ("depth", ctypes.c_int32), ("min_block_rows", ctypes.c_int64),
                 ("reorder", ctypes.c_int32), ("selector", ctypes.c_int32), ("force_tri_impl", ctypes.c_int32),
                 ("force_sq_impl", ctypes.c_int32), ("host_only", ctypes.c_int32), ("sm_count", ctypes.c_int32),
-                ("threads", ctypes.c_int32), ("device", ctypes.c_int32), ("reserved", ctypes.c_int32 * 8)]
+                ("threads", ctypes.c_int32), ("device", ctypes.c_int32), ("transpose", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 7)]
 
 
 class PlanInfo(ctypes.Structure):

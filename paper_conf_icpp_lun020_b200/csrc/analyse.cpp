@@ -150,6 +150,40 @@ void to_lower(LowerCSR& L, int32_t n, const int32_t* rp, const int32_t* ci, cons
   L.val = L.val_own.data();
 }
 
+// Lower CSR of the transposed input (R31): the
+// plan then solves A^T x = b.  A = L (LOWER): L^T is upper and is mapped to
+// J L^T J, entry (i, j) -> (n-1-j, n-1-i); A = U (UPPER): U^T is lower as is,
+// entry (i, j) -> (j, i).  A counting sort by destination row; source rows are
+// walked in the order that makes every destination row's columns ascending
+// (descending i for L, ascending i for U), so the diagonal lands last.
+void to_lower_transposed(LowerCSR& L, int32_t n, const int32_t* rp, const int32_t* ci, const char* val,
+                         size_t vb, sptrsv_fill_t fill) {
+  L.n = n;
+  int64_t nnz = rp[n];
+  const bool low = fill == SPTRSV_LOWER;
+  L.rp.assign((size_t)n + 1, 0);
+  for (int64_t q = 0; q < nnz; ++q) {
+    int32_t r = low ? n - 1 - ci[q] : ci[q];
+    ++L.rp[(size_t)r + 1];
+  }
+  for (int32_t r = 0; r < n; ++r) L.rp[r + 1] += L.rp[r];
+  std::vector<int64_t> pos(L.rp.begin(), L.rp.end() - 1);
+  L.ci_own.resize((size_t)nnz);
+  L.val_own.resize((size_t)nnz * vb);
+  for (int32_t t = 0; t < n; ++t) {
+    int32_t i = low ? n - 1 - t : t;
+    int32_t c = low ? n - 1 - i : i;
+    for (int64_t q = rp[i]; q < rp[i + 1]; ++q) {
+      int32_t r = low ? n - 1 - ci[q] : ci[q];
+      int64_t o = pos[r]++;
+      L.ci_own[o] = c;
+      std::memcpy(&L.val_own[(size_t)o * vb], val + (size_t)q * vb, vb);
+    }
+  }
+  L.ci = L.ci_own.data();
+  L.val = L.val_own.data();
+}
+
 // Reading R2: largest d with d == 0 or floor(n / 2^d) >= T.
 int32_t depth_rule(int64_t n, int64_t T) {
   int32_t d = 0;
@@ -338,7 +372,13 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
   if (e.status) return e;
   clk.lap("validate");
   LowerCSR L;
-  to_lower(L, n, row_ptr, col_idx, val, vb, p.fill, threads);
+  if (p.opts.transpose) {
+    // the system solved is A^T: its fill is the other one (R31)
+    to_lower_transposed(L, n, row_ptr, col_idx, val, vb, p.fill);
+    p.fill = p.fill == SPTRSV_LOWER ? SPTRSV_UPPER : SPTRSV_LOWER;
+  } else {
+    to_lower(L, n, row_ptr, col_idx, val, vb, p.fill, threads);
+  }
   clk.lap("to_lower");
   p.n = n;
   p.nnz = nnz;

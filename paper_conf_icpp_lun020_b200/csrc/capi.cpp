@@ -90,6 +90,7 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_analyse(int32_t n, int64_t nnz, const int32
   if (o.reorder < 0 || o.reorder > 2) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad reorder");
   if (o.selector < 0 || o.selector > 1) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad selector");
   if (o.min_block_rows < 0) return fail(SPTRSV_ERROR_INVALID_VALUE, "min_block_rows < 0");
+  if (o.transpose < 0 || o.transpose > 1) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad transpose");
 
   sptrsv_plan_s* P = new (std::nothrow) sptrsv_plan_s();
   if (!P) return fail(SPTRSV_ERROR_ALLOC, "host allocation failed");

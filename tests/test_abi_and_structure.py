@@ -87,6 +87,35 @@ def test_structure_parity_upper(name):
     _compare(U, plan, st.analyse(U, depth=2))
 
 
+@pytest.mark.parametrize("name", ["C1", "C2", "C3", "C5"])
+@pytest.mark.parametrize("uplo", ["L", "U"])
+def test_structure_parity_transpose(name, uplo):
+    """transpose=1 (R31): the plan of A analysed for A^T x = b is, bit for bit,
+    the oracle's analysis of A^T (the other fill), for both fills of A."""
+    M, _ = g.gen_config(name, small=True)
+    if uplo == "U":
+        M = g.to_upper(M)
+    plan = _analyse(M, depth=2, transpose=True)
+    MT = g.transpose(M)
+    assert plan.info()["fill"] == (C.UPPER if uplo == "L" else C.LOWER)
+    _compare(MT, plan, st.analyse(MT, depth=2))
+
+
+def test_transpose_large_matches_analysed_transpose():
+    """Above the parallel grain: the library's host transpose gives the same
+    plan as analysing the explicitly transposed input (plan hash, perm,
+    segments and P A P^T bit for bit)."""
+    M = g.c5_random_multirhs(n=150_001)
+    a = _analyse(M, depth=3, transpose=True, threads=16)
+    MT = g.transpose(M)
+    b = _analyse(MT, depth=3, threads=16)
+    assert a.hash() == b.hash()
+    assert np.array_equal(a.perm(), b.perm())
+    assert a.segments() == b.segments()
+    for x, y in zip(a.matrix(), b.matrix()):
+        assert np.array_equal(x, y)
+
+
 @pytest.mark.parametrize("name", ["C3", "C4"])
 def test_structure_parity_no_reorder(name):
     M, _ = g.gen_config(name, small=True)

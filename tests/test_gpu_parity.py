@@ -135,6 +135,28 @@ def test_upper(gpu, name):
     _check64(U, b, x)
 
 
+@pytest.mark.parametrize("name", CONFIGS)
+@pytest.mark.parametrize("uplo", ["L", "U"])
+@pytest.mark.parametrize("nrhs", [1, 5])
+def test_transpose(gpu, name, uplo, nrhs):
+    """transpose=1 (R31): the plan of A solves A^T x = b; the oracle solves
+    the explicitly transposed input."""
+    M, b = g.gen_config(name, small=True, nrhs=nrhs)
+    if uplo == "U":
+        M = g.to_upper(M)
+    x, _ = _solve(M, b, depth=2, transpose=True)
+    _check64(g.transpose(M), b, x)
+
+
+@pytest.mark.parametrize("name", ["C2", "C4"])
+def test_full_size_transpose(gpu, name):
+    """Full BASELINE sizes, default options: L^T x = b (the backward sweep of
+    an IC(0) / supernodal preconditioner application)."""
+    M, b = g.gen_config(name, nrhs=1)
+    x, plan = _solve(M, b, transpose=True)
+    _check64(g.transpose(M), b, x)
+
+
 def test_repeated_solves_epoch(gpu):
     M, b = g.gen_config("C3", small=True, nrhs=1)
     plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, depth=2, force_tri_impl="TRI_SYNCFREE")

@@ -91,6 +91,36 @@ def test_brute_force_upper(seed):
     assert on.rel_err(x, ref) < 1e-13
 
 
+@pytest.mark.parametrize("seed", [0, 1])
+@pytest.mark.parametrize("uplo", ["L", "U"])
+def test_brute_force_transposed(seed, uplo):
+    """The transposed-solve inputs (R31): transpose() is the dense transpose
+    entry for entry, and the oracle's solve of it is a dense solve with A^T."""
+    M = g.shape_random_small(80, 0.25, seed=seed + 3)
+    if uplo == "U":
+        M = g.to_upper(M)
+    MT = g.transpose(M)
+    assert MT.uplo != M.uplo
+    assert np.array_equal(_dense(MT), _dense(M).T)
+    T = g.transpose(MT)
+    assert np.array_equal(T.row_ptr, M.row_ptr) and np.array_equal(T.col_idx, M.col_idx)
+    assert np.array_equal(T.val, M.val)
+    b = g.gen_rhs(M.n, 2, seed=seed + 30)
+    x = on.solve(MT, b)
+    ref = scipy.linalg.solve_triangular(_dense(M), b.T, lower=(uplo == "L"), trans="T").T
+    assert on.rel_err(x, ref) < 1e-13
+
+
+def test_transposed_bidiagonal_suffix_sums():
+    """L = unit lower bidiagonal with -1 below the diagonal: L^T x = b is
+    x_i = b_i + x_{i+1}, the suffix sums (exact in integers)."""
+    n = 400
+    L = g.shape_bidiagonal(n, a=1.0)
+    rng = np.random.default_rng(9)
+    b = rng.integers(-9, 9, size=n).astype(np.float64)
+    assert np.array_equal(on.solve(g.transpose(L), b), np.cumsum(b[::-1])[::-1])
+
+
 def test_upper_bidiagonal_suffix_sums():
     n = 500
     U = g.to_upper(g.shape_bidiagonal(n, a=1.0))

@@ -431,3 +431,20 @@ def to_upper(L: Matrix) -> Matrix:
     np.cumsum(counts, out=rp[1:])
     return Matrix(n=n, row_ptr=rp.astype(np.int32), col_idx=nc[order].astype(np.int32),
                   val=L.val[order].copy(), name=L.name + "_upper", meta=dict(L.meta), uplo="U")
+
+
+def transpose(M: Matrix) -> Matrix:
+    """M^T as CSR (the other fill): LOWER L -> upper L^T with the diagonal first
+    in each row, UPPER U -> lower U^T with the diagonal last.  Pure re-indexing
+    (a stable sort of the entries by (column, row)); the input of the
+    transposed-solve parity tests (R31)."""
+    n = M.n
+    rows = np.repeat(np.arange(n, dtype=np.int64), np.diff(M.row_ptr.astype(np.int64)))
+    cols = M.col_idx.astype(np.int64)
+    order = np.lexsort((rows, cols))
+    counts = np.bincount(cols, minlength=n)
+    rp = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(counts, out=rp[1:])
+    return Matrix(n=n, row_ptr=rp.astype(np.int32), col_idx=rows[order].astype(np.int32),
+                  val=M.val[order].copy(), name=M.name + "_T", meta=dict(M.meta),
+                  uplo="U" if M.uplo == "L" else "L")
