@@ -55,6 +55,8 @@ def parse():
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0, help="oracle baseline budget")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--transpose", action="store_true",
+                    help="solve A^T x = b from the workload's A (opts.transpose, DESIGN.md R31)")
     ap.add_argument("--dist", action="store_true",
                     help="run the NCCL sharded multi-RHS path even at world size 1 (tests the code path)")
     return ap.parse_args()
@@ -259,7 +261,7 @@ def main():
     val = M.val if args.dtype == "f64" else M.val.astype(np.float32)
 
     # preprocess (analysis + upload): one warm-up, median of 3
-    kw = dict(selector=args.selector, variant=args.variant)
+    kw = dict(selector=args.selector, variant=args.variant, transpose=args.transpose)
     plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, val, **kw)
     pre = []
     for _ in range(3):
@@ -429,13 +431,13 @@ def main():
         cols = list(range(nrhs)) if nrhs <= 4 else [0, nrhs // 2, nrhs - 1]
         xs = X.double().cpu().numpy()
         xs = xs[None] if xs.ndim == 1 else xs.T[cols]
-        ref = on.solve(M, b_np[cols], threads=min(len(cols), 8))
+        ref = on.solve(g.transpose(M) if args.transpose else M, b_np[cols], threads=min(len(cols), 8))
         parity = {"rel_err": on.rel_err(xs, ref), "tol": 1e-10 if vb == 8 else 1e-4,
                   "columns_checked": len(cols)}
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(M, b_np, args.cpu_seconds)
+        cpu = cpu_baseline(g.transpose(M) if args.transpose else M, b_np, args.cpu_seconds)
 
     if rank == 0:
         line = {
@@ -445,6 +447,7 @@ def main():
             "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
             "config": {"workload": WORKLOAD[cfg], "n": M.n, "nnz": M.nnz, "nrhs": nrhs_total,
                        "nrhs_per_rank": nrhs, "selector": args.selector, "variant": args.variant,
+                       "op": "A^T x = b" if args.transpose else "A x = b",
                        "depth": info["depth"], "segments": len(segs),
                        "l2": "flushed (256 MB write) between timed solves" if not args.no_flush else "not flushed",
                        "parallelism": (f"rhs-columns sharded x{ws} (NCCL scatter/gather only in e2e)" if sharded
