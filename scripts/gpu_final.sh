@@ -23,7 +23,7 @@ for c in ${NCU_CONFIGS:-C2 C3 C4 C5}; do
   steps=2; nr=""; [ $c = C5 ] && nr="--nrhs 512"
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_$c.csv python bench.py --config $c --steps 2 --warmup 3 --no-cpu-baseline > $O/ncu_launch_$c.log 2>&1; echo "ncu launches $c rc=$?"
   case $c in
-    C2) K=tri_wave; S=2;; C3) K=tri_syncfree; S=0;; C4) K=tri_supernode; S=0;; C5) K=sq_multi; S=1;;
+    C2) K=tri_wave; S=1;; C3) K=tri_syncfree; S=0;; C4) K=tri_supernode; S=0;; C5) K=sq_multi; S=1;;
   esac
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:$K -s $S -c 1 -o $O/prof_$c -f python scripts/prof_solve.py --config $c --reps 2 $nr > $O/ncu_$c.log 2>&1; echo "ncu full $c rc=$?"
   # summarise on the box (gpurun brings back <= 64 MiB): launch list, full-set
