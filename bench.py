@@ -332,11 +332,14 @@ def main():
     def run_impl(sg):
         """The kernel family that actually runs the segment at this nrhs: the
         plan's impl for one RHS; with many RHS squares run the SpMM (sq_multi)
-        and the supernodal / wave triangles the multi-RHS sync-free kernel."""
+        and the wave triangles the multi-RHS sync-free kernel; supernodal
+        triangles run tri_supernode_multi from 16 RHS (exec.cu kSnMultiMinRhs)."""
         if nrhs == 1:
             return sg["impl"]
         if sg["kind"] == "SQ":
             return "SQ_SPMM"
+        if sg["impl"] == "TRI_SUPERNODE" and nrhs >= 16 and not os.environ.get("SPTRSV_NO_SN_MULTI"):
+            return "TRI_SUPERNODE_MULTI"
         return {"TRI_SUPERNODE": "TRI_SYNCFREE", "TRI_PIPE": "TRI_SYNCFREE"}.get(sg["impl"], sg["impl"])
 
     names = ["permute_in"] + [f"seg{i}:{run_impl(s)}" for i, s in enumerate(segs)] + ["permute_out"]

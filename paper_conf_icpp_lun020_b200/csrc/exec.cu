@@ -28,6 +28,11 @@ namespace {
 
 size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 
+// Supernodal triangles with at least this many RHS run tri_supernode_multi
+// (dense per-piece tiles over 64-column chunks); fewer columns would leave
+// most of a chunk's lanes idle, so they take the sync-free SpTRSM kernel.
+constexpr int kSnMultiMinRhs = 16;
+
 // SpMM lane geometry for nrhs > 1: G lanes per row, RPT columns per lane per
 // pass (capped by SPTRSV_SPMM="RPTMAX,UN" for tuning; default 8,2), UN row entries per
 // gather round.  `multi_sync` is the sync-free triangle, which always uses
@@ -910,7 +915,15 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
                                                   S.ticket_slot);
             break;
           }
-          [[fallthrough]];  // nrhs > 1: the multi-RHS sync-free kernel on the CSR copy
+          if (nrhs >= kSnMultiMinRhs && !std::getenv("SPTRSV_NO_SN_MULTI")) {
+            const int np = (int)S.sn_ptr.size() - 1;
+            const unsigned g = std::max(1u, std::min<unsigned>(np, p.sm_count * 4));
+            k::tri_supernode_multi<T><<<g, 256, 0, s>>>(np, (const k::SnDesc*)S.d_sn_desc, S.d_sn_cols,
+                                                        (const T*)S.d_sn_vals, (const T*)S.d_sn_blk, bw, xs, st,
+                                                        S.ticket_slot, nrhs);
+            break;
+          }
+          [[fallthrough]];  // 1 < nrhs < 16: the multi-RHS sync-free kernel on the CSR copy
         default: {  // SPTRSV_IMPL_TRI_SYNCFREE
           // enough resident warps for about two of the triangle's widest
           // levels: more only spin on rows whose dependencies are levels away

@@ -821,6 +821,146 @@ __global__ void __launch_bounds__(256, SPTRSV_SN_MINB) tri_supernode(int npieces
   }
 }
 
+// Supernodal SpTRSM (B200 selector, nrhs >= 16): a CTA per
+// supernode piece J = rows [s, s+w), w <= 32, claimed in row order from the
+// segment's ticket, and the RHS in chunks of 64 columns.  Per chunk:
+//   1. Y = B'_J - V_J X[E_J, :] as a register-tiled dense product: the 32
+//      external columns of a round are polled (per-row epoch flags, one thread
+//      each), their X rows (32 x 64) and the matching V_J panel (32 x w) are
+//      staged in shared memory, and warp wi accumulates rows 4wi..4wi+3 x 64
+//      columns (lane and lane+32): 8 DFMA per 4 shared loads, V_J read once
+//      per chunk instead of once per RHS column;
+//   2. X_J = T_J^{-1} Y for the dense unit-lower diagonal block: warp wi owns
+//      8 columns, lane t row t, 31 shfl/DFMA steps with T_J's row in registers;
+//   3. X_J stored coalesced; after the last chunk the piece's row flags are
+//      published (fence, barrier, flag = epoch).
+// In fp64 on B200 the DMMA tensor-core rate is not above the DFMA rate, so
+// the dense tiles run on the FMA pipes (f-3).
+constexpr int kSnmCols = 64;
+template <typename T>
+__global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const SnDesc* __restrict__ desc,
+                                                           const int* __restrict__ cols, const T* __restrict__ V,
+                                                           const T* __restrict__ Tb, const T* __restrict__ bw,
+                                                           T* __restrict__ xs, SolveState st, int slot, int nrhs) {
+  __shared__ __align__(16) T Vs[32][32];
+  __shared__ __align__(16) T Xs[32][kSnmCols];
+  __shared__ __align__(16) T Ys[32][kSnmCols + 1];
+  __shared__ int Js[32];
+  __shared__ int Jsh;
+  const int tid = threadIdx.x, lane = tid & 31, wi = tid >> 5;
+  uint32_t* ticket = st.tickets + slot;
+  const uint32_t epoch = st.epoch;
+  while (true) {
+    if (tid == 0) Jsh = (int)atomicAdd(ticket, 1u);
+    __syncthreads();
+    const int J = Jsh;
+    __syncthreads();  // Jsh is rewritten by the next claim
+    if (J >= npieces) break;
+    const SnDesc d = desc[J];
+    for (int c0 = 0; c0 < nrhs; c0 += kSnmCols) {
+      T acc[4][2];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+          const int t = wi * 4 + i, c = c0 + lane + 32 * u;
+          acc[i][u] = (t < d.w && c < nrhs) ? bw[(int64_t)(d.s + t) * nrhs + c] : T(0);
+        }
+      for (int q0 = 0; q0 < d.ne; q0 += 32) {
+        const int nq = min(32, d.ne - q0);
+        if (tid < nq) {
+          const int j = ldg_nc(cols + d.coff + q0 + tid);
+          Js[tid] = j;
+          if (c0 == 0) {  // later column chunks find the rows already published
+            uint32_t spins = 0;
+            unsigned ns = 0;
+            while (ld_flag(st.flags + j) != epoch) {
+              if (++spins > kWatchdogSpins) {
+                watchdog_trip(st);
+                break;
+              }
+              ns = backoff(ns, st.backoff_ns);
+            }
+            __threadfence();
+          }
+        }
+        // all staging loads of a round are issued before any shared store
+        // (ld_strong is an asm volatile with a memory clobber: interleaved
+        // with the stores it would serialise on the load latency)
+        const T* Vq = V + d.voff + (long long)q0 * d.w;
+        T vr[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int q = (tid >> 5) + 8 * k, t = tid & 31;
+          vr[k] = (q < nq && t < d.w) ? ldg_nc(Vq + (long long)q * d.w + t) : T(0);
+        }
+        __syncthreads();  // Js and the readiness of its rows
+        T xr[32 * kSnmCols / 256];
+#pragma unroll
+        for (int k = 0; k < 32 * kSnmCols / 256; ++k) {
+          const int idx = tid + 256 * k, q = idx / kSnmCols, c = idx % kSnmCols;
+          xr[k] = (q < nq && c0 + c < nrhs) ? ld_strong(xs + (int64_t)Js[q] * nrhs + c0 + c) : T(0);
+        }
+#pragma unroll
+        for (int k = 0; k < 4; ++k) Vs[(tid >> 5) + 8 * k][tid & 31] = vr[k];
+#pragma unroll
+        for (int k = 0; k < 32 * kSnmCols / 256; ++k) {
+          const int idx = tid + 256 * k;
+          Xs[idx / kSnmCols][idx % kSnmCols] = xr[k];
+        }
+        __syncthreads();
+        for (int q = 0; q < nq; ++q) {
+          const T x0 = Xs[q][lane], x1 = Xs[q][lane + 32];
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const T v = Vs[q][wi * 4 + i];
+            acc[i][0] -= v * x0;
+            acc[i][1] -= v * x1;
+          }
+        }
+        __syncthreads();  // Vs / Xs / Js are restaged next round
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        Ys[wi * 4 + i][lane] = acc[i][0];
+        Ys[wi * 4 + i][lane + 32] = acc[i][1];
+      }
+      // T_J column-major in shared memory (aliasing Xs, free after the
+      // product): column c holds rows c+1 .. w-1 (packed as in tri_supernode)
+      T(*Ts)[32] = reinterpret_cast<T(*)[32]>(&Xs[0][0]);
+      for (int idx = tid; idx < 32 * 32; idx += 256) {
+        const int c = idx >> 5, t = idx & 31;
+        const long long off = d.boff + (long long)c * (d.w - 1) - (long long)c * (c - 1) / 2 + (t - c - 1);
+        Ts[c][t] = (t < d.w && t > c && c < d.w - 1) ? ldg_nc(Tb + off) : T(0);
+      }
+      __syncthreads();
+      T y[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) y[i] = Ys[lane][wi * 8 + i];
+#pragma unroll 4
+      for (int c = 0; c < d.w - 1; ++c) {  // CTA-uniform
+        const T tc = Ts[c][lane];          // lanes <= c read 0
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const T xc = __shfl_sync(0xffffffffu, y[i], c);
+          y[i] -= tc * xc;
+        }
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i) Ys[lane][wi * 8 + i] = y[i];
+      __syncthreads();
+      for (int idx = tid; idx < 32 * kSnmCols; idx += 256) {
+        const int t = idx / kSnmCols, c = idx % kSnmCols;
+        if (t < d.w && c0 + c < nrhs) xs[(int64_t)(d.s + t) * nrhs + c0 + c] = Ys[t][c];
+      }
+      __syncthreads();  // Ys is rewritten by the next chunk
+    }
+    __threadfence();  // the piece's x stores are visible at gpu scope ...
+    __syncthreads();
+    if (tid < d.w) st_flag(st.flags + d.s + tid, epoch);  // ... before its row flags
+  }
+}
+
 // Multi-RHS sync-free (SpTRSM): a group of G lanes per component, lanes over
 // the RHS columns.  Readiness is a per-row flag holding the solve's epoch
 // (no per-solve reset, no n x nrhs sentinel fill): the G lanes store the row,

@@ -113,6 +113,37 @@ def test_supernodal_default_and_reorders(gpu, name, reorder):
     _check64(M, b, x)
 
 
+@pytest.mark.parametrize("nrhs", [15, 16, 64, 65, 130])
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+@pytest.mark.parametrize("layout", ["col", "row"])
+def test_supernode_multi_rhs(gpu, nrhs, dtype, layout):
+    """f-3: C4's supernodal plan with nrhs >= 16 runs tri_supernode_multi
+    (64-column chunks, ragged last chunk at 65 / 130, ragged 32-row pieces);
+    15 RHS take the sync-free SpTRSM kernel."""
+    M, b = g.gen_config("C4", small=True, nrhs=nrhs)
+    x, plan = _solve(M, b, dtype=dtype, layout=layout, depth=1)
+    assert any(s["impl"] == "TRI_SUPERNODE" for s in plan.segments())
+    if dtype == torch.float64:
+        _check64(M, b, x)
+    else:
+        assert on.rel_err(x, on.solve(M, b)) <= TOL32
+
+
+def test_full_size_c4_supernode_multi_sampled(gpu):
+    """C4 at full size (n=500K, 80M nnz) with 64 RHS through the default
+    plan: sampled columns against the oracle."""
+    M, b = g.gen_config("C4", nrhs=64)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val)
+    X = sp.sptrsv_solve(plan, torch.from_numpy(b).cuda().T)
+    torch.cuda.synchronize()
+    cols = [0, 31, 32, 63]
+    xs = X[:, cols].T.cpu().numpy()
+    ref = on.solve(M, b[cols], threads=4)
+    assert on.rel_err(xs, ref) <= TOL64
+    ok, worst = on.residual_bound_ok(M, xs, b[cols])
+    assert ok, worst
+
+
 @pytest.mark.parametrize("layout", ["col", "row"])
 def test_layouts(gpu, layout):
     M, b = g.gen_config("C5", small=True, nrhs=9)
@@ -284,7 +315,8 @@ def test_full_size_configs(gpu, name):
     err = _check64(M, b, x)
     # the plan's structure at full size is the oracle's (for the reorder the
     # B200 default chose: none for the supernodal C4, level otherwise, R29)
-    A = st.analyse(M, min_block_rows=B200_T, reorder=plan.info()["reorder"] == 0)
+    # at the depth the plan reports (the B200 depth retune keeps C2 whole, R30)
+    A = st.analyse(M, depth=plan.info()["depth"], reorder=plan.info()["reorder"] == 0)
     segs = plan.segments()
     assert [(s["row0"], s["row1"], s["col0"], s["col1"], s["nnz"], s["nlevels"], s["kernel"])
             for s in segs] == [(o.row0, o.row1, o.col0, o.col1, o.nnz, o.nlevels, o.kernel) for o in A.segs]
