@@ -845,7 +845,7 @@ __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const
   __shared__ __align__(16) T Vs[32][32];
   __shared__ __align__(16) T Xs[32][kSnmCols];
   __shared__ __align__(16) T Ys[32][kSnmCols + 1];
-  __shared__ int Js[32];
+  __shared__ int Js[2][32];
   __shared__ int Jsh;
   const int tid = threadIdx.x, lane = tid & 31, wi = tid >> 5;
   uint32_t* ticket = st.tickets + slot;
@@ -866,11 +866,15 @@ __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const
           const int t = wi * 4 + i, c = c0 + lane + 32 * u;
           acc[i][u] = (t < d.w && c < nrhs) ? bw[(int64_t)(d.s + t) * nrhs + c] : T(0);
         }
-      for (int q0 = 0; q0 < d.ne; q0 += 32) {
+      // round prologue for external columns [q0, q0+32): one thread per
+      // column loads its index into Js[buf] and (first chunk only) polls its
+      // epoch flag; every thread loads its part of the V_J panel to registers
+      T vr[4];
+      auto prep = [&](int q0, int buf) {
         const int nq = min(32, d.ne - q0);
         if (tid < nq) {
           const int j = ldg_nc(cols + d.coff + q0 + tid);
-          Js[tid] = j;
+          Js[buf][tid] = j;
           if (c0 == 0) {  // later column chunks find the rows already published
             uint32_t spins = 0;
             unsigned ns = 0;
@@ -884,22 +888,28 @@ __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const
             __threadfence();
           }
         }
-        // all staging loads of a round are issued before any shared store
-        // (ld_strong is an asm volatile with a memory clobber: interleaved
-        // with the stores it would serialise on the load latency)
         const T* Vq = V + d.voff + (long long)q0 * d.w;
-        T vr[4];
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
           const int q = (tid >> 5) + 8 * k, t = tid & 31;
           vr[k] = (q < nq && t < d.w) ? ldg_nc(Vq + (long long)q * d.w + t) : T(0);
         }
-        __syncthreads();  // Js and the readiness of its rows
+      };
+      prep(0, 0);
+      __syncthreads();  // Js[0] and the readiness of its rows
+      // two barriers per round: the next round's prologue runs between the
+      // product and the barrier that ends the round (Js is double-buffered;
+      // Vs / Xs are rewritten only after that barrier)
+      for (int q0 = 0, buf = 0; q0 < d.ne; q0 += 32, buf ^= 1) {
+        const int nq = min(32, d.ne - q0);
+        // all staging loads of a round are issued before any shared store
+        // (ld_strong is an asm volatile with a memory clobber: interleaved
+        // with the stores it would serialise on the load latency)
         T xr[32 * kSnmCols / 256];
 #pragma unroll
         for (int k = 0; k < 32 * kSnmCols / 256; ++k) {
           const int idx = tid + 256 * k, q = idx / kSnmCols, c = idx % kSnmCols;
-          xr[k] = (q < nq && c0 + c < nrhs) ? ld_strong(xs + (int64_t)Js[q] * nrhs + c0 + c) : T(0);
+          xr[k] = (q < nq && c0 + c < nrhs) ? ld_strong(xs + (int64_t)Js[buf][q] * nrhs + c0 + c) : T(0);
         }
 #pragma unroll
         for (int k = 0; k < 4; ++k) Vs[(tid >> 5) + 8 * k][tid & 31] = vr[k];
@@ -918,7 +928,8 @@ __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const
             acc[i][1] -= v * x1;
           }
         }
-        __syncthreads();  // Vs / Xs / Js are restaged next round
+        if (q0 + 32 < d.ne) prep(q0 + 32, buf ^ 1);
+        __syncthreads();  // Vs / Xs are restaged next round, Js[buf ^ 1] is ready
       }
 #pragma unroll
       for (int i = 0; i < 4; ++i) {

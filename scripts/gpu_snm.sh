@@ -1,6 +1,6 @@
 #!/bin/bash
 # tri_supernode_multi iteration: parity tests, C4 multi-RHS bench lines, one ncu capture
-O=gpurun_out/snm
+O=gpurun_out/${OUTDIR:-snm}
 mkdir -p $O
 timeout 900 python -m pytest tests -m gpu -q -k "supernode_multi or (test_multi_rhs and SUPERNODE) or test_supernodal" > $O/pytest.log 2>&1; echo "pytest rc=$?"; tail -2 $O/pytest.log
 summ() { python - "$1" <<'PY'
