@@ -4,6 +4,7 @@ bit-exact against the structural oracle (levels, permutation, block
 partition, features, Alg 7 labels, formats, the permuted matrix).
 
 No compute call is made here (host_only plans: no device is touched)."""
+import ctypes
 import os
 import re
 
@@ -218,6 +219,28 @@ def test_validation_errors():
     _expect("NOT_TRIANGULAR", [0, 1, 3], [0, 0, 1], [1.0, 2.0, 1.0], fill="U")  # (1,0) below diag
     _expect("INVALID_VALUE", [0, 1, 3], [0, 0, 5], [1.0, 2.0, 1.0])     # column out of range
     _expect("INVALID_VALUE", [1, 1, 3], [0, 0, 1], [1.0, 2.0, 1.0])     # row_ptr[0] != 0
+
+
+def test_transpose_validates_the_given_fill():
+    """transpose=1 (R31) checks A with its own fill before transposing: an
+    entry above the diagonal of a LOWER input is still NOT_TRIANGULAR, a
+    missing diagonal still ZERO_PIVOT; a bad transpose value is rejected."""
+    _expect("NOT_TRIANGULAR", [0, 2, 3], [0, 1, 1], [1.0, 2.0, 1.0], transpose=True)
+    _expect("ZERO_PIVOT", [0, 1, 2], [0, 0], [1.0, 2.0], transpose=True)
+    _expect("NOT_TRIANGULAR", [0, 1, 3], [0, 0, 1], [1.0, 2.0, 1.0], fill="U", transpose=True)
+    o = C.Opts()
+    C.lib().sptrsv_opts_default(ctypes.byref(o))
+    assert o.transpose == 0
+    o.transpose = 2
+    o.host_only = 1
+    rp = np.array([0, 1], dtype=np.int32)
+    ci = np.array([0], dtype=np.int32)
+    va = np.array([1.0])
+    h = ctypes.c_void_p()
+    st_ = C.lib().sptrsv_analyse(1, 1, rp.ctypes.data_as(ctypes.c_void_p), ci.ctypes.data_as(ctypes.c_void_p),
+                                 va.ctypes.data_as(ctypes.c_void_p), 0, C.LOWER, ctypes.byref(o), None,
+                                 ctypes.byref(h))
+    assert st_ == 1 and not h.value  # SPTRSV_ERROR_INVALID_VALUE, no plan
 
 
 def test_validation_error_names_row():
