@@ -360,7 +360,9 @@ def main():
         dbytes = M.n * 4 + 2 * M.n * nrhs * vb
         dimpl = "PERMUTE"
     achieved = dbytes / (seg_mean[dom] / 1e3) / 1e9
-    tr = load_traffic(f"{cfg}:{dimpl}")
+    # the committed capture is per (config, kernel) at the config's default
+    # RHS count; other RHS counts carry their own key ("C4:...@64")
+    tr = load_traffic(f"{cfg}:{dimpl}" + (f"@{nrhs}" if nrhs_total != DEFAULT_NRHS[cfg] else ""))
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": tr, "kernel": names[dom], "share_of_step": float(seg_mean[dom] / seg_mean.sum()),
                 "alg_bytes_per_launch": dbytes,
