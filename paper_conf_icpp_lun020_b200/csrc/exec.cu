@@ -918,9 +918,21 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
           if (nrhs >= kSnMultiMinRhs && !std::getenv("SPTRSV_NO_SN_MULTI")) {
             const int np = (int)S.sn_ptr.size() - 1;
             const unsigned g = std::max(1u, std::min<unsigned>(np, p.sm_count * 4));
-            k::tri_supernode_multi<T><<<g, 256, 0, s>>>(np, (const k::SnDesc*)S.d_sn_desc, S.d_sn_cols,
-                                                        (const T*)S.d_sn_vals, (const T*)S.d_sn_blk, bw, xs, st,
-                                                        S.ticket_slot, nrhs);
+            // one launch per 64-column chunk: inside a launch a piece's
+            // chunks would run one after the other on the elimination-tree
+            // chain; as separate launches each chain is one chunk long.
+            // Launch i polls and publishes epoch + i and reclaims pieces from
+            // a re-zeroed ticket.
+            const int nch = (int)cdiv(nrhs, k::kSnmCols);
+            for (int c = 0; c < nch; ++c) {
+              k::SolveState sc = st;
+              sc.epoch = st.epoch + (uint32_t)c;
+              if (c > 0) CUDA_TRY(cudaMemsetAsync(st.tickets + S.ticket_slot, 0, 4, s));
+              k::tri_supernode_multi<T><<<g, 256, 0, s>>>(np, (const k::SnDesc*)S.d_sn_desc, S.d_sn_cols,
+                                                          (const T*)S.d_sn_vals, (const T*)S.d_sn_blk, bw, xs, sc,
+                                                          S.ticket_slot, nrhs, c * k::kSnmCols,
+                                                          std::min(nrhs, (c + 1) * k::kSnmCols));
+            }
             break;
           }
           [[fallthrough]];  // 1 < nrhs < 16: the multi-RHS sync-free kernel on the CSR copy
@@ -1045,11 +1057,15 @@ Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs
       CUDA_TRY(cudaMemsetAsync(p.ws.flags, 0, (size_t)std::max(1, n) * 4, s));
       p.epoch = 0;
     }
-    if (++p.epoch == 0) {  // wrapped after 2^32 solves: restart from clean flags
+    // a solve owns epochs [base, base + span): the supernodal SpTRSM runs
+    // one launch per 64-column chunk, each with its own epoch (exec: kSnmSplit)
+    const uint32_t span = (uint32_t)std::max<int64_t>(1, cdiv(nrhs, k::kSnmCols));
+    if (p.epoch > 0xFFFFFFFFu - span - 1u) {  // about to wrap: restart from clean flags
       CUDA_TRY(cudaMemsetAsync(p.ws.flags, 0, (size_t)std::max(1, n) * 4, s));
-      p.epoch = 1;
+      p.epoch = 0;
     }
-    epoch = p.epoch;
+    epoch = p.epoch + 1;
+    p.epoch += span;
   }
   k::SolveState st{p.d_tickets, p.nticket, p.d_error, (uint32_t*)p.ws.flags, epoch, p.backoff_ns};
   cudaEvent_t* ev = nullptr;

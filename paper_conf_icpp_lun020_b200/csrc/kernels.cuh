@@ -841,7 +841,8 @@ template <typename T>
 __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const SnDesc* __restrict__ desc,
                                                            const int* __restrict__ cols, const T* __restrict__ V,
                                                            const T* __restrict__ Tb, const T* __restrict__ bw,
-                                                           T* __restrict__ xs, SolveState st, int slot, int nrhs) {
+                                                           T* __restrict__ xs, SolveState st, int slot, int nrhs,
+                                                           int c_lo, int c_hi) {
   __shared__ __align__(16) T Vs[32][32];
   __shared__ __align__(16) T Xs[32][kSnmCols];
   __shared__ __align__(16) T Ys[32][kSnmCols + 1];
@@ -857,7 +858,7 @@ __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const
     __syncthreads();  // Jsh is rewritten by the next claim
     if (J >= npieces) break;
     const SnDesc d = desc[J];
-    for (int c0 = 0; c0 < nrhs; c0 += kSnmCols) {
+    for (int c0 = c_lo; c0 < c_hi; c0 += kSnmCols) {
       T acc[4][2];
 #pragma unroll
       for (int i = 0; i < 4; ++i)
@@ -875,7 +876,7 @@ __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const
         if (tid < nq) {
           const int j = ldg_nc(cols + d.coff + q0 + tid);
           Js[buf][tid] = j;
-          if (c0 == 0) {  // later column chunks find the rows already published
+          if (c0 == c_lo) {  // later column chunks find the rows already published
             uint32_t spins = 0;
             unsigned ns = 0;
             while (ld_flag(st.flags + j) != epoch) {

@@ -2,7 +2,7 @@
 # tri_supernode_multi iteration: parity tests, C4 multi-RHS bench lines, one ncu capture
 O=gpurun_out/${OUTDIR:-snm}
 mkdir -p $O
-timeout 900 python -m pytest tests -m gpu -q -k "supernode_multi or (test_multi_rhs and SUPERNODE) or test_supernodal" > $O/pytest.log 2>&1; echo "pytest rc=$?"; tail -2 $O/pytest.log
+timeout 900 python -m pytest tests -m gpu -q -k "supernode_multi or test_multi_rhs or test_supernodal or epoch or pipelined or layouts or full_size_c5" > $O/pytest.log 2>&1; echo "pytest rc=$?"; tail -2 $O/pytest.log
 summ() { python - "$1" <<'PY'
 import json,sys
 for l in open(sys.argv[1]):

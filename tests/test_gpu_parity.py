@@ -129,6 +129,20 @@ def test_supernode_multi_rhs(gpu, nrhs, dtype, layout):
         assert on.rel_err(x, on.solve(M, b)) <= TOL32
 
 
+def test_supernode_multi_repeated_solves_epochs(gpu):
+    """A multi-RHS solve owns one epoch per 64-column chunk (one supernodal
+    launch per chunk): repeated solves on one plan with changing RHS counts
+    never see a stale flag."""
+    M, b = g.gen_config("C4", small=True, nrhs=130)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, depth=1)
+    for k in (130, 20, 130, 64, 3, 130):
+        bk = np.ascontiguousarray(b[:k]) * (1.0 + 0.1 * k)
+        X = sp.sptrsv_solve(plan, torch.from_numpy(bk).cuda().T)
+        torch.cuda.synchronize()
+        _check64(M, bk, X.T.cpu().numpy())
+    plan.free()
+
+
 def test_full_size_c4_supernode_multi_sampled(gpu):
     """C4 at full size (n=500K, 80M nnz) with 64 RHS through the default
     plan: sampled columns against the oracle."""
