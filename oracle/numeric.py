@@ -34,8 +34,6 @@ def lib():
                                   ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32]
         L.oracle_levels.restype = ctypes.c_int32
         L.oracle_levels.argtypes = [ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]
-        L.oracle_forward_f32.restype = None
-        L.oracle_forward_f32.argtypes = [ctypes.c_int32] + [ctypes.c_void_p] * 5
         _lib = L
     return _lib
 

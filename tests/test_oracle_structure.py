@@ -77,10 +77,46 @@ def test_c3_levels_by_construction():
     assert np.array_equal(lev, want)
 
 
+# PAPER.md:L329-L334 (Table 4): n, #level-sets, parallelism min / ave. / max as printed
+TABLE4 = [
+    ("nlpkkt200", 16240000, 2, 8000000, 8120000, 8240000),
+    ("mawi_201512020030", 68863315, 19, 11, 3624385, 34544376),
+    ("kkt_power", 2063494, 17, 1090, 121382, 626597),
+    ("FullChip", 2987012, 324, 1, 9219, 468405),
+    ("vas_stokes_4M", 4382246, 2815, 1, 1556, 37519),
+    ("tmt_sym", 726713, 726235, 1, 1, 135),
+]
+
+
+def _levels_with_sizes(n, nl, mn, mx):
+    """A level vector of n rows in nl levels whose smallest level has mn rows
+    and whose largest has mx rows (the rest filled greedily within [mn, mx])."""
+    sizes = np.full(nl, mn, dtype=np.int64)
+    sizes[-1] = mx
+    rest = n - sizes.sum()
+    assert rest >= 0
+    i = 1
+    while rest > 0:
+        add = min(rest, mx - sizes[i])
+        sizes[i] += add
+        rest -= add
+        i += 1
+    assert sizes.sum() == n and sizes.min() == mn and sizes.max() == mx
+    return np.repeat(np.arange(nl, dtype=np.int32), sizes)
+
+
+@pytest.mark.parametrize("row", TABLE4, ids=[r[0] for r in TABLE4])
+def test_table4_level_stats_reproduce_printed_parallelism(row):
+    """level_stats against every Table 4 row: a level
+    vector with the printed n, #level-sets and min / max widths must give the
+    printed 'ave.' -- floor(n / #levels): FullChip (9219.2) and vas_stokes_4M
+    (1556.7) separate floor from rounding."""
+    _name, n, nl, mn, ave, mx = row
+    lev = _levels_with_sizes(n, nl, mn, mx)
+    assert st.level_stats(lev, nl) == (mn, ave, mx)
+
+
 def test_table4_average_parallelism_convention():
-    # floor, not round
-    assert 4382246 // 2815 == 1556
-    assert 726713 // 726235 == 1
     lev = np.array([0, 0, 0, 1, 1, 2, 3], dtype=np.int32)
     assert st.level_stats(lev, 4) == (1, 1, 3)
 
@@ -137,7 +173,9 @@ def test_alg7_triangle_boundaries():
     assert S.select_tri(1, 1) == S.TRI_COMPLETELY_PARALLEL
     assert S.select_tri(1, 40) == S.TRI_COMPLETELY_PARALLEL
     assert S.select_tri(20001, 1) == S.TRI_NEAR_SERIAL
-    assert S.select_tri(20000, 1) == S.TRI_LEVEL_SET if 20000 <= 100 else S.TRI_SYNC_FREE
+    # 20000 levels at nnz/row 1: not <= 100 levels (first level-set branch), not
+    # <= 20 levels (second), not > 20000 (near-serial) -> Sync-free
+    assert S.select_tri(20000, 1) == S.TRI_SYNC_FREE
     assert S.select_tri(100, 1) == S.TRI_LEVEL_SET
     assert S.select_tri(101, 1) == S.TRI_SYNC_FREE
     assert S.select_tri(20, 15) == S.TRI_LEVEL_SET
@@ -269,6 +307,17 @@ def test_reorder_none_keeps_identity():
     A = st.analyse(M, depth=2, reorder=False)
     assert np.array_equal(A.perm, np.arange(M.n))
     assert sum(s.nnz for s in A.segs) == M.nnz
+
+
+def test_clamp_depth_brute_force():
+    """R1b by brute force: the clamped depth is the LARGEST d <= the forced
+    depth whose REC partition (mid = lo + floor((hi-lo)/2))
+    leaves every one of its 2^d triangles non-empty."""
+    for n in range(1, 80):
+        for forced in range(0, 9):
+            ok = [d for d in range(forced + 1)
+                  if all(s.row1 > s.row0 for s in st.partition(n, d, "REC") if s.kind == "TRI")]
+            assert st.clamp_depth(n, forced) == max(ok), (n, forced)
 
 
 def test_degenerate_sizes():
