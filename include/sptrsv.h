@@ -120,7 +120,24 @@ typedef struct {
                                system solved has the other fill (sptrsv_plan_info reports it).
                                The transpose is built on the host during the analysis; the solve
                                path is the one of an analysed A^T (R31).             */
-  int32_t reserved[7];
+  int32_t max_nrhs;         /* solve workspace sized at analysis for this many right-hand sides
+                               (0 = allocated at the first solve that needs it)                 */
+  int32_t graphs;           /* 1 (default) = a device solve whose (b, x, ldb, ldx, nrhs, layout)
+                               repeats the previous uncaptured one is captured into a CUDA graph;
+                               later solves with a captured key replay it (one graph launch).
+                               0 = always launch the kernels one by one                        */
+  int32_t reserved[5];
+  /* Device-memory hooks (SURVEY 8(b) "PyTorch for device memory"): when
+   * dev_alloc is set, EVERY device allocation of the plan (arena, solve
+   * workspace, flags, staging) goes through dev_alloc(bytes, stream, ctx) and
+   * is returned by dev_free(ptr, stream, ctx); the Python binding passes the
+   * torch CUDA caching allocator.  NULL = cudaMalloc / cudaFree.  dev_alloc
+   * returns NULL on failure (SPTRSV_ERROR_ALLOC).  Both are called from the
+   * thread calling sptrsv_analyse / sptrsv_solve / sptrsv_free, never during
+   * graph capture or from device code. */
+  void* (*dev_alloc)(size_t bytes, void* stream, void* ctx);
+  void (*dev_free)(void* ptr, void* stream, void* ctx);
+  void* alloc_ctx;
 } sptrsv_opts_t;
 
 /* Fill *o with the defaults above. */
@@ -161,14 +178,24 @@ sptrsv_status_t sptrsv_analyse(int32_t n, int64_t nnz, const int32_t* row_ptr, c
  *   Mixed host/device b and x is INVALID_VALUE.
  * One solve may be in flight per plan (the plan owns the solve workspace and
  * the per-row ready flags); concurrent use from two streams is undefined.
- * The first call for a given nrhs may allocate workspace.
+ * The first call for a given nrhs may allocate workspace (none when
+ * opts.max_nrhs covers it).  With opts.graphs, the second consecutive device
+ * solve with the same (b, x, ldb, ldx, nrhs, layout) captures the solve into
+ * a CUDA graph and every later solve with that key is one graph launch
+ * (at most 8 graphs are cached per plan, least recently used evicted).  If
+ * the caller's stream is itself being captured, the kernels are enqueued
+ * into the caller's capture instead.
+ * b and x must live on the plan's device (INVALID_VALUE otherwise) and hold
+ * the plan's dtype (not checkable here: the Python binding checks it).
  * Errors: INVALID_VALUE, NOT_SUPPORTED (host_only plan, non-sm_100 device),
  * ALLOC, CUDA, DEADLOCK (a watchdog of an EARLIER solve tripped).
  */
 sptrsv_status_t sptrsv_solve(sptrsv_plan_t plan, const void* b, int64_t ldb, void* x, int64_t ldx,
                              int32_t nrhs, sptrsv_layout_t layout, void* stream);
 
-/* Release the plan (synchronises the device first).  NULL is a no-op. */
+/* Release the plan.  Waits for the plan's last solve (an event recorded on
+ * that solve's stream) -- not for the whole device -- then returns every
+ * device allocation (through dev_free when given).  NULL is a no-op. */
 sptrsv_status_t sptrsv_free(sptrsv_plan_t plan);
 
 /* ---------------------------------------------------------------- introspection

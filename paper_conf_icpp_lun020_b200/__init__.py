@@ -72,10 +72,11 @@ def _stream_handle(stream):
 class Plan:
     """Owns an sptrsv_plan_t (the preprocessed, blocked matrix on the device)."""
 
-    def __init__(self, handle: int, n: int, dtype_code: int, keep=None):
+    def __init__(self, handle: int, n: int, dtype_code: int, keep=None, device: int = -1):
         self._h = ctypes.c_void_p(handle)
         self.n = n
         self.dtype_code = dtype_code
+        self.device = device
         self._keep = keep
 
     # ---------------------------------------------------------------- solve
@@ -171,17 +172,47 @@ class Plan:
         self.free()
 
 
+# torch's CUDA caching allocator behind the C ABI's dev_alloc / dev_free hooks
+# (include/sptrsv.h): the plan's arena and solve workspace are then torch
+# memory (visible in torch.cuda.memory_allocated).  alloc_ctx carries the
+# device ordinal + 1.  The ctypes thunks live for the whole process.
+def _torch_alloc(nbytes, stream, ctx):
+    try:
+        import torch
+        return torch.cuda.caching_allocator_alloc(int(nbytes), device=int(ctx or 1) - 1, stream=int(stream or 0))
+    except Exception:  # noqa: BLE001 -- reported to C as NULL -> SPTRSV_ERROR_ALLOC
+        return None
+
+
+def _torch_free(ptr, stream, ctx):
+    try:
+        import torch
+        torch.cuda.caching_allocator_delete(int(ptr))
+    except Exception:  # noqa: BLE001 -- interpreter shutdown
+        pass
+
+
+_TORCH_ALLOC = C.DEV_ALLOC(_torch_alloc)
+_TORCH_FREE = C.DEV_FREE(_torch_free)
+
+
 def sptrsv_analyse(row_ptr, col_idx, val, n: int | None = None, fill: str = "L", variant: str = "REC",
                    depth: int = -1, min_block_rows: int = 0, reorder="auto", selector: str = "B200",
                    force_tri_impl: str | None = None, force_sq_impl: str | None = None,
                    host_only: bool = False, sm_count: int = 0, threads: int = 0, stream=None,
-                   device: int | None = None, transpose: bool = False) -> Plan:
+                   device: int | None = None, transpose: bool = False, max_nrhs: int = 0,
+                   graphs: bool = True, allocator: str | None = "torch") -> Plan:
     """Preprocess a CSR lower (fill='L') or upper (fill='U') triangular matrix.
 
     transpose=True: the plan solves A^T x = b for the given A (R31).
 
     reorder: True = level-set reordering of every triangle (the paper, L231),
     False = none, "auto" = none for supernodal inputs, else level (R29).
+
+    allocator: "torch" = every device allocation of the plan goes through
+    torch's CUDA caching allocator (C-ABI dev_alloc hooks); None = cudaMalloc.
+    max_nrhs: size the solve workspace now for this many RHS columns.
+    graphs: replay repeated solves (same b, x, layout) as one CUDA graph.
     """
     rp = _as_int32(row_ptr)
     ci = _as_int32(col_idx)
@@ -206,15 +237,21 @@ def sptrsv_analyse(row_ptr, col_idx, val, n: int | None = None, fill: str = "L",
     o.threads = threads
     o.device = -1
     o.transpose = 1 if transpose else 0
+    o.max_nrhs = int(max_nrhs)
+    o.graphs = 1 if graphs else 0
     if not host_only:
         import torch
         if torch.cuda.is_available():
             o.device = torch.cuda.current_device() if device is None else int(device)
+            if allocator == "torch":
+                o.dev_alloc = _TORCH_ALLOC
+                o.dev_free = _TORCH_FREE
+                o.alloc_ctx = o.device + 1
     h = ctypes.c_void_p()
     st = C.lib().sptrsv_analyse(n, nnz, _ptr(rp), _ptr(ci), _ptr(val), code, C.LOWER if fill == "L" else C.UPPER,
                                 ctypes.byref(o), _stream_handle(stream), ctypes.byref(h))
     C.check(st, "sptrsv_analyse")
-    return Plan(h.value, n, code)
+    return Plan(h.value, n, code, device=o.device)
 
 
 analyse = sptrsv_analyse
@@ -249,6 +286,14 @@ def sptrsv_solve(plan: Plan, b, x=None, stream=None):
     n = plan.n
     if b.shape[0] != n:
         raise ValueError(f"b has {b.shape[0]} rows, plan has n={n}")
+    # the C ABI carries no dtype: b and x must hold the plan's value type
+    # (a float32 x under a float64 plan would be written past its end)
+    for name, t in (("b", b), ("x", x)):
+        if t is not None and _dtype_code(t) != plan.dtype_code:
+            raise TypeError(f"{name} is {t.dtype}, the plan was analysed for "
+                            f"{'float64' if plan.dtype_code == C.R64F else 'float32'}")
+        if t is not None and _is_torch(t) and t.is_cuda and plan.device >= 0 and t.device.index != plan.device:
+            raise ValueError(f"{name} is on cuda:{t.device.index}, the plan on cuda:{plan.device}")
     if _is_torch(b):
         import torch
         if _layout(b, n) is None:

@@ -32,12 +32,17 @@ EXPORTS = ["sptrsv_opts_default", "sptrsv_analyse", "sptrsv_solve", "sptrsv_free
            "sptrsv_last_error", "sptrsv_version"]
 
 
+DEV_ALLOC = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+DEV_FREE = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
+
+
 class Opts(ctypes.Structure):
     _fields_ = [("variant", ctypes.c_int32), ("depth", ctypes.c_int32), ("min_block_rows", ctypes.c_int64),
                 ("reorder", ctypes.c_int32), ("selector", ctypes.c_int32), ("force_tri_impl", ctypes.c_int32),
                 ("force_sq_impl", ctypes.c_int32), ("host_only", ctypes.c_int32), ("sm_count", ctypes.c_int32),
                 ("threads", ctypes.c_int32), ("device", ctypes.c_int32), ("transpose", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 7)]
+                ("max_nrhs", ctypes.c_int32), ("graphs", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5),
+                ("dev_alloc", DEV_ALLOC), ("dev_free", DEV_FREE), ("alloc_ctx", ctypes.c_void_p)]
 
 
 class PlanInfo(ctypes.Structure):

@@ -48,6 +48,11 @@ SPTRSV_EXPORT void sptrsv_opts_default(sptrsv_opts_t* o) {
   o->sm_count = 0;
   o->threads = 0;
   o->device = -1;
+  o->max_nrhs = 0;
+  o->graphs = 1;
+  o->dev_alloc = nullptr;
+  o->dev_free = nullptr;
+  o->alloc_ctx = nullptr;
 }
 
 static bool host_copy_if_device(const void* src, size_t bytes, std::vector<char>& dst, const void** out,
@@ -91,6 +96,9 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_analyse(int32_t n, int64_t nnz, const int32
   if (o.selector < 0 || o.selector > 1) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad selector");
   if (o.min_block_rows < 0) return fail(SPTRSV_ERROR_INVALID_VALUE, "min_block_rows < 0");
   if (o.transpose < 0 || o.transpose > 1) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad transpose");
+  if (o.max_nrhs < 0) return fail(SPTRSV_ERROR_INVALID_VALUE, "max_nrhs < 0");
+  if ((o.dev_alloc == nullptr) != (o.dev_free == nullptr))
+    return fail(SPTRSV_ERROR_INVALID_VALUE, "dev_alloc and dev_free must be given together");
 
   sptrsv_plan_s* P = new (std::nothrow) sptrsv_plan_s();
   if (!P) return fail(SPTRSV_ERROR_ALLOC, "host allocation failed");

@@ -24,9 +24,48 @@ namespace sptrsv {
       return Error{SPTRSV_ERROR_CUDA, std::string(#x) + ": " + cudaGetErrorString(e_)}; \
   } while (0)
 
+// Device memory of a plan: through the caller's hooks (the Python binding
+// passes torch's caching allocator) or cudaMalloc / cudaFree.
+void* dalloc(Plan& p, size_t bytes, cudaStream_t s) {
+  if (p.opts.dev_alloc) return p.opts.dev_alloc(bytes, (void*)s, p.opts.alloc_ctx);
+  void* q = nullptr;
+  if (cudaMalloc(&q, bytes) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return q;
+}
+void dfree(Plan& p, void* q, cudaStream_t s) {
+  if (!q) return;
+  if (p.opts.dev_free)
+    p.opts.dev_free(q, (void*)s, p.opts.alloc_ctx);
+  else
+    cudaFree(q);
+}
+
 namespace {
 
 size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+// cudaFuncSetAttribute (max dynamic shared memory, non-portable cluster size)
+// is per device: cache what was set per (kernel, device ordinal), under a
+// mutex (plans may be solved from several threads and live on several GPUs).
+std::mutex attr_mu;
+std::unordered_map<std::string, uint32_t> attr_set;
+cudaError_t ensure_smem_attr(const void* f, uint32_t smem, bool cluster) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  char key[64];
+  std::snprintf(key, sizeof(key), "%p/%d", f, dev);
+  std::lock_guard<std::mutex> g(attr_mu);
+  auto it = attr_set.find(key);
+  if (it != attr_set.end() && it->second >= smem) return cudaSuccess;
+  e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess && cluster) e = cudaFuncSetAttribute(f, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+  if (e == cudaSuccess) attr_set[key] = smem;
+  return e;
+}
 
 // Supernodal triangles with at least this many RHS run tri_supernode_multi
 // (dense per-piece tiles over 64-column chunks); fewer columns would leave
@@ -339,12 +378,7 @@ Error launch_chain_ell(Plan& p, Segment& S, const T* bw, T* xs, cudaStream_t s) 
   const uint32_t smem = NST * k::ell_stage_bytes<T>(K, RMAX, PMAX, SMAX) + k::al16((XW + 2) * (uint32_t)sizeof(T)) +
                         NST * 16;
   constexpr int RG = 2;
-  static uint32_t attr_bytes = 0;  // per template instance
-  if (smem > attr_bytes) {
-    CUDA_TRY(cudaFuncSetAttribute(k::tri_chain_ell<T, K, RG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  (int)smem));
-    attr_bytes = smem;
-  }
+  CUDA_TRY(ensure_smem_attr((const void*)k::tri_chain_ell<T, K, RG>, smem, false));
   const int nst = (int)(S.ell_recs.size() / 16);
   long long* tr = nullptr;
   if (p.trace) {
@@ -723,12 +757,7 @@ Error launch_wave_t(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, c
                 S.wave_ipl};
   const uint32_t smem = k::wave_smem_bytes<T>(g);
   auto kern = k::tri_wave<T, K, E, GPC, GLB>;
-  static uint32_t attr_bytes = 0;  // per template instance
-  if (smem > attr_bytes) {
-    CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
-    attr_bytes = smem;
-  }
+  CUDA_TRY(ensure_smem_attr((const void*)kern, smem, true));
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(S.wave_C);
   cfg.blockDim = dim3(32 * (S.wave_W + 1));  // + the TMA producer warp
@@ -876,12 +905,7 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
           } else if (nrhs == 1 && !S.chain_recs.empty()) {
             const k::ChainGeom cg = frozen_geometry(p);
             const uint32_t smem = k::chain_smem_bytes<T>(cg);
-            static uint32_t attr_bytes = 0;  // per template instance
-            if (smem > attr_bytes) {
-              CUDA_TRY(cudaFuncSetAttribute(k::tri_chain_tma<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                            (int)smem));
-              attr_bytes = smem;
-            }
+            CUDA_TRY(ensure_smem_attr((const void*)k::tri_chain_tma<T>, smem, false));
             const int nst = (int)(S.chain_recs.size() / 16);
             long long* tr = nullptr;
             if (p.trace) {  // debug: SPTRSV_TRACE=1, per-stage clock64 stamps
@@ -926,7 +950,7 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
             const int nch = (int)cdiv(nrhs, k::kSnmCols);
             for (int c = 0; c < nch; ++c) {
               k::SolveState sc = st;
-              sc.epoch = st.epoch + (uint32_t)c;
+              sc.epoch_off = (uint32_t)c;
               if (c > 0) CUDA_TRY(cudaMemsetAsync(st.tickets + S.ticket_slot, 0, 4, s));
               k::tri_supernode_multi<T><<<g, 256, 0, s>>>(np, (const k::SnDesc*)S.d_sn_desc, S.d_sn_cols,
                                                           (const T*)S.d_sn_vals, (const T*)S.d_sn_blk, bw, xs, sc,
@@ -950,7 +974,16 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
             if (const char* ev2 = std::getenv("SPTRSV_SF_CTAS")) c = std::max(1, std::atoi(ev2));
             return (unsigned)std::min<int64_t>({c, (int64_t)cap, (int64_t)cdiv(rows_total, rows_per_cta)});
           };
-          if (nrhs == 1) {
+          if (nrhs == 1 && !S.sf_items.empty()) {
+            const int nitem = (int)(S.sf_items.size() / 8);
+            static const int per_sm = [] {
+              const char* e2 = std::getenv("SPTRSV_SF_PERSM");  // tuning: resident CTAs per SM
+              return e2 ? std::max(1, std::atoi(e2)) : SPTRSV_SF_MINB;
+            }();
+            const unsigned g = std::max(1u, std::min<unsigned>(cdiv(nitem, 8), (unsigned)(per_sm * p.sm_count)));
+            k::tri_sf_items<T><<<g, 256, 0, s>>>(I.row0, nitem, (const k::SfItem*)S.d_sf_items, S.d_rp, S.d_ci, val,
+                                                 bw, xs, (T*)p.d_part, st, S.ticket_slot);
+          } else if (nrhs == 1) {
             if (tri_use_warp(S))
               k::tri_syncfree_warp<T, 8><<<std::max(1u, ctas(8, m)), 256, 0, s>>>(I.row0, m, S.d_rp, S.d_ci, val,
                                                                                   bw, xs, st, S.ticket_slot);
@@ -1023,51 +1056,76 @@ void dump_trace(Plan& p, cudaStream_t s) {
   }
 }
 
-template <typename T>
-Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs, sptrsv_layout_t layout,
-                   cudaStream_t s) {
+// Epochs one solve hands out (multi-RHS sync-free triangles poll per-row
+// flags holding the epoch of the solve that published them; the supernodal
+// SpTRSM runs one launch per 64-column chunk, each with its own epoch).
+uint32_t epoch_span(const Plan& p, int nrhs) {
+  if (nrhs <= 1 || !p.needs_flags) return 0;
+  return (uint32_t)std::max<int64_t>(1, cdiv(nrhs, k::kSnmCols));
+}
+
+void drop_graphs(Plan& p) {
+  for (auto& g : p.graphs)
+    if (g.exec) cudaGraphExecDestroy((cudaGraphExec_t)g.exec);
+  p.graphs.clear();
+  p.pending = GraphEntry{};
+}
+
+// Everything a solve of nrhs columns needs that is not a kernel launch:
+// workspace, flags, epoch wrap.  Runs before (never inside) a graph capture.
+Error prepare_solve(Plan& p, int nrhs, cudaStream_t s) {
   const int n = p.n;
-  size_t need = (size_t)n * nrhs * sizeof(T);
+  const size_t need = (size_t)n * nrhs * p.vbytes;
   if (need > p.ws.w_bytes) {
-    if (p.ws.bw) cudaFree(p.ws.bw);
-    if (p.ws.xs) cudaFree(p.ws.xs);
+    drop_graphs(p);  // captured solves reference the old workspace
+    dfree(p, p.ws.bw, s);
+    dfree(p, p.ws.xs, s);
     p.ws.bw = p.ws.xs = nullptr;
     p.ws.w_bytes = 0;
     // +256 B: the staged chain kernel's 16-byte-aligned TMA windows may read
     // up to 15 bytes past the last row
-    if (cudaMalloc(&p.ws.bw, need + 256) != cudaSuccess || cudaMalloc(&p.ws.xs, need + 256) != cudaSuccess) {
-      cudaGetLastError();
-      return {SPTRSV_ERROR_ALLOC, "workspace allocation failed"};
-    }
+    p.ws.bw = dalloc(p, need + 256, s);
+    p.ws.xs = dalloc(p, need + 256, s);
+    if (!p.ws.bw || !p.ws.xs) return {SPTRSV_ERROR_ALLOC, "workspace allocation failed"};
     p.ws.w_bytes = need;
   }
+  const uint32_t span = epoch_span(p, nrhs);
+  if (span) {
+    if (!p.ws.flags) {
+      drop_graphs(p);
+      p.ws.flags_n = std::max(1, n);
+      p.ws.flags = dalloc(p, (size_t)p.ws.flags_n * 4, s);
+      if (!p.ws.flags) return {SPTRSV_ERROR_ALLOC, "flag workspace allocation failed"};
+      CUDA_TRY(cudaMemsetAsync(p.ws.flags, 0, (size_t)p.ws.flags_n * 4, s));
+      CUDA_TRY(cudaMemsetAsync(p.d_epoch, 0, 8, s));
+      p.epoch = 0;
+    }
+    // the device counter is mirrored here: about to wrap -> restart from
+    // clean flags (stream-ordered, before the solve that would wrap)
+    if (p.epoch > 0xFFFFFFFFu - span - 1u) {
+      CUDA_TRY(cudaMemsetAsync(p.ws.flags, 0, (size_t)p.ws.flags_n * 4, s));
+      CUDA_TRY(cudaMemsetAsync(p.d_epoch, 0, 8, s));
+      p.epoch = 0;
+    }
+    p.epoch += span;
+  }
+  return {SPTRSV_SUCCESS, ""};
+}
+
+// The kernels of one solve (permute-in, Alg 7's segment loop, permute-out)
+// enqueued on s; no allocation, no host synchronisation (capturable).
+template <typename T>
+Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs, sptrsv_layout_t layout,
+                   cudaStream_t s) {
+  const int n = p.n;
   T* bw = (T*)p.ws.bw;
   T* xs = (T*)p.ws.xs;
   const T* rd = (const T*)p.d_rdiag;
   // nrhs == 1: sync-free rows poll their dependencies' values, which start
   // as the sentinel; nrhs > 1: they poll per-row epoch flags instead
   const int fill = (p.needs_sentinel && nrhs == 1) ? 1 : 0;
-  uint32_t epoch = 0;
-  if (nrhs > 1 && p.needs_flags) {
-    if (!p.ws.flags) {
-      if (cudaMalloc(&p.ws.flags, (size_t)std::max(1, n) * 4) != cudaSuccess) {
-        cudaGetLastError();
-        return {SPTRSV_ERROR_ALLOC, "flag workspace allocation failed"};
-      }
-      CUDA_TRY(cudaMemsetAsync(p.ws.flags, 0, (size_t)std::max(1, n) * 4, s));
-      p.epoch = 0;
-    }
-    // a solve owns epochs [base, base + span): the supernodal SpTRSM runs
-    // one launch per 64-column chunk, each with its own epoch (exec: kSnmSplit)
-    const uint32_t span = (uint32_t)std::max<int64_t>(1, cdiv(nrhs, k::kSnmCols));
-    if (p.epoch > 0xFFFFFFFFu - span - 1u) {  // about to wrap: restart from clean flags
-      CUDA_TRY(cudaMemsetAsync(p.ws.flags, 0, (size_t)std::max(1, n) * 4, s));
-      p.epoch = 0;
-    }
-    epoch = p.epoch + 1;
-    p.epoch += span;
-  }
-  k::SolveState st{p.d_tickets, p.nticket, p.d_error, (uint32_t*)p.ws.flags, epoch, p.backoff_ns};
+  k::SolveState st{p.d_tickets,         p.nticket,    p.d_error, (uint32_t*)p.ws.flags, p.d_epoch, 0u,
+                   epoch_span(p, nrhs), p.backoff_ns, p.d_derr,  p.wd_spins, (unsigned long long*)p.d_sf_trace};
   cudaEvent_t* ev = nullptr;
   if (p.profiling) {
     size_t need_ev = p.segs.size() + 3;
@@ -1082,7 +1140,8 @@ Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs
   const int* iperm = p.d_perm + n;  // old -> new, stored right after perm
   if (nrhs == 1) {
     int64_t stride = layout == SPTRSV_ROW_MAJOR ? ldb : 1;
-    k::perm_in_1<T><<<std::max(1u, cdiv(n, 256)), 256, 0, s>>>(n, p.d_perm, rd, b, stride, bw, xs, fill, st);
+    k::perm_in_1<T><<<std::max(1u, cdiv(std::max(n, p.npart), 256)), 256, 0, s>>>(n, p.d_perm, rd, b, stride, bw, xs,
+                                                                                  fill, st, (T*)p.d_part, p.npart);
   } else if (layout == SPTRSV_COL_MAJOR) {
     k::perm_in_cm<T><<<std::max(1u, cdiv(n, 32)), 256, 0, s>>>(n, nrhs, iperm, rd, b, ldb, bw, xs, fill, st);
   } else {
@@ -1108,16 +1167,39 @@ Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs
     p.last_nseg_timed = (int)p.segs.size();
   }
   if (p.trace) dump_trace(p, s);
+  if (p.d_sf_trace) {  // debug: the last solve's per-row stamps -> $SPTRSV_SF_TRACE/sf_trace.bin
+    cudaStreamSynchronize(s);
+    std::vector<unsigned long long> h((size_t)n * 2);
+    cudaMemcpy(h.data(), p.d_sf_trace, h.size() * 8, cudaMemcpyDeviceToHost);
+    std::string path = std::string(std::getenv("SPTRSV_SF_TRACE")) + "/sf_trace.bin";
+    if (FILE* f = std::fopen(path.c_str(), "wb")) {
+      std::fwrite(h.data(), 8, h.size(), f);
+      std::fclose(f);
+    }
+    cudaMemsetAsync(p.d_sf_trace, 0, h.size() * 8, s);
+  }
   return {SPTRSV_SUCCESS, ""};
 }
 
-bool is_device_ptr(const void* ptr) {
+// prepare + enqueue (the host-pointer paths)
+Error solve_device_any(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int nrhs, sptrsv_layout_t layout,
+                       cudaStream_t s) {
+  Error e = prepare_solve(p, nrhs, s);
+  if (e.status) return e;
+  return p.dtype == SPTRSV_R64F
+             ? solve_device<double>(p, (const double*)b, ldb, (double*)x, ldx, nrhs, layout, s)
+             : solve_device<float>(p, (const float*)b, ldb, (float*)x, ldx, nrhs, layout, s);
+}
+
+// memory type (0 host / unregistered, 1 device or managed) and device ordinal
+int ptr_kind(const void* ptr, int* device) {
   cudaPointerAttributes a;
   if (cudaPointerGetAttributes(&a, ptr) != cudaSuccess) {
     cudaGetLastError();
-    return false;
+    return 0;
   }
-  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+  *device = a.device;
+  return (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) ? 1 : 0;
 }
 
 }  // namespace
@@ -1158,6 +1240,48 @@ void build_sq_items(Segment& S) {
       ++t;
     }
     push(start, t, rp[start], rp[t], false);
+  }
+}
+
+// Work items of the row-block sync-free kernel (k::tri_sf_items): greedy
+// runs of <= 32 consecutive rows holding <= kSfNB off-diagonal entries; a
+// longer row is cut into kSfNB-entry pieces (kind 1, each with a partial-sum
+// slot out of the plan's `part` array) closed by its last piece (kind 2),
+// which adds the earlier pieces' partial sums.  SPTRSV_SF_V1 keeps the
+// round-1 kernels (thread / warp per row).
+void build_sf_items(Segment& S, int32_t& part_base) {
+  S.sf_items.clear();
+  const auto& I = S.info;
+  if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_SYNCFREE || !std::getenv("SPTRSV_SF_ITEMS")) return;
+  const int m = I.row1 - I.row0;
+  const std::vector<int32_t>& rp = S.rp;
+  auto push = [&](int t0, int t1, int p0, int p1, int kind, int s0, int s1) {
+    const int32_t rec[8] = {t0, t1, p0, p1, kind, s0, s1, 0};
+    S.sf_items.insert(S.sf_items.end(), rec, rec + 8);
+  };
+  int t = 0;
+  while (t < m) {
+    const int len = rp[t + 1] - rp[t];
+    if (len > k::kSfNB) {
+      const int np = (len + k::kSfNB - 1) / k::kSfNB;
+      const int first = part_base;
+      for (int q = 0; q < np; ++q) {
+        const int a = rp[t] + q * k::kSfNB, b = std::min(a + k::kSfNB, rp[t + 1]);
+        if (q < np - 1)
+          push(t, t + 1, a, b, 1, part_base++, 0);
+        else
+          push(t, t + 1, a, b, 2, first, part_base);
+      }
+      ++t;
+      continue;
+    }
+    const int start = t;
+    int tot = 0;
+    while (t < m && t - start < 32 && tot + (rp[t + 1] - rp[t]) <= k::kSfNB) {
+      tot += rp[t + 1] - rp[t];
+      ++t;
+    }
+    push(start, t, rp[start], rp[t], 0, 0, 0);
   }
 }
 
@@ -1248,16 +1372,22 @@ Error upload(Plan& p, void* stream_v) {
   };
   size_t o_perm = take((size_t)2 * n * 4);  // perm (new->old) then iperm (old->new)
   size_t o_rdiag = take((size_t)n * vb);
-  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed, sd, sc, sv, sbk, ps, pd, pc, sq; };
+  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed, sd, sc, sv, sbk, ps, pd, pc, sq, sf; };
   std::vector<Offs> so(p.segs.size());
   p.trace = std::getenv("SPTRSV_TRACE") != nullptr;
   p.spmm = spmm_cfg();
   p.backoff_ns = 128;
   if (const char* e = std::getenv("SPTRSV_SF_BACKOFF")) p.backoff_ns = (uint32_t)std::max(0, std::atoi(e));
+  p.wd_spins = k::kWatchdogSpins;
+  if (std::getenv("SPTRSV_SF_TRACE") && !p.d_sf_trace)  // debug: per-row claim/done stamps (SF_TRACE builds)
+    if (cudaMalloc(&p.d_sf_trace, (size_t)std::max(1, n) * 16) != cudaSuccess) p.d_sf_trace = nullptr;
+  if (const char* e = std::getenv("SPTRSV_WATCHDOG_SPINS"))  // tests: trip the watchdog quickly
+    p.wd_spins = (uint32_t)std::max(1024, std::atoi(e));
   const k::ChainGeom cg = chain_geometry(p);
   p.chain_geom[0] = cg.NST; p.chain_geom[1] = cg.RMAX; p.chain_geom[2] = cg.EMAX;
   p.chain_geom[3] = cg.XW; p.chain_geom[4] = cg.LMAX;
   p.nticket = 0;
+  p.npart = 0;
   p.needs_sentinel = false;
   p.needs_flags = false;
   for (size_t i = 0; i < p.segs.size(); ++i) build_wave(p, p.segs[i], vb);  // may switch a segment to CHAIN
@@ -1346,6 +1476,7 @@ Error upload(Plan& p, void* stream_v) {
     build_chain_ell(S, vb);
     build_supernodes(S, vb);
     build_sq_items(S);
+    build_sf_items(S, p.npart);
     so[i].er = take(S.ell_recs.size() * 4);
     so[i].ed = take(S.ell_data.size());
     so[i].rp = take(dv[i].nrp * 4);
@@ -1362,6 +1493,7 @@ Error upload(Plan& p, void* stream_v) {
     so[i].pd = take(S.wave_data.size());
     so[i].pc = take(S.wave_crows.size() * 4);
     so[i].sq = take(S.sq_items.size() * 4);
+    so[i].sf = take(S.sf_items.size() * 4);
     if (S.info.kind == 0) S.ticket_slot = p.nticket++;
     if (S.info.kind == 0 && (S.info.impl == SPTRSV_IMPL_TRI_SYNCFREE || S.info.impl == SPTRSV_IMPL_TRI_SUPERNODE ||
                              (S.info.impl == SPTRSV_IMPL_TRI_PIPE && (S.wave_K == 0 || S.wave_global > 0))))
@@ -1371,16 +1503,16 @@ Error upload(Plan& p, void* stream_v) {
       p.needs_flags = true;
   }
   size_t o_tickets = take((size_t)std::max(1, p.nticket) * 4);
+  size_t o_ctl = take(16);  // {watchdog word, pad, epoch base, last epoch}
+  size_t o_part = take((size_t)std::max(1, p.npart) * vb);
   p.arena_bytes = off;
   clk.lap("upload: chain/ell/supernode");
 
   int dev;
   CUDA_TRY(cudaGetDevice(&dev));
   p.device = dev;
-  if (cudaMalloc(&p.arena, std::max<size_t>(off, 256)) != cudaSuccess) {
-    cudaGetLastError();
-    return {SPTRSV_ERROR_ALLOC, "plan arena allocation failed (" + std::to_string(off) + " bytes)"};
-  }
+  p.arena = dalloc(p, std::max<size_t>(off, 256), s);
+  if (!p.arena) return {SPTRSV_ERROR_ALLOC, "plan arena allocation failed (" + std::to_string(off) + " bytes)"};
   clk.lap("upload: cudaMalloc");
   // perm / iperm / 1/d are composed on the host (sigma), every segment array
   // is copied straight from its host vector (no staging image of the arena)
@@ -1444,10 +1576,32 @@ Error upload(Plan& p, void* stream_v) {
     S.d_wave_crows = (const int32_t*)(A + so[i].pc);
     CUDA_TRY(put(so[i].sq, S.sq_items.data(), S.sq_items.size() * 4));
     S.d_sq_items = (const int32_t*)(A + so[i].sq);
+    CUDA_TRY(put(so[i].sf, S.sf_items.data(), S.sf_items.size() * 4));
+    S.d_sf_items = (const int32_t*)(A + so[i].sf);
+  }
+  if (std::getenv("SPTRSV_TEST_WEDGE")) {
+    // test hook (DEADLOCK path): the first off-diagonal entry of the first
+    // sync-free triangle points at its own row, which then never becomes ready
+    for (size_t i = 0; i < p.segs.size(); ++i) {
+      Segment& S = p.segs[i];
+      if (S.info.kind != 0 || S.info.impl != SPTRSV_IMPL_TRI_SYNCFREE || S.ci.empty()) continue;
+      const int m = S.info.row1 - S.info.row0;
+      for (int r = 0; r < m; ++r)
+        if (S.rp[r + 1] > S.rp[r]) {
+          const int32_t self = S.info.row0 + r;
+          CUDA_TRY(cudaMemcpyAsync(A + so[i].ci + (size_t)S.rp[r] * 4, &self, 4, cudaMemcpyHostToDevice, s));
+          CUDA_TRY(cudaStreamSynchronize(s));
+          break;
+        }
+      break;
+    }
   }
   p.d_perm = (const int32_t*)(A + o_perm);
   p.d_rdiag = (const void*)(A + o_rdiag);
   p.d_tickets = (uint32_t*)(A + o_tickets);
+  p.d_derr = (int32_t*)(A + o_ctl);
+  p.d_epoch = (uint32_t*)(A + o_ctl + 8);
+  p.d_part = (void*)(A + o_part);
   clk.lap("upload: H2D copies issued");
   // mapped host word for the spin-wait watchdog, from a process-wide pool
   // (cudaHostAlloc costs milliseconds per call)
@@ -1456,6 +1610,11 @@ Error upload(Plan& p, void* stream_v) {
     p.d_error = nullptr;
   } else {
     *p.h_error = 0;
+  }
+  if (p.opts.max_nrhs > 0) {  // size the solve workspace now (no allocation at solve time)
+    Error e = prepare_solve(p, p.opts.max_nrhs, s);
+    if (e.status) return e;
+    p.epoch = 0;  // prepare_solve counted a solve that did not happen
   }
   CUDA_TRY(cudaStreamSynchronize(s));
   clk.lap("upload: H2D complete");
@@ -1476,15 +1635,14 @@ Error solve_host_pipelined(Plan& p, const void* b, int64_t ldb, void* x, int64_t
   const int cb = (nrhs + nblk - 1) / nblk;
   const size_t blk_bytes = (size_t)p.n * cb * vb;
   if (2 * blk_bytes > p.ws.stage_bytes) {
-    if (p.ws.stage_b) cudaFree(p.ws.stage_b);
-    if (p.ws.stage_x) cudaFree(p.ws.stage_x);
+    CUDA_TRY(cudaStreamSynchronize(s));  // the old staging may still be in use
+    dfree(p, p.ws.stage_b, s);
+    dfree(p, p.ws.stage_x, s);
     p.ws.stage_b = p.ws.stage_x = nullptr;
     p.ws.stage_bytes = 0;
-    if (cudaMalloc(&p.ws.stage_b, 2 * blk_bytes) != cudaSuccess ||
-        cudaMalloc(&p.ws.stage_x, 2 * blk_bytes) != cudaSuccess) {
-      cudaGetLastError();
-      return {SPTRSV_ERROR_ALLOC, "staging allocation failed"};
-    }
+    p.ws.stage_b = dalloc(p, 2 * blk_bytes, s);
+    p.ws.stage_x = dalloc(p, 2 * blk_bytes, s);
+    if (!p.ws.stage_b || !p.ws.stage_x) return {SPTRSV_ERROR_ALLOC, "staging allocation failed"};
     p.ws.stage_bytes = 2 * blk_bytes;
   }
   if (!p.ws.h2d) {
@@ -1519,9 +1677,7 @@ Error solve_host_pipelined(Plan& p, const void* b, int64_t ldb, void* x, int64_t
     // solve: needs block k in, and stage_x[u] drained by block k-2's copy out
     CUDA_TRY(cudaStreamWaitEvent(s, ev[u], 0));
     CUDA_TRY(cudaStreamWaitEvent(s, ev[4 + u], 0));
-    Error e = p.dtype == SPTRSV_R64F
-                  ? solve_device<double>(p, (const double*)sb, p.n, (double*)sx, p.n, nc, SPTRSV_COL_MAJOR, s)
-                  : solve_device<float>(p, (const float*)sb, p.n, (float*)sx, p.n, nc, SPTRSV_COL_MAJOR, s);
+    Error e = solve_device_any(p, sb, p.n, sx, p.n, nc, SPTRSV_COL_MAJOR, s);
     if (e.status) return e;
     CUDA_TRY(cudaEventRecord(ev[2 + u], s));
     // out
@@ -1532,83 +1688,187 @@ Error solve_host_pipelined(Plan& p, const void* b, int64_t ldb, void* x, int64_t
   }
   CUDA_TRY(cudaStreamSynchronize(d2h));
   CUDA_TRY(cudaStreamSynchronize(s));
-  if (p.h_error && *(volatile int32_t*)p.h_error) {
-    *(volatile int32_t*)p.h_error = 0;
-    return {SPTRSV_ERROR_DEADLOCK, "spin-wait watchdog tripped"};
+  return {SPTRSV_SUCCESS, ""};
+}
+
+// A trip of the spin-wait watchdog during an earlier solve: report it once
+// and re-arm (host mapped word and its device copy).
+bool take_deadlock(Plan& p, cudaStream_t s) {
+  if (!(p.h_error && *(volatile int32_t*)p.h_error)) return false;
+  *(volatile int32_t*)p.h_error = 0;
+  if (p.d_derr) cudaMemsetAsync(p.d_derr, 0, 4, s);
+  return true;
+}
+
+Error record_done(Plan& p, cudaStream_t s) {
+  if (!p.done_ev) {
+    cudaEvent_t e;
+    CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    p.done_ev = (void*)e;
   }
+  CUDA_TRY(cudaEventRecord((cudaEvent_t)p.done_ev, s));
+  p.done_ev_recorded = true;
+  return {SPTRSV_SUCCESS, ""};
+}
+
+// Device solve with CUDA-graph reuse (opts.graphs): a key (b, x, ld, nrhs,
+// layout) seen twice in a row is captured -- on the plan's private capture
+// stream, so the caller's stream may be the legacy default stream -- and
+// every later solve with a captured key is one cudaGraphLaunch.
+Error solve_device_graphed(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t nrhs,
+                           sptrsv_layout_t layout, cudaStream_t s) {
+  Error e = prepare_solve(p, nrhs, s);
+  if (e.status) return e;
+  auto eager = [&]() {
+    return p.dtype == SPTRSV_R64F
+               ? solve_device<double>(p, (const double*)b, ldb, (double*)x, ldx, nrhs, layout, s)
+               : solve_device<float>(p, (const float*)b, ldb, (float*)x, ldx, nrhs, layout, s);
+  };
+  bool use_graph = p.opts.graphs != 0 && !p.profiling && !p.trace && !p.d_sf_trace;
+  if (use_graph) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    CUDA_TRY(cudaStreamIsCapturing(s, &cs));
+    if (cs != cudaStreamCaptureStatusNone) use_graph = false;  // inside the caller's own capture
+  }
+  if (!use_graph) return eager();
+  ++p.solve_count;
+  auto same = [&](const GraphEntry& g) {
+    return g.b == b && g.x == x && g.ldb == ldb && g.ldx == ldx && g.nrhs == nrhs && g.layout == (int)layout;
+  };
+  for (auto& g : p.graphs)
+    if (same(g)) {
+      g.last_use = p.solve_count;
+      CUDA_TRY(cudaGraphLaunch((cudaGraphExec_t)g.exec, s));
+      return {SPTRSV_SUCCESS, ""};
+    }
+  if (!same(p.pending)) {  // first sighting: run eagerly, remember the key
+    p.pending = GraphEntry{b, x, ldb, ldx, nrhs, (int)layout, nullptr, 0};
+    return eager();
+  }
+  // second sighting in a row: capture
+  if (!p.capture_stream) {
+    cudaStream_t c;
+    CUDA_TRY(cudaStreamCreateWithFlags(&c, cudaStreamNonBlocking));
+    p.capture_stream = (void*)c;
+  }
+  cudaStream_t cs = (cudaStream_t)p.capture_stream;
+  CUDA_TRY(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
+  Error ce = p.dtype == SPTRSV_R64F
+                 ? solve_device<double>(p, (const double*)b, ldb, (double*)x, ldx, nrhs, layout, cs)
+                 : solve_device<float>(p, (const float*)b, ldb, (float*)x, ldx, nrhs, layout, cs);
+  cudaGraph_t graph = nullptr;
+  cudaError_t ee = cudaStreamEndCapture(cs, &graph);
+  if (ce.status || ee != cudaSuccess || !graph) {
+    if (graph) cudaGraphDestroy(graph);
+    cudaGetLastError();
+    p.pending = GraphEntry{};
+    if (ce.status) return ce;
+    return eager();  // capture not possible here: plain launches
+  }
+  cudaGraphExec_t exec = nullptr;
+  ee = cudaGraphInstantiate(&exec, graph, 0);
+  cudaGraphDestroy(graph);
+  if (ee != cudaSuccess) {
+    cudaGetLastError();
+    p.pending = GraphEntry{};
+    return eager();
+  }
+  if (p.graphs.size() >= 8) {  // evict the least recently used
+    auto lru = std::min_element(p.graphs.begin(), p.graphs.end(),
+                                [](const GraphEntry& a2, const GraphEntry& b2) { return a2.last_use < b2.last_use; });
+    cudaGraphExecDestroy((cudaGraphExec_t)lru->exec);
+    p.graphs.erase(lru);
+  }
+  GraphEntry g = p.pending;
+  g.exec = (void*)exec;
+  g.last_use = p.solve_count;
+  p.graphs.push_back(g);
+  p.pending = GraphEntry{};
+  CUDA_TRY(cudaGraphLaunch(exec, s));
   return {SPTRSV_SUCCESS, ""};
 }
 
 Error solve(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t nrhs, sptrsv_layout_t layout,
             void* stream_v) {
   cudaStream_t s = (cudaStream_t)stream_v;
-  if (p.h_error && *(volatile int32_t*)p.h_error) {
-    *(volatile int32_t*)p.h_error = 0;
-    return {SPTRSV_ERROR_DEADLOCK, "a spin-wait watchdog tripped during an earlier solve on this plan"};
-  }
-  if (nrhs == 0 || p.n == 0) return {SPTRSV_SUCCESS, ""};
   // the plan is bound to its device (our runtime's current device is not
   // torch's: make it explicit on every call)
   int cur = -1;
   if (cudaGetDevice(&cur) != cudaSuccess || cur != p.device) CUDA_TRY(cudaSetDevice(p.device));
-  bool bd = is_device_ptr(b), xd = is_device_ptr(x);
+  if (take_deadlock(p, s))
+    return {SPTRSV_ERROR_DEADLOCK, "a spin-wait watchdog tripped during an earlier solve on this plan"};
+  if (nrhs == 0 || p.n == 0) return {SPTRSV_SUCCESS, ""};
+  int bdev = -1, xdev = -1;
+  const int bd = ptr_kind(b, &bdev), xd = ptr_kind(x, &xdev);
   if (bd != xd) return {SPTRSV_ERROR_INVALID_VALUE, "b and x must both be device or both be host pointers"};
   const size_t vb = p.vbytes;
   if (bd) {
-    if (p.dtype == SPTRSV_R64F)
-      return solve_device<double>(p, (const double*)b, ldb, (double*)x, ldx, nrhs, layout, s);
-    return solve_device<float>(p, (const float*)b, ldb, (float*)x, ldx, nrhs, layout, s);
+    if (bdev != p.device || xdev != p.device)
+      return {SPTRSV_ERROR_INVALID_VALUE, "b / x live on device " + std::to_string(bdev) + " / " +
+                                              std::to_string(xdev) + ", the plan on device " +
+                                              std::to_string(p.device)};
+    Error e = solve_device_graphed(p, b, ldb, x, ldx, nrhs, layout, s);
+    if (e.status) return e;
+    return record_done(p, s);
   }
+  Error out{SPTRSV_SUCCESS, ""};
   // host buffers, many column-major RHS: pipelined by column blocks
-  if (layout == SPTRSV_COL_MAJOR && nrhs >= 32 && std::getenv("SPTRSV_NO_PIPELINE") == nullptr)
-    return solve_host_pipelined(p, b, ldb, x, ldx, nrhs, s);
-  // host buffers: stage through the device (end-to-end path), then sync
-  size_t need = (size_t)p.n * nrhs * vb;
-  if (need > p.ws.stage_bytes) {
-    if (p.ws.stage_b) cudaFree(p.ws.stage_b);
-    if (p.ws.stage_x) cudaFree(p.ws.stage_x);
-    p.ws.stage_b = p.ws.stage_x = nullptr;
-    p.ws.stage_bytes = 0;
-    if (cudaMalloc(&p.ws.stage_b, need) != cudaSuccess || cudaMalloc(&p.ws.stage_x, need) != cudaSuccess) {
-      cudaGetLastError();
-      return {SPTRSV_ERROR_ALLOC, "staging allocation failed"};
-    }
-    p.ws.stage_bytes = need;
-  }
-  // compact copies: col-major n x nrhs (ld n) or row-major n x nrhs (ld nrhs)
-  size_t width, height;
-  int64_t dld;
-  if (layout == SPTRSV_COL_MAJOR) {
-    width = (size_t)p.n * vb;
-    height = nrhs;
-    dld = p.n;
+  if (layout == SPTRSV_COL_MAJOR && nrhs >= 32 && std::getenv("SPTRSV_NO_PIPELINE") == nullptr) {
+    out = solve_host_pipelined(p, b, ldb, x, ldx, nrhs, s);
   } else {
-    width = (size_t)nrhs * vb;
-    height = p.n;
-    dld = nrhs;
+    // host buffers: stage through the device (end-to-end path), then sync
+    size_t need = (size_t)p.n * nrhs * vb;
+    if (need > p.ws.stage_bytes) {
+      CUDA_TRY(cudaStreamSynchronize(s));
+      dfree(p, p.ws.stage_b, s);
+      dfree(p, p.ws.stage_x, s);
+      p.ws.stage_b = p.ws.stage_x = nullptr;
+      p.ws.stage_bytes = 0;
+      p.ws.stage_b = dalloc(p, need, s);
+      p.ws.stage_x = dalloc(p, need, s);
+      if (!p.ws.stage_b || !p.ws.stage_x) return {SPTRSV_ERROR_ALLOC, "staging allocation failed"};
+      p.ws.stage_bytes = need;
+    }
+    // compact copies: col-major n x nrhs (ld n) or row-major n x nrhs (ld nrhs)
+    size_t width, height;
+    int64_t dld;
+    if (layout == SPTRSV_COL_MAJOR) {
+      width = (size_t)p.n * vb;
+      height = nrhs;
+      dld = p.n;
+    } else {
+      width = (size_t)nrhs * vb;
+      height = p.n;
+      dld = nrhs;
+    }
+    CUDA_TRY(cudaMemcpy2DAsync(p.ws.stage_b, width, b, (size_t)ldb * vb, width, height, cudaMemcpyHostToDevice, s));
+    Error e = solve_device_any(p, p.ws.stage_b, dld, p.ws.stage_x, dld, nrhs, layout, s);
+    if (e.status) return e;
+    CUDA_TRY(cudaMemcpy2DAsync(x, (size_t)ldx * vb, p.ws.stage_x, width, width, height, cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
   }
-  CUDA_TRY(cudaMemcpy2DAsync(p.ws.stage_b, width, b, (size_t)ldb * vb, width, height, cudaMemcpyHostToDevice, s));
-  Error e = p.dtype == SPTRSV_R64F
-                ? solve_device<double>(p, (const double*)p.ws.stage_b, dld, (double*)p.ws.stage_x, dld, nrhs, layout, s)
-                : solve_device<float>(p, (const float*)p.ws.stage_b, dld, (float*)p.ws.stage_x, dld, nrhs, layout, s);
+  if (out.status) return out;
+  Error e = record_done(p, s);
   if (e.status) return e;
-  CUDA_TRY(cudaMemcpy2DAsync(x, (size_t)ldx * vb, p.ws.stage_x, width, width, height, cudaMemcpyDeviceToHost, s));
-  CUDA_TRY(cudaStreamSynchronize(s));
-  if (p.h_error && *(volatile int32_t*)p.h_error) {
-    *(volatile int32_t*)p.h_error = 0;
-    return {SPTRSV_ERROR_DEADLOCK, "spin-wait watchdog tripped"};
-  }
+  if (take_deadlock(p, s)) return {SPTRSV_ERROR_DEADLOCK, "spin-wait watchdog tripped"};
   return {SPTRSV_SUCCESS, ""};
 }
 
 void release(Plan& p) {
-  if (p.device >= 0) cudaDeviceSynchronize();
-  if (p.arena) cudaFree(p.arena);
-  if (p.ws.bw) cudaFree(p.ws.bw);
-  if (p.ws.xs) cudaFree(p.ws.xs);
-  if (p.ws.stage_b) cudaFree(p.ws.stage_b);
-  if (p.ws.stage_x) cudaFree(p.ws.stage_x);
-  if (p.ws.flags) cudaFree(p.ws.flags);
+  if (p.device >= 0) {
+    cudaSetDevice(p.device);
+    // wait for this plan's last solve only (not the whole device)
+    if (p.done_ev && p.done_ev_recorded) cudaEventSynchronize((cudaEvent_t)p.done_ev);
+  }
+  drop_graphs(p);
+  if (p.capture_stream) cudaStreamDestroy((cudaStream_t)p.capture_stream);
+  if (p.done_ev) cudaEventDestroy((cudaEvent_t)p.done_ev);
+  dfree(p, p.arena, nullptr);
+  dfree(p, p.ws.bw, nullptr);
+  dfree(p, p.ws.xs, nullptr);
+  dfree(p, p.ws.stage_b, nullptr);
+  dfree(p, p.ws.stage_x, nullptr);
+  dfree(p, p.ws.flags, nullptr);
   if (p.ws.h2d) cudaStreamDestroy((cudaStream_t)p.ws.h2d);
   if (p.ws.d2h) cudaStreamDestroy((cudaStream_t)p.ws.d2h);
   for (void* e : p.ws.ev)
@@ -1616,11 +1876,15 @@ void release(Plan& p) {
   if (p.h_error) watchdog_word_release(p.h_error);
   for (auto& S : p.segs)
     if (S.d_trace) cudaFree(S.d_trace);
+  if (p.d_sf_trace) cudaFree(p.d_sf_trace);
+  p.d_sf_trace = nullptr;
   for (void* e : p.events) cudaEventDestroy((cudaEvent_t)e);
   p.arena = nullptr;
   p.ws = Workspace{};
   p.h_error = nullptr;
   p.events.clear();
+  p.capture_stream = nullptr;
+  p.done_ev = nullptr;
 }
 
 // seg times helper used by the C ABI

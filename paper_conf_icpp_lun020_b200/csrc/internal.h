@@ -126,6 +126,9 @@ struct Segment {
   // wave triangle is uploaded as DCSR with explicit (execution-order) rows
   bool dev_dcsr = false;
   int32_t dev_nzr = 0;
+  // row-block sync-free triangle kernel (k::tri_sf_items, nrhs == 1): k::SfItem[] as 8 ints
+  std::vector<int32_t> sf_items;
+  const int32_t* d_sf_items = nullptr;
   // row-block square kernel (k::sq_adapt_1, nrhs == 1): k::SqItem[] as 4 ints
   std::vector<int32_t> sq_items;
   const int32_t* d_sq_items = nullptr;
@@ -151,10 +154,22 @@ struct Workspace {
   void* stage_x = nullptr;
   size_t stage_bytes = 0;
   void* flags = nullptr;    // nrhs > 1 sync-free: per-row ready flags (n x u32), epoch-valued
+  int flags_n = 0;
   // pipelined host path (exec.cu solve_host_pipelined): copy streams + events
   void* h2d = nullptr;      // cudaStream_t
   void* d2h = nullptr;
   void* ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};  // in[2], comp[2], out[2]
+};
+
+// A captured solve (CUDA graph) for one argument set; replayed when a later
+// device solve has the same key (exec.cu solve()).
+struct GraphEntry {
+  const void* b = nullptr;
+  void* x = nullptr;
+  int64_t ldb = 0, ldx = 0;
+  int32_t nrhs = 0, layout = 0;
+  void* exec = nullptr;  // cudaGraphExec_t
+  uint64_t last_use = 0;
 };
 
 // SpMM lane geometry for nrhs > 1 (exec.cu: dispatch_multi_un)
@@ -194,6 +209,8 @@ struct Plan {
   const int32_t* d_perm = nullptr;
   const void* d_rdiag = nullptr;  // 1/d in new order (permute-in scaling)
   uint32_t* d_tickets = nullptr;  // [nticket] sync-free row-claim counters
+  void* d_part = nullptr;         // partial sums of split long rows (k::tri_sf_items), sentinel-reset per solve
+  int32_t npart = 0;
   int32_t nticket = 0;
   bool needs_sentinel = false;    // nrhs == 1: a triangle polls xs (value-as-flag)
   bool needs_flags = false;       // nrhs > 1: a sync-free triangle polls per-row epoch flags
@@ -204,7 +221,18 @@ struct Plan {
   Workspace ws;
   SpmmCfg spmm;
   uint32_t backoff_ns = 128;  // sync-free polling backoff cap
-  uint32_t epoch = 0;  // last multi-RHS solve's epoch (flags hold it when a row is solved)
+  uint32_t wd_spins = 0;      // watchdog: unsuccessful polls before SPTRSV_ERROR_DEADLOCK
+  void* d_sf_trace = nullptr; // SPTRSV_SF_TRACE: {claim, done} timestamps per row (debug)
+  uint32_t epoch = 0;  // host mirror of the device epoch counter (wrap detection only)
+  uint32_t* d_epoch = nullptr;  // device words {this solve's base epoch, last epoch handed out}
+  int32_t* d_derr = nullptr;    // device copy of the watchdog word
+  // CUDA graphs of repeated device solves (key: b, x, ld, nrhs, layout)
+  std::vector<GraphEntry> graphs;
+  GraphEntry pending;           // last uncaptured key (captured when it repeats)
+  uint64_t solve_count = 0;
+  void* capture_stream = nullptr;  // cudaStream_t used only to capture
+  void* done_ev = nullptr;         // recorded after every solve; sptrsv_free waits on it
+  bool done_ev_recorded = false;
   int launches_per_solve = 0;
 
   // profiling

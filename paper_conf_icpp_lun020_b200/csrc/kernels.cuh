@@ -76,16 +76,66 @@ struct SolveState {
   int nticket;
   int* error;         // mapped host word (watchdog)
   uint32_t* flags;    // nrhs > 1: per-row ready flags (global row index), value = epoch when solved
-  uint32_t epoch;     // this solve's epoch (>= 1; flags start at 0)
+  // Epochs live on the device so a captured solve (CUDA graph) replays
+  // correctly: epoch_dev[0] = this solve's first epoch, epoch_dev[1] = the
+  // last epoch handed out; permute-in (block 0) advances them by `span`.
+  uint32_t* epoch_dev;
+  uint32_t epoch_off;   // offset of this launch inside the solve's span (supernodal chunk index)
+  uint32_t span;        // epochs this solve uses (0: no flags polled)
   uint32_t backoff_ns;  // cap of the sync-free polling backoff (0 = spin)
+  int* derr;            // device copy of the watchdog word: later polls give up at once
+  uint32_t wd_spins;    // unsuccessful polls before the watchdog trips (kWatchdogSpins)
+  unsigned long long* sf_trace;  // SPTRSV_SF_TRACE builds: {claim, done} globaltimer per row
 };
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#ifdef SPTRSV_SF_TRACE
+#define SF_TRACE(st, row, which) \
+  do {                                                       \
+    if ((st).sf_trace) (st).sf_trace[2 * (size_t)(row) + (which)] = gtimer(); \
+  } while (0)
+#else
+#define SF_TRACE(st, row, which) \
+  do {                         \
+  } while (0)
+#endif
 
 __device__ __forceinline__ void reset_tickets(const SolveState& st, int tid, int nthreads) {
   for (int t = tid; t < st.nticket; t += nthreads) st.tickets[t] = 0;
 }
 
+// permute-in, block 0, thread 0: hand out this solve's epochs [base, base + span)
+__device__ __forceinline__ void advance_epoch(const SolveState& st) {
+  if (st.span && st.epoch_dev) {
+    const uint32_t base = st.epoch_dev[1] + 1u;
+    st.epoch_dev[0] = base;
+    st.epoch_dev[1] = base + st.span - 1u;
+  }
+}
+
+// this launch's epoch (written by permute-in, an earlier kernel of the stream)
+__device__ __forceinline__ uint32_t solve_epoch(const SolveState& st) {
+  return *(volatile const uint32_t*)st.epoch_dev + st.epoch_off;
+}
+
 __device__ __forceinline__ void watchdog_trip(const SolveState& st) {
   if (st.error) *(volatile int*)st.error = 1;
+  if (st.derr) *(volatile int*)st.derr = 1;
+}
+
+// One more unsuccessful poll: true = give up (this poll's watchdog tripped,
+// or another one already did -- checked every 1024 polls, so the chunk
+// launches after a trip do not each spin kWatchdogSpins again).
+__device__ __forceinline__ bool wd_giveup(uint32_t& spins, const SolveState& st) {
+  if (++spins > st.wd_spins) {
+    watchdog_trip(st);
+    return true;
+  }
+  return (spins & 1023u) == 0 && st.derr && *(volatile int*)st.derr;
 }
 
 // ------------------------------------------------------------------ permute
@@ -93,13 +143,18 @@ __device__ __forceinline__ void watchdog_trip(const SolveState& st) {
 // polls it).  nrhs == 1; stride = ldb for row-major input, 1 otherwise.
 template <typename T>
 __global__ void perm_in_1(int n, const int* __restrict__ perm, const T* __restrict__ rd, const T* __restrict__ b,
-                          int64_t stride, T* __restrict__ bw, T* __restrict__ xs, int fill_sent, SolveState st) {
-  if (blockIdx.x == 0) reset_tickets(st, threadIdx.x, blockDim.x);
+                          int64_t stride, T* __restrict__ bw, T* __restrict__ xs, int fill_sent, SolveState st,
+                          T* __restrict__ part, int npart) {
+  if (blockIdx.x == 0) {
+    reset_tickets(st, threadIdx.x, blockDim.x);
+    if (threadIdx.x == 0) advance_epoch(st);
+  }
   int k = blockIdx.x * blockDim.x + threadIdx.x;
   if (k < n) {
     bw[k] = b[(int64_t)perm[k] * stride] * rd[k];
     if (fill_sent) xs[k] = sent<T>();
   }
+  if (k < npart) part[k] = sent<T>();  // split long rows' partial sums (tri_sf_items)
 }
 
 // x[perm[k]] = xs[k]
@@ -126,7 +181,10 @@ __global__ void __launch_bounds__(256) perm_in_cm(int n, int nrhs, const int* __
   __shared__ int ks[32];
   __shared__ T rs[32];
   const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
-  if (blockIdx.x == 0) reset_tickets(st, threadIdx.x, 256);
+  if (blockIdx.x == 0) {
+    reset_tickets(st, threadIdx.x, 256);
+    if (threadIdx.x == 0) advance_epoch(st);
+  }
   const int i0 = blockIdx.x * 32, i = i0 + tx;
   const bool iv = i < n;
   if (threadIdx.x < 32) {
@@ -210,7 +268,10 @@ template <typename T>
 __global__ void perm_in_rm(int n, int nrhs, const int* __restrict__ perm, const T* __restrict__ rd,
                            const T* __restrict__ b, int64_t ldb, T* __restrict__ bw, T* __restrict__ xs,
                            int fill_sent, SolveState st) {
-  if (blockIdx.x == 0) reset_tickets(st, threadIdx.x, blockDim.x);
+  if (blockIdx.x == 0) {
+    reset_tickets(st, threadIdx.x, blockDim.x);
+    if (threadIdx.x == 0) advance_epoch(st);
+  }
   int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (e < (int64_t)n * nrhs) {
     int k = (int)(e / nrhs), c = (int)(e % nrhs);
@@ -588,6 +649,7 @@ __global__ void __launch_bounds__(256) tri_syncfree_thread(int r0, int m, const 
     int p = 0, e = 0;
     T s = 0;
     if (!done) {
+      SF_TRACE(st, r, 0);
       p = rp[k];
       e = rp[k + 1];
       s = bw[r];
@@ -625,6 +687,7 @@ __global__ void __launch_bounds__(256) tri_syncfree_thread(int r0, int m, const 
         }
         if (p == e) {
           st_strong(xs + r, s);
+          SF_TRACE(st, r, 1);
           done = true;
           prog = true;
         }
@@ -667,13 +730,13 @@ __global__ void __launch_bounds__(256) tri_syncfree_thread(int r0, int m, const 
           p = min(wp, we);
           if (p == e) {
             st_strong(xs + r, s);
+            SF_TRACE(st, r, 1);
             done = true;
           }
         }
       }
       if (!__any_sync(0xffffffffu, prog)) {
-        if (++spins > kWatchdogSpins) {
-          if (!done) watchdog_trip(st);
+        if (wd_giveup(spins, st)) {
           done = true;  // give up: garbage result, reported to the host
         } else {
           ns = backoff(ns, st.backoff_ns);
@@ -703,6 +766,7 @@ __global__ void __launch_bounds__(256) tri_syncfree_warp(int r0, int m, const in
     k = __shfl_sync(0xffffffffu, k, 0);
     if (k >= m) break;
     const int r = r0 + k;
+    if (lane == 0) SF_TRACE(st, r, 0);
     const int a = rp[k], e = rp[k + 1];
     T s = 0;
     for (int p0 = a; p0 < e; p0 += 32 * U) {
@@ -724,10 +788,7 @@ __global__ void __launch_bounds__(256) tri_syncfree_warp(int r0, int m, const in
         if (p0 + lane + 32 * u < e) {
           uint32_t spins = 0;
           while (is_sent(x[u])) {
-            if (++spins > kWatchdogSpins) {
-              watchdog_trip(st);
-              break;
-            }
+            if (wd_giveup(spins, st)) break;
             x[u] = ld_strong(xs + j[u]);
           }
           s += v[u] * x[u];
@@ -735,7 +796,170 @@ __global__ void __launch_bounds__(256) tri_syncfree_warp(int r0, int m, const in
       }
     }
     s = warp_sum(s);
-    if (lane == 0) st_strong(xs + r, bw[r] - s);
+    if (lane == 0) {
+      st_strong(xs + r, bw[r] - s);
+      SF_TRACE(st, r, 1);
+    }
+  }
+}
+
+// Sync-free over nnz-balanced ROW BLOCKS (B200 selector, nrhs == 1): the
+// sync-free solve of Alg 3 (L105-L125) in pull form, with the work cut at
+// upload into items of <= 32 consecutive rows holding <= kSfNB off-diagonal
+// entries together (exec.cu build_sf_items); a row longer than kSfNB is cut
+// into kSfNB-entry PIECES, each an item of its own:
+//   - a partial piece (kind 1) writes its partial sum to a slot of `part`
+//     (value-as-flag: slots hold the sentinel until written, reset by
+//     permute-in);
+//   - the row's last piece (kind 2) adds its own entries and the partial sums
+//     of the earlier pieces, in piece order (deterministic), and publishes x.
+// A warp claims one item per ticket (row order: deadlock-free like K3, the
+// pieces of a row precede its last piece).  All entries of the item are
+// loaded coalesced and all their x_j polled at once (kSfNB/32 loads in flight
+// per lane); a ready product goes to shared memory and bumps its row's
+// counter; a row whose counter is complete is summed by its own lane in entry
+// order and published with one strong store.  Dependencies inside the item
+// are read from shared memory (the rows' solved x are forwarded there), so a
+// chain inside an item costs no L2 round trip.  Long rows (the power-law hubs
+// of L136) thus take one round of loads spread over several warps instead of
+// a serial walk by one warp.
+#ifndef SPTRSV_SF_NB
+#define SPTRSV_SF_NB 256
+#endif
+#ifndef SPTRSV_SF_MINB
+#define SPTRSV_SF_MINB 2  // resident CTAs per SM requested from ptxas
+#endif
+constexpr int kSfNB = SPTRSV_SF_NB;
+struct SfItem {
+  int t0, t1;  // local rows [t0, t1) (a piece: t1 = t0 + 1)
+  int p0, p1;  // entries [p0, p1) of the segment's CSR
+  int kind;    // 0 rows, 1 partial piece (-> part[s0]), 2 last piece (+ part[s0 .. s1))
+  int s0, s1, pad;
+};
+
+template <typename T>
+__global__ void __launch_bounds__(256, SPTRSV_SF_MINB) tri_sf_items(int r0, int nitem, const SfItem* __restrict__ items,
+                                                    const int* __restrict__ rp, const int* __restrict__ ci,
+                                                    const T* __restrict__ val, const T* __restrict__ bw,
+                                                    T* __restrict__ xs, T* __restrict__ part, SolveState st,
+                                                    int slot) {
+  constexpr int U = kSfNB / 32;
+  __shared__ T prod_s[8][kSfNB];
+  __shared__ T xloc_s[8][32];
+  __shared__ int lrp_s[8][33];
+  __shared__ int cnt_s[8][32];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  T* prod = prod_s[warp];
+  T* xloc = xloc_s[warp];
+  int* lrp = lrp_s[warp];
+  int* cnt = cnt_s[warp];
+  uint32_t* ticket = st.tickets + slot;
+  for (;;) {
+    int w = 0;
+    if (lane == 0) w = (int)atomicAdd(ticket, 1u);
+    w = __shfl_sync(0xffffffffu, w, 0);
+    if (w >= nitem) break;
+    const int4 h0 = __ldg((const int4*)(items + w));
+    const int4 h1 = __ldg((const int4*)(items + w) + 1);
+    const int t0 = h0.x, nr = h0.y - h0.x, p0 = h0.z, ne = h0.w - h0.z, kind = h1.x;
+    // row pointers of the item, relative to p0 (a piece is one row of ne entries)
+    if (lane < nr) {
+      lrp[lane] = kind == 0 ? rp[t0 + lane] - p0 : 0;
+      SF_TRACE(st, r0 + t0 + lane, 0);
+    }
+    if (lane == 0) lrp[nr] = ne;
+    cnt[lane] = 0;
+    xloc[lane] = sent<T>();
+    __syncwarp();
+    const int jlo = r0 + t0, jhi = r0 + t0 + nr;  // the item's own rows (global)
+    int j[U], rw[U];
+    T v[U], x[U];
+    uint32_t pend = 0;
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int e = lane + 32 * u;
+      if (e < ne) {
+        j[u] = ldg_nc(ci + p0 + e);
+        v[u] = ldg_nc(val + p0 + e);
+        pend |= 1u << u;
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {  // row of entry e: the last row start <= e
+      const int e = lane + 32 * u;
+      int lo = 0;
+      if (e < ne && kind == 0) {
+        int hi = nr;  // lrp[lo] <= e < lrp[hi]
+        while (hi - lo > 1) {
+          const int mid = (lo + hi) >> 1;
+          if (lrp[mid] <= e) lo = mid;
+          else hi = mid;
+        }
+      }
+      rw[u] = lo;
+    }
+    bool rdone = lane >= nr;  // this lane's row (lane < nr) is published
+    uint32_t spins = 0;
+    unsigned ns = 0;
+    for (;;) {
+      // poll every pending dependency at once (shared memory for the item's own rows)
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        if (pend & (1u << u)) {
+          if (kind == 0 && j[u] >= jlo && j[u] < jhi)
+            x[u] = *(volatile T*)&xloc[j[u] - jlo];
+          else
+            x[u] = ld_strong(xs + j[u]);
+        }
+      bool prog = false;
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        if ((pend & (1u << u)) && !is_sent(x[u])) {
+          prod[lane + 32 * u] = v[u] * x[u];
+          atomicAdd(&cnt[rw[u]], 1);
+          pend &= ~(1u << u);
+          prog = true;
+        }
+      __syncwarp();
+      if (!rdone && cnt[lane] == lrp[lane + 1] - lrp[lane]) {
+        // every product of the row is in shared memory: sum in entry order
+        T acc = 0;
+        for (int q = lrp[lane]; q < lrp[lane + 1]; ++q) acc += prod[q];
+        if (kind == 1) {
+          st_strong(part + h1.y, acc);
+          rdone = true;
+        } else {
+          bool ready = true;
+          if (kind == 2) {  // the partial sums of the row's earlier pieces
+            T ps = 0;
+            for (int q = h1.y; q < h1.z; ++q) {
+              const T pv = ld_strong(part + q);
+              ready &= !is_sent(pv);
+              ps += pv;
+            }
+            acc = ps + acc;
+          }
+          if (ready) {
+            const int r = r0 + t0 + lane;
+            const T xv = bw[r] - acc;
+            xloc[lane] = xv;
+            st_strong(xs + r, xv);
+            SF_TRACE(st, r, 1);
+            rdone = true;
+          }
+        }
+        prog |= rdone;
+      }
+      if (__all_sync(0xffffffffu, rdone)) break;
+      if (__any_sync(0xffffffffu, prog)) {
+        ns = 0;
+      } else {
+        if (wd_giveup(spins, st)) break;
+        ns = backoff(ns, st.backoff_ns);
+      }
+      __syncwarp();
+    }
+    __syncwarp();  // shared state is rewritten by the next item
   }
 }
 
@@ -787,10 +1011,7 @@ __global__ void __launch_bounds__(256, SPTRSV_SN_MINB) tri_supernode(int npieces
       uint32_t spins = 0;
       unsigned ns = 0;
       while (__any_sync(0xffffffffu, inq && is_sent(xj))) {
-        if (++spins > kWatchdogSpins) {
-          watchdog_trip(st);
-          break;
-        }
+        if (wd_giveup(spins, st)) break;
         ns = backoff(ns, st.backoff_ns);
         if (inq && is_sent(xj)) xj = ld_strong(xs + j);
       }
@@ -850,7 +1071,7 @@ __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const
   __shared__ int Jsh;
   const int tid = threadIdx.x, lane = tid & 31, wi = tid >> 5;
   uint32_t* ticket = st.tickets + slot;
-  const uint32_t epoch = st.epoch;
+  const uint32_t epoch = solve_epoch(st);
   while (true) {
     if (tid == 0) Jsh = (int)atomicAdd(ticket, 1u);
     __syncthreads();
@@ -880,10 +1101,7 @@ __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const
             uint32_t spins = 0;
             unsigned ns = 0;
             while (ld_flag(st.flags + j) != epoch) {
-              if (++spins > kWatchdogSpins) {
-                watchdog_trip(st);
-                break;
-              }
+              if (wd_giveup(spins, st)) break;
               ns = backoff(ns, st.backoff_ns);
             }
             __threadfence();
@@ -986,7 +1204,7 @@ __global__ void __launch_bounds__(256) tri_syncfree_multi(int r0, int m, const i
   const int lane = threadIdx.x % G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << ((threadIdx.x & 31) / G * G));
   uint32_t* ticket = st.tickets + slot;
-  const uint32_t epoch = st.epoch;
+  const uint32_t epoch = solve_epoch(st);
   while (true) {
     int k = 0;
     if (lane == 0) k = (int)atomicAdd(ticket, 1u);
@@ -1006,10 +1224,7 @@ __global__ void __launch_bounds__(256) tri_syncfree_multi(int r0, int m, const i
           uint32_t spins = 0;
           unsigned ns = 0;
           while (ld_flag(st.flags + j) != epoch) {
-            if (++spins > kWatchdogSpins) {
-              watchdog_trip(st);
-              break;
-            }
+            if (wd_giveup(spins, st)) break;
             ns = backoff(ns, st.backoff_ns);
           }
         }
