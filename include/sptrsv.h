@@ -126,7 +126,17 @@ typedef struct {
                                repeats the previous uncaptured one is captured into a CUDA graph;
                                later solves with a captured key replay it (one graph launch).
                                0 = always launch the kernels one by one                        */
-  int32_t reserved[5];
+  int32_t analysis;         /* where sptrsv_analyse runs: 0 = auto (default):
+                               on the device when row_ptr, col_idx and val are all device
+                               pointers, else on the host; 1 = host; 2 = device (a host CSR is
+                               copied to the device first).  Both give the same plan, bit for
+                               bit (sptrsv_plan_hash).  The device analysis finishes on the host
+                               when a segment's kernel needs a host-built format (strand
+                               wavefront, TMA/ELL chain, supernode packing); it does not support
+                               transpose = 1 (then the host analysis runs).  A device-analysed
+                               plan keeps no host copy of P L P^T: sptrsv_plan_matrix returns
+                               NOT_SUPPORTED for it.                                            */
+  int32_t reserved[4];
   /* Device-memory hooks (SURVEY 8(b) "PyTorch for device memory"): when
    * dev_alloc is set, EVERY device allocation of the plan (arena, solve
    * workspace, flags, staging) goes through dev_alloc(bytes, stream, ctx) and
@@ -210,7 +220,8 @@ typedef struct {
   int64_t device_bytes;       /* device memory owned by the plan (arena, excl. workspace)  */
   int32_t depth_rule;         /* 0 = the paper's rule (L299), 1 = B200 retune (a root with
                                  only narrow levels stays whole: DESIGN.md R30), 2 = caller's */
-  int32_t reserved_info;
+  int32_t analysis;           /* where the analysis ran: 0 host, 1 device (f-2), 2 device levels /
+                                 reorder / P L P^T + host-built kernel formats                */
 } sptrsv_plan_info_t;
 
 typedef struct {

@@ -201,7 +201,7 @@ def sptrsv_analyse(row_ptr, col_idx, val, n: int | None = None, fill: str = "L",
                    force_tri_impl: str | None = None, force_sq_impl: str | None = None,
                    host_only: bool = False, sm_count: int = 0, threads: int = 0, stream=None,
                    device: int | None = None, transpose: bool = False, max_nrhs: int = 0,
-                   graphs: bool = True, allocator: str | None = "torch") -> Plan:
+                   graphs: bool = True, allocator: str | None = "torch", analysis: str = "auto") -> Plan:
     """Preprocess a CSR lower (fill='L') or upper (fill='U') triangular matrix.
 
     transpose=True: the plan solves A^T x = b for the given A (R31).
@@ -213,6 +213,8 @@ def sptrsv_analyse(row_ptr, col_idx, val, n: int | None = None, fill: str = "L",
     torch's CUDA caching allocator (C-ABI dev_alloc hooks); None = cudaMalloc.
     max_nrhs: size the solve workspace now for this many RHS columns.
     graphs: replay repeated solves (same b, x, layout) as one CUDA graph.
+    analysis: "auto" = on the GPU when the CSR arrays are CUDA tensors, else on
+    the host; "host"; "device" (both give the same plan).
     """
     rp = _as_int32(row_ptr)
     ci = _as_int32(col_idx)
@@ -239,6 +241,7 @@ def sptrsv_analyse(row_ptr, col_idx, val, n: int | None = None, fill: str = "L",
     o.transpose = 1 if transpose else 0
     o.max_nrhs = int(max_nrhs)
     o.graphs = 1 if graphs else 0
+    o.analysis = {"auto": 0, "host": 1, "device": 2}[analysis]
     if not host_only:
         import torch
         if torch.cuda.is_available():

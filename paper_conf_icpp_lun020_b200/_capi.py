@@ -41,7 +41,8 @@ class Opts(ctypes.Structure):
                 ("reorder", ctypes.c_int32), ("selector", ctypes.c_int32), ("force_tri_impl", ctypes.c_int32),
                 ("force_sq_impl", ctypes.c_int32), ("host_only", ctypes.c_int32), ("sm_count", ctypes.c_int32),
                 ("threads", ctypes.c_int32), ("device", ctypes.c_int32), ("transpose", ctypes.c_int32),
-                ("max_nrhs", ctypes.c_int32), ("graphs", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5),
+                ("max_nrhs", ctypes.c_int32), ("graphs", ctypes.c_int32), ("analysis", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 4),
                 ("dev_alloc", DEV_ALLOC), ("dev_free", DEV_FREE), ("alloc_ctx", ctypes.c_void_p)]
 
 
@@ -52,7 +53,7 @@ class PlanInfo(ctypes.Structure):
                 ("min_block_rows", ctypes.c_int64), ("sm_count", ctypes.c_int32),
                 ("launches_per_solve", ctypes.c_int32), ("analyse_ms", ctypes.c_double),
                 ("device_bytes", ctypes.c_int64), ("depth_rule", ctypes.c_int32),
-                ("reserved_info", ctypes.c_int32)]
+                ("analysis", ctypes.c_int32)]
 
 
 class SegInfo(ctypes.Structure):

@@ -13,7 +13,7 @@ INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(HERE, "libsptrsv_b200.so")
 BUILD = os.path.join(ROOT, "build", "sptrsv")
 
-SOURCES = ["analyse.cpp", "capi.cpp", "exec.cu"]
+SOURCES = ["analyse.cpp", "analyse_dev.cu", "capi.cpp", "exec.cu"]
 HEADERS = ["internal.h", "kernels.cuh"]
 
 NVCC = os.environ.get("NVCC", shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc")

@@ -345,7 +345,7 @@ struct Reorderer {
 
 }  // namespace
 
-static int32_t select_tri(int32_t nlevels, int32_t npr) {
+int32_t select_tri(int32_t nlevels, int32_t npr) {
   // Alg 7, PAPER.md:L270-L278 (branch order: reading R12)
   if (nlevels == 1) return SPTRSV_K_COMPLETELY_PARALLEL;
   if (nlevels > 20000) return SPTRSV_K_NEAR_SERIAL;
@@ -353,7 +353,7 @@ static int32_t select_tri(int32_t nlevels, int32_t npr) {
   return SPTRSV_K_SYNC_FREE;
 }
 
-static int32_t select_sq(int32_t npr, int64_t empty, int64_t m) {
+int32_t select_sq(int32_t npr, int64_t empty, int64_t m) {
   // Alg 7, PAPER.md:L281-L292 with L258's thresholds; emptyratio compared in
   // integers (reading R9)
   if (npr <= 12) return (2 * empty <= m) ? SPTRSV_K_SCALAR_CSR : SPTRSV_K_SCALAR_DCSR;
@@ -530,12 +530,20 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
   p.lower_old = R.perm;
 
   clk.lap("P L P^T");
-  // ---- segment geometry in execution order ----
-  struct Geo { int32_t kind, r0, r1, c0, c1, leaf; };
-  std::vector<Geo> geo;
-  std::vector<std::pair<int32_t, int32_t>> leaves = nodes;  // in order
+  e = build_segments_host(p, nodes, leaf_nl, threads);
+  if (e.status) return e;
+  clk.lap("segments + Alg 7");
+  choose_impls(p);
+  clk.lap("choose_impls");
+  return {SPTRSV_SUCCESS, ""};
+}
+
+// Segment geometry in execution order (Alg 4-6, readings R16-R18).
+std::vector<SegGeo> segment_geometry(int32_t n, int32_t depth, int32_t variant,
+                                     const std::vector<std::pair<int32_t, int32_t>>& leaves) {
+  std::vector<SegGeo> geo;
   if (n > 0) {
-    if (p.opts.variant == SPTRSV_VARIANT_REC) {
+    if (variant == SPTRSV_VARIANT_REC) {
       std::function<void(int32_t, int32_t, int32_t)> rec = [&](int32_t lo, int32_t hi, int32_t d) {
         if (d == 0) {
           int32_t li = (int32_t)(std::lower_bound(leaves.begin(), leaves.end(), std::make_pair(lo, hi)) - leaves.begin());
@@ -547,12 +555,12 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
         geo.push_back({1, mid, hi, lo, mid, -1});
         rec(mid, hi, d - 1);
       };
-      rec(0, n, p.depth);
+      rec(0, n, depth);
     } else {
       int32_t K = (int32_t)leaves.size();
       for (int32_t k = 0; k < K; ++k) {
         int32_t s = leaves[k].first, e2 = leaves[k].second;
-        if (p.opts.variant == SPTRSV_VARIANT_COL) {  // Alg 4, reading R16
+        if (variant == SPTRSV_VARIANT_COL) {  // Alg 4, reading R16
           geo.push_back({0, s, e2, s, e2, k});
           if (k != K - 1) geo.push_back({1, e2, n, s, e2, -1});
         } else {  // Alg 5, reading R17
@@ -562,11 +570,23 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
       }
     }
   }
+  return geo;
+}
+
+// Blocks, features and Alg 7 labels from the host P L P^T (p.p_rp / p_ci /
+// p_val, p.diag_new, p.leaf_level); leaves = the recursion's leaf ranges in
+// order, leaf_nl = their level counts.
+Error build_segments_host(Plan& p, const std::vector<std::pair<int32_t, int32_t>>& nodes,
+                          const std::vector<int32_t>& leaf_nl, int threads) {
+  const int32_t n = p.n;
+  const size_t vb = p.vbytes;
+  // ---- segment geometry in execution order ----
+  const std::vector<SegGeo> geo = segment_geometry(n, p.depth, p.opts.variant, nodes);
 
   // ---- extract blocks, features, Alg 7 ----
   p.segs.resize(geo.size());
   auto build_seg = [&](size_t si, int inner) {
-    const Geo& g = geo[si];
+    const SegGeo& g = geo[si];
     Segment& S = p.segs[si];
     sptrsv_seg_info_t& I = S.info;
     I.kind = g.kind;
@@ -633,6 +653,9 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
         }
         S.sn_ptr.push_back(m);
       }
+      S.npieces = (int64_t)S.sn_ptr.size() - 1;
+      S.kmax_indeg = 0;
+      for (int32_t k = 0; k < m; ++k) S.kmax_indeg = std::max(S.kmax_indeg, S.in_degree[k]);
     } else {
       I.nnz = tot;
       I.nnz_per_row = m ? (int32_t)(tot / m) : 0;
@@ -712,9 +735,6 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
   } else {
     for (size_t k = 0; k < geo.size(); ++k) build_seg(k, threads);
   }
-  clk.lap("segments + Alg 7");
-  choose_impls(p);
-  clk.lap("choose_impls");
   return {SPTRSV_SUCCESS, ""};
 }
 
@@ -731,7 +751,7 @@ void choose_impls(Plan& p) {
         case SPTRSV_K_NEAR_SERIAL: impl = SPTRSV_IMPL_TRI_CHAIN; break;
         default: impl = SPTRSV_IMPL_TRI_SYNCFREE; break;
       }
-      const int64_t npieces = (int64_t)S.sn_ptr.size() - 1;
+      const int64_t npieces = S.npieces;
       const bool supernodal = npieces > 0 && (double)(I.row1 - I.row0) / (double)npieces >= 8.0;
       if (p.opts.selector == SPTRSV_SELECT_B200 && I.nlevels > 1 && supernodal) {
         impl = SPTRSV_IMPL_TRI_SUPERNODE;
@@ -744,8 +764,7 @@ void choose_impls(Plan& p) {
           // wavefront over one thread-block cluster (exec.cu build_wave, which
           // falls back to the single-CTA chain when the rows' dependencies
           // do not stay inside their strands); else one CTA walks the chain
-          int32_t kmax = 0;
-          for (int64_t r = 0; r < m; ++r) kmax = std::max(kmax, S.in_degree[r]);
+          const int32_t kmax = S.kmax_indeg;
           impl = (kmax >= 1 && kmax <= 8 && m >= 4096 && std::getenv("SPTRSV_NO_WAVE") == nullptr)
                      ? SPTRSV_IMPL_TRI_PIPE
                      : SPTRSV_IMPL_TRI_CHAIN;

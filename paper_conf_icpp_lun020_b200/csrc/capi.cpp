@@ -50,6 +50,7 @@ SPTRSV_EXPORT void sptrsv_opts_default(sptrsv_opts_t* o) {
   o->device = -1;
   o->max_nrhs = 0;
   o->graphs = 1;
+  o->analysis = 0;
   o->dev_alloc = nullptr;
   o->dev_free = nullptr;
   o->alloc_ctx = nullptr;
@@ -97,6 +98,7 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_analyse(int32_t n, int64_t nnz, const int32
   if (o.min_block_rows < 0) return fail(SPTRSV_ERROR_INVALID_VALUE, "min_block_rows < 0");
   if (o.transpose < 0 || o.transpose > 1) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad transpose");
   if (o.max_nrhs < 0) return fail(SPTRSV_ERROR_INVALID_VALUE, "max_nrhs < 0");
+  if (o.analysis < 0 || o.analysis > 2) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad analysis");
   if ((o.dev_alloc == nullptr) != (o.dev_free == nullptr))
     return fail(SPTRSV_ERROR_INVALID_VALUE, "dev_alloc and dev_free must be given together");
 
@@ -130,6 +132,53 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_analyse(int32_t n, int64_t nnz, const int32
                                                   "; this library is built for sm_100a (B200) only");
     }
     p.sm_count = o.sm_count > 0 ? o.sm_count : sms;
+    // device analysis (f-2): CSR in device memory (auto) or requested
+    bool on_dev = false;
+    if (!o.transpose && o.analysis != 1) {
+      auto is_dev = [](const void* q) {
+        cudaPointerAttributes a;
+        if (cudaPointerGetAttributes(&a, q) != cudaSuccess) {
+          cudaGetLastError();
+          return false;
+        }
+        return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+      };
+      const bool all_dev = is_dev(row_ptr) && (nnz == 0 || (is_dev(col_idx) && is_dev(val)));
+      on_dev = o.analysis == 2 || all_dev;
+      if (on_dev && n > 0) {
+        cudaStream_t s = (cudaStream_t)stream;
+        const void *drp = row_ptr, *dci = col_idx, *dval = val;
+        void* tmp = nullptr;
+        if (!all_dev) {  // host CSR, device analysis requested: one copy in
+          const size_t b1 = (size_t)(n + 1) * 4, b2 = (size_t)nnz * 4, b3 = (size_t)nnz * p.vbytes;
+          tmp = dalloc(p, b1 + b2 + b3 + 512, s);
+          if (!tmp) {
+            delete P;
+            return fail(SPTRSV_ERROR_ALLOC, "device copy of the CSR failed");
+          }
+          char* t = (char*)tmp;
+          drp = t;
+          dci = t + ((b1 + 255) / 256) * 256;
+          dval = (char*)dci + ((b2 + 255) / 256) * 256;
+          cudaMemcpyAsync((void*)drp, row_ptr, b1, cudaMemcpyHostToDevice, s);
+          cudaMemcpyAsync((void*)dci, col_idx, b2, cudaMemcpyHostToDevice, s);
+          cudaMemcpyAsync((void*)dval, val, b3, cudaMemcpyHostToDevice, s);
+        }
+        Error de = analyse_device(p, n, nnz, (const int32_t*)drp, (const int32_t*)dci, dval, stream);
+        if (tmp) {
+          cudaStreamSynchronize(s);
+          dfree(p, tmp, s);
+        }
+        if (de.status) {
+          release(p);
+          delete P;
+          return fail(de);
+        }
+        p.analyse_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+        *plan_out = P;
+        return SPTRSV_SUCCESS;
+      }
+    }
     Error ce{SPTRSV_SUCCESS, ""};
     if (!host_copy_if_device(row_ptr, (size_t)(n + 1) * 4, hrp, &rp_h, &ce) ||
         (nnz > 0 && !host_copy_if_device(col_idx, (size_t)nnz * 4, hci, &ci_h, &ce)) ||
@@ -205,7 +254,7 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_info(sptrsv_plan_t plan, sptrsv_plan_i
   out->launches_per_solve = p.launches_per_solve;
   out->analyse_ms = p.analyse_ms;
   out->depth_rule = p.opts.depth >= 0 ? 2 : p.depth_retuned;
-  out->reserved_info = 0;
+  out->analysis = p.analysis_where;
   out->device_bytes = (int64_t)p.arena_bytes;
   return SPTRSV_SUCCESS;
 }
@@ -219,14 +268,24 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_segments(sptrsv_plan_t plan, sptrsv_se
   return SPTRSV_SUCCESS;
 }
 
+// device-analysed plans fetch their host copies on first introspection
+static sptrsv_status_t host_view(Plan& p) {
+  if (p.host_ready) return SPTRSV_SUCCESS;
+  Error e = materialize_host(p);
+  if (e.status) return fail(e);
+  return SPTRSV_SUCCESS;
+}
+
 SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_perm(sptrsv_plan_t plan, int32_t* host_new_to_old) {
   if (!plan || (!host_new_to_old && plan->p.n)) return fail(SPTRSV_ERROR_INVALID_VALUE, "NULL argument");
+  if (sptrsv_status_t st = host_view(plan->p)) return st;
   std::memcpy(host_new_to_old, plan->p.perm.data(), plan->p.perm.size() * 4);
   return SPTRSV_SUCCESS;
 }
 
 SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_levels(sptrsv_plan_t plan, int32_t* host_leaf_level) {
   if (!plan || (!host_leaf_level && plan->p.n)) return fail(SPTRSV_ERROR_INVALID_VALUE, "NULL argument");
+  if (sptrsv_status_t st = host_view(plan->p)) return st;
   std::memcpy(host_leaf_level, plan->p.leaf_level.data(), plan->p.leaf_level.size() * 4);
   return SPTRSV_SUCCESS;
 }
@@ -234,6 +293,7 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_levels(sptrsv_plan_t plan, int32_t* ho
 SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_seg_array(sptrsv_plan_t plan, int32_t seg, int32_t which,
                                                     int32_t* host_out, int64_t cap, int64_t* count) {
   if (!plan) return fail(SPTRSV_ERROR_INVALID_VALUE, "plan is NULL");
+  if (sptrsv_status_t st = host_view(plan->p)) return st;
   const Plan& p = plan->p;
   if (seg < 0 || seg >= (int32_t)p.segs.size()) return fail(SPTRSV_ERROR_INVALID_VALUE, "segment out of range");
   const Segment& S = p.segs[seg];
@@ -263,6 +323,8 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_matrix(sptrsv_plan_t plan, int64_t* ro
                                                  void* val) {
   if (!plan) return fail(SPTRSV_ERROR_INVALID_VALUE, "plan is NULL");
   const Plan& p = plan->p;
+  if (p.dev_analysed)
+    return fail(SPTRSV_ERROR_NOT_SUPPORTED, "a device-analysed plan keeps no host copy of P L P^T");
   if (row_ptr) std::memcpy(row_ptr, p.p_rp.data(), p.p_rp.size() * 8);
   if (col_idx) std::memcpy(col_idx, p.p_ci.data(), p.p_ci.size() * 4);
   if (val) std::memcpy(val, p.p_val.data(), p.p_val.size());
@@ -295,6 +357,7 @@ struct Fnv {
 
 SPTRSV_EXPORT sptrsv_status_t sptrsv_plan_hash(sptrsv_plan_t plan, uint64_t* out) {
   if (!plan || !out) return fail(SPTRSV_ERROR_INVALID_VALUE, "NULL argument");
+  if (sptrsv_status_t st = host_view(plan->p)) return st;
   const Plan& p = plan->p;
   Fnv f;
   int64_t hdr[6] = {p.n, p.nnz, (int64_t)p.dtype, (int64_t)p.fill, p.depth, (int64_t)p.segs.size()};

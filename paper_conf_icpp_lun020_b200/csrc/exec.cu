@@ -976,13 +976,16 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
           };
           if (nrhs == 1 && !S.sf_items.empty()) {
             const int nitem = (int)(S.sf_items.size() / 8);
-            static const int per_sm = [] {
-              const char* e2 = std::getenv("SPTRSV_SF_PERSM");  // tuning: resident CTAs per SM
-              return e2 ? std::max(1, std::atoi(e2)) : SPTRSV_SF_MINB;
-            }();
-            const unsigned g = std::max(1u, std::min<unsigned>(cdiv(nitem, 8), (unsigned)(per_sm * p.sm_count)));
-            k::tri_sf_items<T><<<g, 256, 0, s>>>(I.row0, nitem, (const k::SfItem*)S.d_sf_items, S.d_rp, S.d_ci, val,
-                                                 bw, xs, (T*)p.d_part, st, S.ticket_slot);
+            int nctas = SPTRSV_SF_MINB * p.sm_count;
+            if (const char* e2 = std::getenv("SPTRSV_SF_CTAS")) nctas = std::max(1, std::atoi(e2));  // tuning
+            const unsigned g = std::max(1u, std::min<unsigned>(cdiv(nitem, 8), (unsigned)nctas));
+            if (S.sf_mixed)
+              k::tri_sf_mixed<T, 4><<<std::max(1u, ctas(256, m)), 256, 0, s>>>(
+                  I.row0, nitem, (const k::SfItem*)S.d_sf_items, S.d_rp, S.d_ci, val, bw, xs, (T*)p.d_part, st,
+                  S.ticket_slot);
+            else
+              k::tri_sf_items<T><<<g, 256, 0, s>>>(I.row0, nitem, (const k::SfItem*)S.d_sf_items, S.d_rp, S.d_ci,
+                                                   val, bw, xs, (T*)p.d_part, st, S.ticket_slot);
           } else if (nrhs == 1) {
             if (tri_use_warp(S))
               k::tri_syncfree_warp<T, 8><<<std::max(1u, ctas(8, m)), 256, 0, s>>>(I.row0, m, S.d_rp, S.d_ci, val,
@@ -1124,6 +1127,7 @@ Error solve_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, int nrhs
   // nrhs == 1: sync-free rows poll their dependencies' values, which start
   // as the sentinel; nrhs > 1: they poll per-row epoch flags instead
   const int fill = (p.needs_sentinel && nrhs == 1) ? 1 : 0;
+  if (const char* e = std::getenv("SPTRSV_SF_BACKOFF")) p.backoff_ns = (uint32_t)std::max(0, std::atoi(e));  // tuning
   k::SolveState st{p.d_tickets,         p.nticket,    p.d_error, (uint32_t*)p.ws.flags, p.d_epoch, 0u,
                    epoch_span(p, nrhs), p.backoff_ns, p.d_derr,  p.wd_spins, (unsigned long long*)p.d_sf_trace};
   cudaEvent_t* ev = nullptr;
@@ -1249,10 +1253,14 @@ void build_sq_items(Segment& S) {
 // slot out of the plan's `part` array) closed by its last piece (kind 2),
 // which adds the earlier pieces' partial sums.  SPTRSV_SF_V1 keeps the
 // round-1 kernels (thread / warp per row).
+void build_sf_mixed(Segment& S, int32_t& part_base);
 void build_sf_items(Segment& S, int32_t& part_base) {
   S.sf_items.clear();
   const auto& I = S.info;
-  if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_SYNCFREE || !std::getenv("SPTRSV_SF_ITEMS")) return;
+  if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_SYNCFREE) return;
+  S.sf_mixed = std::getenv("SPTRSV_SF_MIXED") != nullptr;
+  if (S.sf_mixed) return build_sf_mixed(S, part_base);
+  if (!std::getenv("SPTRSV_SF_ITEMS")) return;
   const int m = I.row1 - I.row0;
   const std::vector<int32_t>& rp = S.rp;
   auto push = [&](int t0, int t1, int p0, int p1, int kind, int s0, int s1) {
@@ -1281,6 +1289,44 @@ void build_sf_items(Segment& S, int32_t& part_base) {
       tot += rp[t + 1] - rp[t];
       ++t;
     }
+    push(start, t, rp[start], rp[t], 0, 0, 0);
+  }
+}
+
+// Work items of the mixed-granularity sync-free kernel (k::tri_sf_mixed):
+// runs of <= 32 consecutive rows with <= kSfLong entries each (kind 0); a
+// longer row is one warp item (kind 3) up to kSfNB entries, else kSfNB-entry
+// pieces (kind 1) closed by its last piece (kind 2) with partial-sum slots.
+void build_sf_mixed(Segment& S, int32_t& part_base) {
+  const auto& I = S.info;
+  const int m = I.row1 - I.row0;
+  const std::vector<int32_t>& rp = S.rp;
+  auto push = [&](int t0, int t1, int p0, int p1, int kind, int s0, int s1) {
+    const int32_t rec[8] = {t0, t1, p0, p1, kind, s0, s1, 0};
+    S.sf_items.insert(S.sf_items.end(), rec, rec + 8);
+  };
+  int t = 0;
+  while (t < m) {
+    const int len = rp[t + 1] - rp[t];
+    if (len > k::kSfLong) {
+      if (len <= k::kSfNB) {
+        push(t, t + 1, rp[t], rp[t + 1], 3, 0, 0);
+      } else {
+        const int np = (len + k::kSfNB - 1) / k::kSfNB;
+        const int first = part_base;
+        for (int q = 0; q < np; ++q) {
+          const int a = rp[t] + q * k::kSfNB, b = std::min(a + k::kSfNB, rp[t + 1]);
+          if (q < np - 1)
+            push(t, t + 1, a, b, 1, part_base++, 0);
+          else
+            push(t, t + 1, a, b, 2, first, part_base);
+        }
+      }
+      ++t;
+      continue;
+    }
+    const int start = t;
+    while (t < m && t - start < 32 && rp[t + 1] - rp[t] <= k::kSfLong) ++t;
     push(start, t, rp[start], rp[t], 0, 0, 0);
   }
 }
@@ -1377,7 +1423,6 @@ Error upload(Plan& p, void* stream_v) {
   p.trace = std::getenv("SPTRSV_TRACE") != nullptr;
   p.spmm = spmm_cfg();
   p.backoff_ns = 128;
-  if (const char* e = std::getenv("SPTRSV_SF_BACKOFF")) p.backoff_ns = (uint32_t)std::max(0, std::atoi(e));
   p.wd_spins = k::kWatchdogSpins;
   if (std::getenv("SPTRSV_SF_TRACE") && !p.d_sf_trace)  // debug: per-row claim/done stamps (SF_TRACE builds)
     if (cudaMalloc(&p.d_sf_trace, (size_t)std::max(1, n) * 16) != cudaSuccess) p.d_sf_trace = nullptr;
@@ -1912,5 +1957,8 @@ Error device_info(int* sm_count, int* major, int* minor) {
   CUDA_TRY(cudaDeviceGetAttribute(minor, cudaDevAttrComputeCapabilityMinor, dev));
   return {SPTRSV_SUCCESS, ""};
 }
+
+int count_launches_public(const Plan& p) { return count_launches(p); }
+Error prepare_solve_public(Plan& p, int nrhs, cudaStream_t s) { return prepare_solve(p, nrhs, s); }
 
 }  // namespace sptrsv

@@ -13,6 +13,8 @@
 #include <string>
 #include <vector>
 
+#include <cuda_runtime.h>
+
 #include "sptrsv.h"
 
 namespace sptrsv {
@@ -93,6 +95,8 @@ struct Segment {
   std::vector<int32_t> in_degree;  // TRI: off-diagonal count per local row
   std::vector<int32_t> sn_ptr;     // TRI: fundamental-supernode pieces (<= 32 rows), local row starts + m
   int32_t nzr = 0;                 // SQ: stored rows (== m for CSR)
+  int32_t kmax_indeg = 0;          // TRI: largest in_degree (selector feature)
+  int64_t npieces = 0;             // TRI: fundamental-supernode pieces (selector feature)
   // ----- device -----
   const int32_t* d_rp = nullptr;
   const int32_t* d_ci = nullptr;
@@ -128,6 +132,7 @@ struct Segment {
   int32_t dev_nzr = 0;
   // row-block sync-free triangle kernel (k::tri_sf_items, nrhs == 1): k::SfItem[] as 8 ints
   std::vector<int32_t> sf_items;
+  bool sf_mixed = false;
   const int32_t* d_sf_items = nullptr;
   // row-block square kernel (k::sq_adapt_1, nrhs == 1): k::SqItem[] as 4 ints
   std::vector<int32_t> sq_items;
@@ -202,8 +207,12 @@ struct Plan {
   dvec<int32_t> p_ci;
   dvec<char> p_val;
 
+  bool dev_analysed = false;  // the analysis ran on the device (analyse_dev.cu)
+  int32_t analysis_where = 0; // 0 host, 1 device, 2 device + host-built formats
+  bool host_ready = true;     // host copies of the stored arrays exist (else materialize_host)
   // ----- device -----
   int device = -1;
+  const int32_t* d_leaf_level = nullptr;  // device-analysed plans: leaf levels (introspection)
   void* arena = nullptr;
   size_t arena_bytes = 0;
   const int32_t* d_perm = nullptr;
@@ -247,6 +256,26 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
 
 // kernel implementation choice per segment (selector / forced)
 void choose_impls(Plan& p);
+
+// segment geometry + host extraction (analyse.cpp); used by both analyses
+struct SegGeo {
+  int32_t kind, r0, r1, c0, c1, leaf;
+};
+std::vector<SegGeo> segment_geometry(int32_t n, int32_t depth, int32_t variant,
+                                     const std::vector<std::pair<int32_t, int32_t>>& leaves);
+Error build_segments_host(Plan& p, const std::vector<std::pair<int32_t, int32_t>>& leaves,
+                          const std::vector<int32_t>& leaf_nl, int threads);
+int32_t select_tri(int32_t nlevels, int32_t npr);
+int32_t select_sq(int32_t npr, int64_t empty, int64_t m);
+
+// device-resident analysis (analyse_dev.cu): CSR given as
+// device pointers; builds the arena on the device (no upload()).
+Error analyse_device(Plan& p, int32_t n, int64_t nnz, const int32_t* d_rp, const int32_t* d_ci, const void* d_val,
+                     void* stream);
+// host copies of a device-analysed plan's arrays (introspection, hash)
+Error materialize_host(Plan& p);
+void* dalloc(Plan& p, size_t bytes, cudaStream_t s);
+void dfree(Plan& p, void* q, cudaStream_t s);
 
 // device side (exec.cu)
 Error upload(Plan& p, void* stream);

@@ -830,6 +830,10 @@ __global__ void __launch_bounds__(256) tri_syncfree_warp(int r0, int m, const in
 #define SPTRSV_SF_MINB 2  // resident CTAs per SM requested from ptxas
 #endif
 constexpr int kSfNB = SPTRSV_SF_NB;
+#ifndef SPTRSV_SF_LONG
+#define SPTRSV_SF_LONG 32
+#endif
+constexpr int kSfLong = SPTRSV_SF_LONG;  // tri_sf_mixed: rows with more entries get a warp
 struct SfItem {
   int t0, t1;  // local rows [t0, t1) (a piece: t1 = t0 + 1)
   int p0, p1;  // entries [p0, p1) of the segment's CSR
@@ -872,6 +876,7 @@ __global__ void __launch_bounds__(256, SPTRSV_SF_MINB) tri_sf_items(int r0, int 
     xloc[lane] = sent<T>();
     __syncwarp();
     const int jlo = r0 + t0, jhi = r0 + t0 + nr;  // the item's own rows (global)
+    const T bwr = (lane < nr && kind != 1) ? bw[jlo + lane] : T(0);  // off the critical path
     int j[U], rw[U];
     T v[U], x[U];
     uint32_t pend = 0;
@@ -941,7 +946,7 @@ __global__ void __launch_bounds__(256, SPTRSV_SF_MINB) tri_sf_items(int r0, int 
           }
           if (ready) {
             const int r = r0 + t0 + lane;
-            const T xv = bw[r] - acc;
+            const T xv = bwr - acc;
             xloc[lane] = xv;
             st_strong(xs + r, xv);
             SF_TRACE(st, r, 1);
@@ -960,6 +965,175 @@ __global__ void __launch_bounds__(256, SPTRSV_SF_MINB) tri_sf_items(int r0, int 
       __syncwarp();
     }
     __syncwarp();  // shared state is rewritten by the next item
+  }
+}
+
+// Sync-free, mixed granularity (B200 selector, nrhs == 1; exec.cu
+// build_sf_mixed).  Work items in row order, one per ticket (deadlock-free
+// like K3):
+//   kind 0  a GROUP of <= 32 consecutive rows with <= kSfLong off-diagonal
+//           entries each, one lane per row (the thread-per-component form of
+//           L247).  A lane consumes its dependencies in batches of U loads;
+//           when it meets an unsolved x_j it keeps that ONE address and the
+//           warp enters a lean spin (one strong load per blocked lane, a
+//           ballot, a branch -- no other issue slots taken from the SM's
+//           critical warps) until some lane's value lands.
+//   kind 3  a LONG row of <= kSfNB entries, solved by the whole warp (a warp
+//           per component, L247): all its loads in flight at once.
+//   kind 1/2 the pieces of a row longer than kSfNB: partial sums to `part`
+//           slots (sentinel until written), the last piece adds them in piece
+//           order (deterministic) and publishes x.
+template <typename T, int U>
+__global__ void __launch_bounds__(256) tri_sf_mixed(int r0, int nitem, const SfItem* __restrict__ items,
+                                                    const int* __restrict__ rp, const int* __restrict__ ci,
+                                                    const T* __restrict__ val, const T* __restrict__ bw,
+                                                    T* __restrict__ xs, T* __restrict__ part, SolveState st,
+                                                    int slot) {
+  constexpr int UW = kSfNB / 32;
+  const int lane = threadIdx.x & 31;
+  uint32_t* ticket = st.tickets + slot;
+  uint32_t spins = 0;
+  for (;;) {
+    int w = 0;
+    if (lane == 0) w = (int)atomicAdd(ticket, 1u);
+    w = __shfl_sync(0xffffffffu, w, 0);
+    if (w >= nitem) break;
+    const int4 h0 = __ldg((const int4*)(items + w));
+    const int4 h1 = __ldg((const int4*)(items + w) + 1);
+    if (h1.x == 0) {  // ---------------------------------------- row group
+      const int k = h0.x + lane;
+      bool done = k >= h0.y;
+      const int r = r0 + k;
+      int p = 0, e = 0;
+      T s = 0;
+      if (!done) {
+        SF_TRACE(st, r, 0);
+        p = rp[k];
+        e = rp[k + 1];
+        s = bw[r];
+      }
+      int jb = 0;
+      T vb = 0, xb = 0;
+      bool blocked = false;
+      for (;;) {
+        if (!done) {
+          if (blocked && !is_sent(xb)) {
+            s -= vb * xb;
+            ++p;
+            blocked = false;
+          }
+          while (!blocked && p < e) {
+            const int cnt = min(U, e - p);
+            int j[U];
+            T v[U], x[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+              if (u < cnt) {
+                j[u] = ldg_nc(ci + p + u);
+                v[u] = ldg_nc(val + p + u);
+              }
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+              if (u < cnt) x[u] = ld_strong(xs + j[u]);
+            int took = 0;
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+              if (u < cnt && took == u) {
+                if (!is_sent(x[u])) {
+                  s -= v[u] * x[u];
+                  ++took;
+                } else {
+                  jb = j[u];
+                  vb = v[u];
+                  xb = x[u];
+                  blocked = true;
+                }
+              }
+            p += took;
+          }
+          if (!blocked) {
+            st_strong(xs + r, s);
+            SF_TRACE(st, r, 1);
+            done = true;
+          }
+        }
+        if (__all_sync(0xffffffffu, done)) break;
+        // lean spin until some blocked lane's value has landed
+        bool give = false;
+        while (!__any_sync(0xffffffffu, !done && !is_sent(xb))) {
+          if (wd_giveup(spins, st)) {
+            give = true;
+            break;
+          }
+          if (!done) xb = ld_strong(xs + jb);
+        }
+        if (give) break;
+      }
+      continue;
+    }
+    // ------------------------------------------- a long row / a piece of one
+    const int kind = h1.x, p0 = h0.z, ne = h0.w - h0.z;
+    const int r = r0 + h0.x;
+    if (lane == 0) SF_TRACE(st, r, 0);
+    const T bwr = (kind != 1 && lane == 0) ? bw[r] : T(0);
+    int j[UW];
+    T v[UW], x[UW];
+    uint32_t pend = 0;
+#pragma unroll
+    for (int u = 0; u < UW; ++u) {
+      const int e = lane + 32 * u;
+      if (e < ne) {
+        j[u] = ldg_nc(ci + p0 + e);
+        v[u] = ldg_nc(val + p0 + e);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < UW; ++u)
+      if (lane + 32 * u < ne) {
+        x[u] = ld_strong(xs + j[u]);
+        if (is_sent(x[u])) pend |= 1u << u;
+      } else {
+        x[u] = T(0);
+        v[u] = T(0);
+      }
+    bool give = false;
+    while (__any_sync(0xffffffffu, pend != 0)) {
+      if (wd_giveup(spins, st)) {
+        give = true;
+        break;
+      }
+#pragma unroll
+      for (int u = 0; u < UW; ++u)
+        if (pend & (1u << u)) {
+          x[u] = ld_strong(xs + j[u]);
+          if (!is_sent(x[u])) pend &= ~(1u << u);
+        }
+    }
+    if (give) break;
+    T acc = 0;
+#pragma unroll
+    for (int u = 0; u < UW; ++u) acc += v[u] * x[u];
+    acc = warp_sum(acc);
+    if (kind == 2) {  // add the earlier pieces' partial sums, in piece order
+      const int np = h1.z - h1.y;
+      T pv = T(0);
+      if (lane < np) {
+        pv = ld_strong(part + h1.y + lane);
+        while (is_sent(pv)) {
+          if (wd_giveup(spins, st)) break;
+          pv = ld_strong(part + h1.y + lane);
+        }
+      }
+      acc += warp_sum(pv);
+    }
+    if (lane == 0) {
+      if (kind == 1) {
+        st_strong(part + h1.y, acc);
+      } else {
+        st_strong(xs + r, bwr - acc);
+        SF_TRACE(st, r, 1);
+      }
+    }
   }
 }
 

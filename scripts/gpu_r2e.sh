@@ -1,0 +1,14 @@
+#!/bin/bash
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+export SPTRSV_GEN_CACHE=/tmp/gencache
+SPTRSV_SF_MIXED=1 timeout 900 python -m pytest tests/test_gpu_parity.py -m gpu -x -q -k "small_configs or forced_kernels or variants or fp32 or upper or adversarial or long_chain or (full_size_configs and C3)" > gpurun_out/r2e_pytest.log 2>&1; echo "pytest mixed rc=$?"; tail -3 gpurun_out/r2e_pytest.log
+echo "== MIXED"
+SPTRSV_SF_MIXED=1 timeout 900 python scripts/sweep_sf.py C3 SPTRSV_SF_CTAS=148 SPTRSV_SF_CTAS=592 SPTRSV_SF_BACKOFF=0 2>&1 | tail -4
+for L in 16 64; do
+SPTRSV_NVCC_FLAGS="-DSPTRSV_SF_LONG=$L" python -c "from paper_conf_icpp_lun020_b200 import build; build.build(force=True)" > /dev/null 2>&1
+echo "== MIXED LONG=$L"; SPTRSV_SF_MIXED=1 timeout 900 python scripts/sweep_sf.py C3 2>&1 | tail -1
+done
+SPTRSV_NVCC_FLAGS=-DSPTRSV_SF_TRACE python -c "from paper_conf_icpp_lun020_b200 import build; build.build(force=True)" > /dev/null 2>&1
+mkdir -p /tmp/sft
+echo "== trace MIXED"; SPTRSV_SF_MIXED=1 SPTRSV_SF_TRACE=/tmp/sft timeout 600 python scripts/sf_trace.py C3 2>&1 | tail -40
