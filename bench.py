@@ -286,17 +286,29 @@ def main():
     b_np = g.gen_rhs_cols(M.n, c0, c1, seed=seed)  # (nrhs, n): this rank's columns
     val = M.val if args.dtype == "f64" else M.val.astype(np.float32)
 
-    # preprocess (analysis + upload): one warm-up, median of 3
+    # preprocess (analysis + upload, median of 3 after one
+    # warm-up).  The CSR resident on the device runs the device analysis
+    # (f-2, analyse_dev.cu); a host CSR runs the host analysis + upload.
     kw = dict(selector=args.selector, variant=args.variant, transpose=args.transpose)
-    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, val, **kw)
-    pre = []
-    for _ in range(3):
-        t0 = time.perf_counter()
-        p2 = sp.sptrsv_analyse(M.row_ptr, M.col_idx, val, **kw)
-        torch.cuda.synchronize()
-        pre.append((time.perf_counter() - t0) * 1e3)
-        p2.free()
-    preprocess_ms = float(np.median(pre))
+    dcsr = [torch.from_numpy(a).to(dev) for a in (M.row_ptr, M.col_idx, val)]
+    torch.cuda.synchronize()
+
+    def time_analyse(src, **extra):
+        ts = []
+        for i in range(4):
+            t0 = time.perf_counter()
+            p2 = sp.sptrsv_analyse(*src, **kw, **extra)
+            torch.cuda.synchronize()
+            if i:
+                ts.append((time.perf_counter() - t0) * 1e3)
+            where = p2.info()["analysis"]
+            p2.free()
+        return float(np.median(ts)), where
+
+    preprocess_ms, analysis_where = time_analyse(dcsr)
+    preprocess_host_ms, _ = time_analyse((M.row_ptr, M.col_idx, val))
+    plan = sp.sptrsv_analyse(*dcsr, **kw)
+    del dcsr
     info = plan.info()
     segs = plan.segments()
     if use_dist:
@@ -515,6 +527,17 @@ def main():
                        "parallelism": (f"rhs-columns sharded x{ws} (NCCL scatter/gather only in e2e)" if sharded
                                        else f"rhs-replicas x{ws}")},
             "preprocess_ms": preprocess_ms,
+            "preprocess": {
+                "device_csr_ms": preprocess_ms,
+                "analysis": ["host", "device", "device levels/reorder + host formats"][analysis_where],
+                "host_csr_ms": preprocess_host_ms,
+                "over_solve": preprocess_ms / ms_per_step,
+                # Table 5: preprocessing + k solves, and the
+                # share of preprocessing in it
+                "amortised": {str(k): {"total_ms": preprocess_ms + k * ms_per_step,
+                                       "pre_share": preprocess_ms / (preprocess_ms + k * ms_per_step)}
+                              for k in (1, 100, 500, 1000)},
+            },
             "hbm_whole_solve": whole,
             "roofline": roofline,
             "timing": timing,

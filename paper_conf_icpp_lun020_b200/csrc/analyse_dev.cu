@@ -27,6 +27,7 @@
 #include <cstring>
 #include <numeric>
 #include <string>
+#include <mutex>
 #include <thread>
 
 #include "internal.h"
@@ -37,7 +38,8 @@ namespace sptrsv {
 Error upload(Plan& p, void* stream);
 int count_launches_public(const Plan& p);
 void build_sq_items(Segment& S);
-void build_sf_items(Segment& S, int32_t& part_base);
+void build_sf_items(Segment& S, int32_t& part_base, int selector);
+void fuse_square_items(Segment& T, Segment& Q);
 bool watchdog_word_acquire(int32_t** h, int32_t** d);
 Error prepare_solve_public(Plan& p, int nrhs, cudaStream_t s);
 
@@ -123,6 +125,7 @@ __global__ void __launch_bounds__(256) level_sweep(int lo, int hi, const int* __
                                                    const int* __restrict__ o2n, int identity,
                                                    const int* __restrict__ rp, const int* __restrict__ ci,
                                                    int* __restrict__ lev, unsigned* ticket, int* nlev) {
+  constexpr int U = 8;  // dependencies per batch, all loads in flight together
   const int lane = threadIdx.x & 31, m = hi - lo;
   int mx = 0;
   for (;;) {
@@ -132,28 +135,65 @@ __global__ void __launch_bounds__(256) level_sweep(int lo, int hi, const int* __
     if (base >= m) break;
     const int k = base + lane;
     bool done = k >= m;
-    int q = 0, e = 0, lv = 0;
+    int q = 0, e = 0, lv = 0, cnt = 0;
     if (!done) {
       const int o = identity ? lo + k : perm[lo + k];
       q = rp[o];
       e = rp[o + 1] - 1;  // off-diagonals (the diagonal is last)
     }
-    while (__any_sync(0xffffffffu, !done)) {
+    int c[U], v[U];
+    uint32_t pend = 0;
+    bool have = false;
+    for (;;) {
       if (!done) {
-        while (q < e) {
-          const int c = identity ? ci[q] : o2n[ci[q]];
-          if (c >= lo) {
-            const int v = ld_lev(lev + (c - lo));
-            if (v < 0) break;
-            lv = max(lv, v + 1);
+        for (;;) {
+          if (have) {
+            if (pend) break;
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+              if (u < cnt && c[u] >= lo) lv = max(lv, v[u] + 1);
+            q += cnt;
+            have = false;
           }
-          ++q;
+          if (q >= e) {
+            st_lev(lev + k, lv);
+            mx = max(mx, lv + 1);
+            done = true;
+            break;
+          }
+          cnt = min(U, e - q);
+#pragma unroll
+          for (int u = 0; u < U; ++u)
+            if (u < cnt) c[u] = ci[q + u];
+          if (!identity) {
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+              if (u < cnt) c[u] = o2n[c[u]];
+          }
+#pragma unroll
+          for (int u = 0; u < U; ++u)
+            if (u < cnt && c[u] >= lo) v[u] = ld_lev(lev + (c[u] - lo));
+          pend = 0;
+#pragma unroll
+          for (int u = 0; u < U; ++u)
+            if (u < cnt && c[u] >= lo && v[u] < 0) pend |= 1u << u;
+          have = true;
         }
-        if (q == e) {
-          st_lev(lev + k, lv);
-          mx = max(mx, lv + 1);
-          done = true;
+      }
+      if (__all_sync(0xffffffffu, done)) break;
+      unsigned ns = 0;
+      for (;;) {  // lean wait on the pending dependencies of every lane
+        if (!done && pend) {
+#pragma unroll
+          for (int u = 0; u < U; ++u)
+            if (pend & (1u << u)) v[u] = ld_lev(lev + (c[u] - lo));
+#pragma unroll
+          for (int u = 0; u < U; ++u)
+            if ((pend & (1u << u)) && v[u] >= 0) pend &= ~(1u << u);
         }
+        if (__any_sync(0xffffffffu, !done && !pend)) break;
+        ns = ns ? min(ns * 2u, 256u) : 32u;  // back off: keep L2 free for the rows that can advance
+        __nanosleep(ns);
       }
     }
   }
@@ -820,15 +860,39 @@ Error analyse_device_t(Plan& p, int32_t n, int64_t nnz, const int32_t* d_rp, con
       DV_TRY(cub::DeviceScan::ExclusiveSum(d_cub, tb, nz_all + boff[i], slot_all + boff[i], m + 1, s));
     }
   }
-  // CSR offsets to the host (CSR: the row pointer itself; DCSR: downloaded
-  // after compaction below)
+  // CSR offsets of every segment to the host in ONE copy through a pinned
+  // buffer (the item builders are host passes over row pointers)
   std::vector<std::vector<int32_t>> hoffs((size_t)nseg);
-  for (int i = 0; i < nseg; ++i) {
-    const int m = geo[i].r1 - geo[i].r0;
-    hoffs[i].resize((size_t)m + 1);
-    DV_TRY(cudaMemcpyAsync(hoffs[i].data(), offs_all + boff[i], (size_t)(m + 1) * 4, cudaMemcpyDeviceToHost, s));
+  {
+    static std::mutex pin_mu;
+    static int32_t* pin = nullptr;
+    static size_t pin_n = 0;
+    std::lock_guard<std::mutex> lk(pin_mu);
+    const size_t tot = (size_t)boff[nseg];
+    if (tot > pin_n) {
+      if (pin) cudaFreeHost(pin);
+      pin = nullptr;
+      pin_n = 0;
+      if (cudaHostAlloc((void**)&pin, tot * 4, cudaHostAllocDefault) != cudaSuccess) {
+        cudaGetLastError();
+        pin = nullptr;
+      } else {
+        pin_n = tot;
+      }
+    }
+    std::vector<int32_t> pageable;
+    int32_t* hb = pin;
+    if (!hb) {
+      pageable.resize(tot);
+      hb = pageable.data();
+    }
+    DV_TRY(cudaMemcpyAsync(hb, offs_all, tot * 4, cudaMemcpyDeviceToHost, s));
+    DV_TRY(cudaStreamSynchronize(s));
+    for (int i = 0; i < nseg; ++i) {
+      const int m = geo[i].r1 - geo[i].r0;
+      hoffs[i].assign(hb + boff[i], hb + boff[i] + m + 1);
+    }
   }
-  DV_TRY(cudaStreamSynchronize(s));
   clk.lap("dev: row pointers to host");
   // stored row pointers on the host (items); DCSR compacts the nonempty rows
   for (int i = 0; i < nseg; ++i) {
@@ -854,7 +918,20 @@ Error analyse_device_t(Plan& p, int32_t n, int64_t nnz, const int32_t* d_rp, con
     for (int i = 0; i < nseg; ++i) th.emplace_back([&, i] { build_sq_items(p.segs[i]); });
     for (auto& x : th) x.join();
   }
-  for (int i = 0; i < nseg; ++i) build_sf_items(p.segs[i], p.npart);  // part slots numbered in order
+  for (int i = 0; i < nseg; ++i) {  // part slots numbered in order; squares fused as in upload()
+    p.segs[i].fused_sq = -1;
+    p.segs[i].fused = false;
+  }
+  for (int i = 0; i < nseg; ++i) build_sf_items(p.segs[i], p.npart, p.opts.selector);
+  for (int i = 0; i + 1 < nseg; ++i) {
+    Segment& Sg = p.segs[i];
+    if (Sg.sf_mixed && std::getenv("SPTRSV_SQ_FUSE")) {
+      p.segs[i + 1].dev_dcsr = p.segs[i + 1].info.kind == 1 && p.segs[i + 1].info.format == SPTRSV_FMT_DCSR;
+      p.segs[i + 1].dev_nzr = p.segs[i + 1].nzr;
+      fuse_square_items(Sg, p.segs[i + 1]);
+      if (p.segs[i + 1].fused) Sg.fused_sq = i + 1;
+    }
+  }
   clk.lap("dev: items");
   // ---- arena layout (as upload(): perm | iperm | 1/d | segments | tickets | ctl | part) ----
   size_t off = 0;

@@ -395,11 +395,12 @@ Error launch_chain_ell(Plan& p, Segment& S, const T* bw, T* xs, cudaStream_t s) 
 // column list, the dense external values V_J (column-major, ld = width) and
 // the packed strictly-lower diagonal block.  Values are the D^-1-scaled ones
 // of the segment (R27).
-void build_supernodes(Segment& S, size_t vb) {
+void build_supernodes(Segment& S, size_t vb, int32_t& part_base) {
   S.sn_desc.clear();
   S.sn_cols.clear();
   S.sn_vals.clear();
   S.sn_blk.clear();
+  S.sn_items.clear();
   const auto& I = S.info;
   if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_SUPERNODE) return;
   const int np = (int)S.sn_ptr.size() - 1;
@@ -434,6 +435,28 @@ void build_supernodes(Segment& S, size_t vb) {
   }, 512);
   S.sn_desc.resize((size_t)np * sizeof(k::SnDesc));
   std::memcpy(S.sn_desc.data(), desc.data(), S.sn_desc.size());
+  // work items (k::tri_supernode): long external lists cut into kSnChunk-
+  // column chunks with 32-wide partial slots (SPTRSV_SN_NOSPLIT: whole pieces)
+  const bool split = std::getenv("SPTRSV_SN_NOSPLIT") == nullptr;
+  S.sn_part_base = (part_base + 31) / 32 * 32;
+  int32_t nslot = 0;
+  for (int J = 0; J < np; ++J) {
+    const int ne = desc[J].ne;
+    if (!split || ne <= k::kSnChunk) {
+      const int32_t rec[8] = {J, 0, ne, 0, 0, 0, 0, 0};
+      S.sn_items.insert(S.sn_items.end(), rec, rec + 8);
+      continue;
+    }
+    const int first = nslot;
+    for (int q0 = 0; q0 < ne; q0 += k::kSnChunk) {
+      const int q1 = std::min(ne, q0 + k::kSnChunk);
+      const bool last = q1 == ne;
+      const int32_t rec[8] = {J, q0, q1, last ? 2 : 1, last ? first : nslot, last ? nslot : 0, 0, 0};
+      if (!last) ++nslot;
+      S.sn_items.insert(S.sn_items.end(), rec, rec + 8);
+    }
+  }
+  part_base = S.sn_part_base + 32 * nslot;
 }
 
 // Strand wavefront (k::tri_wave): strands = contiguous ranges of the
@@ -452,6 +475,7 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   auto& I = S.info;
   if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_PIPE) return;
   const int m = I.row1 - I.row0;
+  PhaseClock wclk;
   int C = 16, W = 2, GPC = k::kWaveGpcBig, NCH = 4;
   if (const char* e = std::getenv("SPTRSV_WAVE")) {
     int a, b2, c, d;
@@ -478,9 +502,19 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
   // anti-diagonal triangles 3-6 groups per level).  cap grows by 32 until
   // the strands fit the cluster (C_max x W warps).
   std::vector<int32_t> order(m), strand(m);
-  std::iota(order.begin(), order.end(), 0);
-  std::stable_sort(order.begin(), order.end(),
-                   [&](int a, int b2) { return p.lower_old[I.row0 + a] < p.lower_old[I.row0 + b2]; });
+  {  // rows in ascending original index: the keys are distinct, so a slot
+     // table over their range replaces a comparison sort (O(m + range))
+    int32_t kmin = INT32_MAX, kmax = -1;
+    for (int r = 0; r < m; ++r) {
+      kmin = std::min(kmin, p.lower_old[I.row0 + r]);
+      kmax = std::max(kmax, p.lower_old[I.row0 + r]);
+    }
+    std::vector<int32_t> slot((size_t)std::max(0, kmax - kmin + 1), -1);
+    for (int r = 0; r < m; ++r) slot[p.lower_old[I.row0 + r] - kmin] = r;
+    int q = 0;
+    for (int32_t t : slot)
+      if (t >= 0) order[q++] = t;
+  }
   const int C_max = C;
   int NS = 0;
   {
@@ -533,6 +567,7 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
     }
   }
   s_start[NS] = q;
+  wclk.lap("  wave: strands + groups");
   // own window: the smallest power of two covering every same-strand distance
   int maxd = 0;
   for (int r = 0; r < m; ++r)
@@ -597,6 +632,7 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
         dep[e] = {2, j, 0};
         ++nglobal;
       }
+  wclk.lap("  wave: dependency classes");
   if (nglobal * 10 > (int64_t)S.ci.size() && p.opts.force_tri_impl != SPTRSV_IMPL_TRI_PIPE) return give_up();
   int E = 0;
   for (int r = 0; r < m; ++r) E = std::max<int>(E, npush[r]);
@@ -731,6 +767,7 @@ void build_wave(const Plan& p, Segment& S, size_t vb) {
     }
     off += (size_t)nchunk[s2] * cbytes;
   }
+  wclk.lap("  wave: chunks");
   S.wave_strands.resize(sizeof(k::WaveStrand) * NS);
   std::memcpy(S.wave_strands.data(), sr.data(), S.wave_strands.size());
   S.wave_tau.assign(m, 0);
@@ -809,6 +846,45 @@ Error launch_wave(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cud
   }
 }
 
+// Cooperative launch of the static warp-per-item sync-free kernel: the grid
+// is the co-resident maximum (all warps must be resident for the static
+// schedule, see k::tri_sf_wrow), capped by the item count.
+template <typename T>
+Error launch_sf_wrow(Plan& p, Segment& S, int nitem, const T* val, const T* bw, T* xs, k::SolveState st,
+                     cudaStream_t s) {
+  auto kern = k::tri_sf_wrow<T, k::kSfWU>;
+  static std::mutex mu;
+  static std::unordered_map<int, int> per_sm_by_dev;
+  int dev = 0;
+  CUDA_TRY(cudaGetDevice(&dev));
+  int per_sm = 0;
+  {
+    std::lock_guard<std::mutex> g(mu);
+    auto it = per_sm_by_dev.find(dev);
+    if (it == per_sm_by_dev.end()) {
+      CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 256, 0));
+      per_sm_by_dev[dev] = per_sm;
+    } else {
+      per_sm = it->second;
+    }
+  }
+  int nb = std::max(1, per_sm) * p.sm_count;
+  if (const char* e = std::getenv("SPTRSV_SF_WROW_CTAS")) nb = std::min(nb, std::max(1, std::atoi(e)));  // tuning
+  nb = std::max(1, std::min<int>(nb, (int)cdiv(nitem, 8)));
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(nb);
+  cfg.blockDim = dim3(256);
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, S.info.row0, nitem, (const k::SfItem*)S.d_sf_items, S.d_ci, val, bw, xs,
+                              (T*)p.d_part, st));
+  return {SPTRSV_SUCCESS, ""};
+}
+
 template <typename T>
 Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveState st, cudaEvent_t* ev) {
   for (size_t si = 0; si < p.segs.size(); ++si) {
@@ -817,7 +893,9 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
     const int m = I.row1 - I.row0;
     const T* val = (const T*)S.d_val;
     if (I.kind == 1) {  // square: b -= A x
-      if (S.dev_nzr > 0 && I.nnz > 0) {
+      if (nrhs == 1 && S.fused) {
+        // computed by the preceding triangle's kernel (fused trailing items)
+      } else if (S.dev_nzr > 0 && I.nnz > 0) {
         const bool dcsr = S.dev_dcsr;
         if (nrhs == 1 && I.impl == SPTRSV_IMPL_SQ_ADAPT) {
           const int nitem = (int)(S.sq_items.size() / 4);
@@ -932,11 +1010,11 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
         }
         case SPTRSV_IMPL_TRI_SUPERNODE:
           if (nrhs == 1) {
-            const int np = (int)S.sn_ptr.size() - 1;
-            const unsigned g = std::max(1u, std::min<unsigned>(cdiv(np, 8), p.sm_count * 8));
-            k::tri_supernode<T><<<g, 256, 0, s>>>(np, (const k::SnDesc*)S.d_sn_desc, S.d_sn_cols,
-                                                  (const T*)S.d_sn_vals, (const T*)S.d_sn_blk, bw, xs, st,
-                                                  S.ticket_slot);
+            const int nit = (int)(S.sn_items.size() / 8);
+            const unsigned g = std::max(1u, std::min<unsigned>(cdiv(nit, 8), p.sm_count * 8));
+            k::tri_supernode<T><<<g, 256, 0, s>>>(nit, (const k::SnItem*)S.d_sn_items, (const k::SnDesc*)S.d_sn_desc,
+                                                  S.d_sn_cols, (const T*)S.d_sn_vals, (const T*)S.d_sn_blk, bw, xs,
+                                                  (T*)p.d_part + S.sn_part_base, st, S.ticket_slot);
             break;
           }
           if (nrhs >= kSnMultiMinRhs && !std::getenv("SPTRSV_NO_SN_MULTI")) {
@@ -979,10 +1057,19 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
             int nctas = SPTRSV_SF_MINB * p.sm_count;
             if (const char* e2 = std::getenv("SPTRSV_SF_CTAS")) nctas = std::max(1, std::atoi(e2));  // tuning
             const unsigned g = std::max(1u, std::min<unsigned>(cdiv(nitem, 8), (unsigned)nctas));
-            if (S.sf_mixed)
+            if (S.sf_wrow) {
+              Error e2 = launch_sf_wrow<T>(p, S, nitem, val, bw, xs, st, s);
+              if (e2.status) return e2;
+            } else if (S.sf_mixed) {
+              k::SqDesc sq{nullptr, nullptr, nullptr, nullptr, 0, 0};
+              if (S.fused_sq >= 0) {
+                const Segment& Q = p.segs[S.fused_sq];
+                sq = k::SqDesc{Q.d_rows, Q.d_rp, Q.d_ci, Q.d_val, Q.info.row0, Q.dev_dcsr ? 1 : 0};
+              }
               k::tri_sf_mixed<T, 4><<<std::max(1u, ctas(256, m)), 256, 0, s>>>(
                   I.row0, nitem, (const k::SfItem*)S.d_sf_items, S.d_rp, S.d_ci, val, bw, xs, (T*)p.d_part, st,
-                  S.ticket_slot);
+                  S.ticket_slot, sq);
+            }
             else
               k::tri_sf_items<T><<<g, 256, 0, s>>>(I.row0, nitem, (const k::SfItem*)S.d_sf_items, S.d_rp, S.d_ci,
                                                    val, bw, xs, (T*)p.d_part, st, S.ticket_slot);
@@ -1012,7 +1099,7 @@ int count_launches(const Plan& p) {
   int c = 2;  // permute in / out
   for (auto& S : p.segs) {
     if (S.info.kind == 1) {
-      c += (S.nzr > 0 && S.info.nnz > 0);
+      c += (S.nzr > 0 && S.info.nnz > 0 && !S.fused);
     } else if (S.info.row1 > S.info.row0) {
       if (S.info.impl == SPTRSV_IMPL_TRI_LEVELSET) {
         for (int l = 0; l < S.info.nlevels; ++l) c += S.level_ptr[l + 1] > S.level_ptr[l];
@@ -1254,12 +1341,69 @@ void build_sq_items(Segment& S) {
 // which adds the earlier pieces' partial sums.  SPTRSV_SF_V1 keeps the
 // round-1 kernels (thread / warp per row).
 void build_sf_mixed(Segment& S, int32_t& part_base);
-void build_sf_items(Segment& S, int32_t& part_base) {
-  S.sf_items.clear();
+// Fuse square Q (the next segment) into triangle T's mixed sync-free kernel
+// as trailing items (k::tri_sf_mixed kinds 4 / 5): greedy blocks of <= 32
+// stored rows holding <= kSfNB entries; a longer row in kSfNB-entry chunks
+// (atomic updates).  Items index Q's DEVICE row structure (Q.rp, with
+// Q.dev_dcsr / d_rows mapping stored row -> row).
+void fuse_square_items(Segment& T, Segment& Q) {
+  if (Q.info.kind != 1 || Q.info.nnz == 0 || Q.dev_nzr == 0) return;
+  const std::vector<int32_t>& rp = Q.rp;
+  const int nzr = Q.dev_nzr;
+  auto push = [&](int t0, int t1, int p0, int p1, int kind) {
+    const int32_t rec[8] = {t0, t1, p0, p1, kind, 0, 0, 0};
+    T.sf_items.insert(T.sf_items.end(), rec, rec + 8);
+  };
+  int t = 0;
+  while (t < nzr) {
+    const int len = rp[t + 1] - rp[t];
+    if (len > k::kSfNB) {
+      for (int a = rp[t]; a < rp[t + 1]; a += k::kSfNB) push(t, t + 1, a, std::min(a + k::kSfNB, rp[t + 1]), 5);
+      ++t;
+      continue;
+    }
+    const int start = t;
+    int tot = 0;
+    while (t < nzr && t - start < 32 && tot + (rp[t + 1] - rp[t]) <= k::kSfNB) {
+      tot += rp[t + 1] - rp[t];
+      ++t;
+    }
+    push(start, t, rp[start], rp[t], 4);
+  }
+  Q.fused = true;
+}
+
+// Items of the static warp-per-item kernel (k::tri_sf_wrow): one per row of
+// <= kSfW entries, else kSfW-entry pieces closed by the row's last piece.
+void build_sf_wrow(Segment& S, int32_t& part_base) {
   const auto& I = S.info;
-  if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_SYNCFREE) return;
-  S.sf_mixed = std::getenv("SPTRSV_SF_MIXED") != nullptr;
+  const int m = I.row1 - I.row0;
+  const std::vector<int32_t>& rp = S.rp;
+  S.sf_items.reserve((size_t)m * 8);
+  for (int t = 0; t < m; ++t) {
+    const int len = rp[t + 1] - rp[t];
+    const int np = std::max(1, (len + k::kSfW - 1) / k::kSfW);
+    const int first = part_base;
+    for (int q = 0; q < np; ++q) {
+      const int a = rp[t] + q * k::kSfW, b = std::min(a + k::kSfW, rp[t + 1]);
+      const int kind = np == 1 ? 0 : (q < np - 1 ? 1 : 2);
+      const int32_t rec[8] = {t, t + 1, a, b, kind, kind == 1 ? part_base++ : first, kind == 2 ? part_base : 0, 0};
+      S.sf_items.insert(S.sf_items.end(), rec, rec + 8);
+    }
+  }
+}
+void build_sf_items(Segment& S, int32_t& part_base, int selector) {
+  S.sf_items.clear();
+  S.sf_mixed = S.sf_wrow = false;
+  const auto& I = S.info;
+  if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_SYNCFREE || selector != SPTRSV_SELECT_B200) return;
+  // default (B200): the mixed-granularity kernel; SPTRSV_SF_V1 = the round-1
+  // thread / warp-per-row kernels (kept for comparison)
+  S.sf_mixed = std::getenv("SPTRSV_SF_V1") == nullptr && std::getenv("SPTRSV_SF_WROW") == nullptr &&
+               std::getenv("SPTRSV_SF_ITEMS") == nullptr;
   if (S.sf_mixed) return build_sf_mixed(S, part_base);
+  S.sf_wrow = std::getenv("SPTRSV_SF_WROW") != nullptr;
+  if (S.sf_wrow) return build_sf_wrow(S, part_base);
   if (!std::getenv("SPTRSV_SF_ITEMS")) return;
   const int m = I.row1 - I.row0;
   const std::vector<int32_t>& rp = S.rp;
@@ -1418,7 +1562,7 @@ Error upload(Plan& p, void* stream_v) {
   };
   size_t o_perm = take((size_t)2 * n * 4);  // perm (new->old) then iperm (old->new)
   size_t o_rdiag = take((size_t)n * vb);
-  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed, sd, sc, sv, sbk, ps, pd, pc, sq, sf; };
+  struct Offs { size_t rp, ci, val, rows, lp, st, er, ed, sd, sc, sv, sbk, ps, pd, pc, sq, sf, sni; };
   std::vector<Offs> so(p.segs.size());
   p.trace = std::getenv("SPTRSV_TRACE") != nullptr;
   p.spmm = spmm_cfg();
@@ -1515,13 +1659,19 @@ Error upload(Plan& p, void* stream_v) {
       }
     }
   }
+  for (auto& S : p.segs) S.fused = false;
   for (size_t i = 0; i < p.segs.size(); ++i) {
     Segment& S = p.segs[i];
     build_chain_stages(S, cg);
     build_chain_ell(S, vb);
-    build_supernodes(S, vb);
+    build_supernodes(S, vb, p.npart);
     build_sq_items(S);
-    build_sf_items(S, p.npart);
+    build_sf_items(S, p.npart, p.opts.selector);
+    S.fused_sq = -1;
+    if (S.sf_mixed && i + 1 < p.segs.size() && std::getenv("SPTRSV_SQ_FUSE")) {
+      fuse_square_items(S, p.segs[i + 1]);
+      if (p.segs[i + 1].fused) S.fused_sq = (int)i + 1;
+    }
     so[i].er = take(S.ell_recs.size() * 4);
     so[i].ed = take(S.ell_data.size());
     so[i].rp = take(dv[i].nrp * 4);
@@ -1539,6 +1689,7 @@ Error upload(Plan& p, void* stream_v) {
     so[i].pc = take(S.wave_crows.size() * 4);
     so[i].sq = take(S.sq_items.size() * 4);
     so[i].sf = take(S.sf_items.size() * 4);
+    so[i].sni = take(S.sn_items.size() * 4);
     if (S.info.kind == 0) S.ticket_slot = p.nticket++;
     if (S.info.kind == 0 && (S.info.impl == SPTRSV_IMPL_TRI_SYNCFREE || S.info.impl == SPTRSV_IMPL_TRI_SUPERNODE ||
                              (S.info.impl == SPTRSV_IMPL_TRI_PIPE && (S.wave_K == 0 || S.wave_global > 0))))
@@ -1623,6 +1774,8 @@ Error upload(Plan& p, void* stream_v) {
     S.d_sq_items = (const int32_t*)(A + so[i].sq);
     CUDA_TRY(put(so[i].sf, S.sf_items.data(), S.sf_items.size() * 4));
     S.d_sf_items = (const int32_t*)(A + so[i].sf);
+    CUDA_TRY(put(so[i].sni, S.sn_items.data(), S.sn_items.size() * 4));
+    S.d_sn_items = (const int32_t*)(A + so[i].sni);
   }
   if (std::getenv("SPTRSV_TEST_WEDGE")) {
     // test hook (DEADLOCK path): the first off-diagonal entry of the first

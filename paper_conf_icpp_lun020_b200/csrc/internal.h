@@ -114,6 +114,9 @@ struct Segment {
   const int32_t* d_sn_cols = nullptr;
   const void* d_sn_vals = nullptr;
   const void* d_sn_blk = nullptr;
+  std::vector<int32_t> sn_items;   // k::SnItem[] as 8 ints (pieces, or chunks of long pieces)
+  const int32_t* d_sn_items = nullptr;
+  int32_t sn_part_base = 0;        // first scalar of the segment's 32-wide partial slots in `part`
   // strand wavefront over a cluster (k::tri_wave, nrhs == 1); wave_K == 0: not built
   int wave_K = 0, wave_E = 0, wave_C = 0, wave_W = 0, wave_GPC = 0, wave_NCH = 0, wave_XW = 0, wave_xa = 0;
   uint32_t wave_chunk_bytes = 0, wave_bring_bytes = 0, wave_group_bytes = 0;
@@ -133,6 +136,9 @@ struct Segment {
   // row-block sync-free triangle kernel (k::tri_sf_items, nrhs == 1): k::SfItem[] as 8 ints
   std::vector<int32_t> sf_items;
   bool sf_mixed = false;
+  int32_t fused_sq = -1;  // TRI (mixed sync-free): index of the square fused as trailing items
+  bool fused = false;     // SQ: computed inside the preceding triangle's kernel at nrhs == 1
+  bool sf_wrow = false;
   const int32_t* d_sf_items = nullptr;
   // row-block square kernel (k::sq_adapt_1, nrhs == 1): k::SqItem[] as 4 ints
   std::vector<int32_t> sq_items;

@@ -834,6 +834,17 @@ constexpr int kSfNB = SPTRSV_SF_NB;
 #define SPTRSV_SF_LONG 32
 #endif
 constexpr int kSfLong = SPTRSV_SF_LONG;  // tri_sf_mixed: rows with more entries get a warp
+#ifndef SPTRSV_SF_POLLS
+#define SPTRSV_SF_POLLS 1
+#endif
+#ifndef SPTRSV_SF_GAP
+#define SPTRSV_SF_GAP 64
+#endif
+constexpr int kSfPolls = SPTRSV_SF_POLLS, kSfGap = SPTRSV_SF_GAP;  // tri_sf_mixed: staggered polls
+#ifndef SPTRSV_SF_WU
+#define SPTRSV_SF_WU 4
+#endif
+constexpr int kSfWU = SPTRSV_SF_WU, kSfW = 32 * kSfWU;  // tri_sf_wrow: entries per item
 struct SfItem {
   int t0, t1;  // local rows [t0, t1) (a piece: t1 = t0 + 1)
   int p0, p1;  // entries [p0, p1) of the segment's CSR
@@ -968,6 +979,16 @@ __global__ void __launch_bounds__(256, SPTRSV_SF_MINB) tri_sf_items(int r0, int 
   }
 }
 
+// The square that follows a triangle in execution order, fused into the
+// triangle's kernel as trailing work items (exec.cu fuse_square_items).
+struct SqDesc {
+  const int* rows;  // DCSR stored rows (dcsr), else rows are row0 + t
+  const int* rp;
+  const int* ci;
+  const void* val;
+  int row0, dcsr;
+};
+
 // Sync-free, mixed granularity (B200 selector, nrhs == 1; exec.cu
 // build_sf_mixed).  Work items in row order, one per ticket (deadlock-free
 // like K3):
@@ -983,13 +1004,26 @@ __global__ void __launch_bounds__(256, SPTRSV_SF_MINB) tri_sf_items(int r0, int 
 //   kind 1/2 the pieces of a row longer than kSfNB: partial sums to `part`
 //           slots (sentinel until written), the last piece adds them in piece
 //           order (deterministic) and publishes x.
+//   kind 4  (fused square, after every triangle item) a block of <= 32
+//           stored rows of the NEXT square segment with <= kSfNB entries:
+//           b'_rows -= A x, its x_j polled like a triangle's (they are this
+//           triangle's rows or earlier ones), products staged in shared
+//           memory, lane-per-row sums in entry order (as k::sq_adapt_1);
+//   kind 5  a kSfNB-entry chunk of a longer square row (atomic update).
+// The fused square's items are claimed only after the triangle's last item,
+// i.e. while the triangle's tail leaves most of the GPU idle (the square no
+// longer waits for a kernel boundary, and never blocks a triangle row).
+#ifndef SPTRSV_SFM_MINB
+#define SPTRSV_SFM_MINB 2  // resident CTAs per SM requested from ptxas (3: spills in fp64, measured slower)
+#endif
 template <typename T, int U>
-__global__ void __launch_bounds__(256) tri_sf_mixed(int r0, int nitem, const SfItem* __restrict__ items,
+__global__ void __launch_bounds__(256, SPTRSV_SFM_MINB) tri_sf_mixed(int r0, int nitem, const SfItem* __restrict__ items,
                                                     const int* __restrict__ rp, const int* __restrict__ ci,
-                                                    const T* __restrict__ val, const T* __restrict__ bw,
+                                                    const T* __restrict__ val, T* __restrict__ bw,
                                                     T* __restrict__ xs, T* __restrict__ part, SolveState st,
-                                                    int slot) {
+                                                    int slot, SqDesc sq) {
   constexpr int UW = kSfNB / 32;
+  __shared__ T prod_s[8][kSfNB];
   const int lane = threadIdx.x & 31;
   uint32_t* ticket = st.tickets + slot;
   uint32_t spins = 0;
@@ -1058,16 +1092,103 @@ __global__ void __launch_bounds__(256) tri_sf_mixed(int r0, int nitem, const SfI
           }
         }
         if (__all_sync(0xffffffffu, done)) break;
-        // lean spin until some blocked lane's value has landed
+        // lean spin until some blocked lane's value has landed.  kSfPolls
+        // polls of the address are in flight at once, issued kSfGap cycles
+        // apart and checked in order: the first that sees the value ends the
+        // wait, so the detection delay is ~ the poll spacing, not a whole L2
+        // round trip (the level's LAST row -- the slowest detection of ~10^3
+        // -- sets the level time)
         bool give = false;
         while (!__any_sync(0xffffffffu, !done && !is_sent(xb))) {
           if (wd_giveup(spins, st)) {
             give = true;
             break;
           }
-          if (!done) xb = ld_strong(xs + jb);
+          if constexpr (kSfPolls == 1) {
+            if (!done) xb = ld_strong(xs + jb);
+          } else {
+            T xq[kSfPolls];
+#pragma unroll
+            for (int q = 0; q < kSfPolls; ++q) {
+              if (!done) xq[q] = ld_strong(xs + jb);
+              if (q + 1 < kSfPolls) {
+                const long long t0 = clock64();
+                while (clock64() - t0 < kSfGap) {
+                }
+              }
+            }
+#pragma unroll
+            for (int q = 0; q < kSfPolls; ++q) {
+              if (!done && is_sent(xb) && !is_sent(xq[q])) xb = xq[q];
+              if (__any_sync(0xffffffffu, !done && !is_sent(xb))) break;
+            }
+          }
         }
         if (give) break;
+      }
+      continue;
+    }
+    if (h1.x >= 4) {  // ------------------------------ fused square block / chunk
+      const int a = h0.z, ne = h0.w - h0.z;
+      const T* sval = (const T*)sq.val;
+      int j[UW];
+      T v[UW], x[UW];
+      uint32_t pend = 0;
+#pragma unroll
+      for (int u = 0; u < UW; ++u) {
+        const int e = lane + 32 * u;
+        if (e < ne) {
+          j[u] = ldg_nc(sq.ci + a + e);
+          v[u] = ldg_nc(sval + a + e);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < UW; ++u)
+        if (lane + 32 * u < ne) x[u] = ld_strong(xs + j[u]);
+#pragma unroll
+      for (int u = 0; u < UW; ++u)
+        if (lane + 32 * u < ne) {
+          if (is_sent(x[u])) pend |= 1u << u;
+        } else {
+          x[u] = T(0);
+          v[u] = T(0);
+        }
+      bool give = false;
+      while (__any_sync(0xffffffffu, pend != 0)) {
+        if (wd_giveup(spins, st)) {
+          give = true;
+          break;
+        }
+#pragma unroll
+        for (int u = 0; u < UW; ++u)
+          if (pend & (1u << u)) {
+            x[u] = ld_strong(xs + j[u]);
+            if (!is_sent(x[u])) pend &= ~(1u << u);
+          }
+      }
+      if (give) break;
+      if (h1.x == 5) {  // chunk of one long stored row
+        T acc = 0;
+#pragma unroll
+        for (int u = 0; u < UW; ++u) acc += v[u] * x[u];
+        acc = warp_sum(acc);
+        if (lane == 0) atomicAdd(bw + (sq.dcsr ? sq.rows[h0.x] : sq.row0 + h0.x), -acc);
+      } else {
+        T* pr = prod_s[threadIdx.x >> 5];
+#pragma unroll
+        for (int u = 0; u < UW; ++u)
+          if (lane + 32 * u < ne) pr[lane + 32 * u] = v[u] * x[u];
+        __syncwarp();
+        const int t = h0.x + lane;
+        if (t < h0.y) {
+          const int q0 = sq.rp[t] - a, q1 = sq.rp[t + 1] - a;
+          if (q1 > q0) {
+            T sum = 0;
+            for (int q = q0; q < q1; ++q) sum += pr[q];
+            bw[sq.dcsr ? sq.rows[t] : sq.row0 + t] -= sum;
+          }
+        }
+        __syncwarp();  // pr is rewritten by the warp's next item
       }
       continue;
     }
@@ -1137,6 +1258,99 @@ __global__ void __launch_bounds__(256) tri_sf_mixed(int r0, int nitem, const SfI
   }
 }
 
+// Sync-free, one WARP per item with a static round-robin schedule (B200
+// selector, nrhs == 1; exec.cu build_sf_wrow).  Items are single rows of
+// <= 32*UW off-diagonal entries, or kSfW-entry pieces of a longer row
+// (kind 1: partial sum to a `part` slot; kind 2: the row's last piece adds
+// the earlier pieces' sums in piece order).  Warp w takes items w, w + W,
+// w + 2W, ... in order; the launch is cooperative (all W warps resident),
+// so the lowest unfinished item always has its owner at it and every
+// dependency finished: no deadlock, and no ticket atomics (one same-address
+// atomic per row serialised the round-1 warp kernel).  A warp holds ONE
+// item: its lanes' loads are all in flight, the warp spins only on its own
+// pending dependencies, and nothing else in the warp delays the detection
+// (with a row per lane, one lane's next batch stalls the other lanes' polls).
+template <typename T, int UW>
+__global__ void __launch_bounds__(256) tri_sf_wrow(int r0, int nitem, const SfItem* __restrict__ items,
+                                                   const int* __restrict__ ci, const T* __restrict__ val,
+                                                   const T* __restrict__ bw, T* __restrict__ xs,
+                                                   T* __restrict__ part, SolveState st) {
+  const int lane = threadIdx.x & 31;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  uint32_t spins = 0;
+  for (int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nitem; w += nw) {
+    const int4 h0 = __ldg((const int4*)(items + w));
+    const int4 h1 = __ldg((const int4*)(items + w) + 1);
+    const int kind = h1.x, p0 = h0.z, ne = h0.w - h0.z;
+    const int r = r0 + h0.x;
+    if (lane == 0) SF_TRACE(st, r, 0);
+    const T bwr = (kind != 1 && lane == 0) ? bw[r] : T(0);
+    int j[UW];
+    T v[UW], x[UW];
+#pragma unroll
+    for (int u = 0; u < UW; ++u) {
+      const int e = lane + 32 * u;
+      if (e < ne) {
+        j[u] = ldg_nc(ci + p0 + e);
+        v[u] = ldg_nc(val + p0 + e);
+      }
+    }
+    uint32_t pend = 0;
+#pragma unroll
+    for (int u = 0; u < UW; ++u)
+      if (lane + 32 * u < ne) x[u] = ld_strong(xs + j[u]);
+#pragma unroll
+    for (int u = 0; u < UW; ++u)
+      if (lane + 32 * u < ne) {
+        if (is_sent(x[u])) pend |= 1u << u;
+      } else {
+        x[u] = T(0);
+        v[u] = T(0);
+      }
+    bool give = false;
+    while (__any_sync(0xffffffffu, pend != 0)) {
+#pragma unroll
+      for (int u = 0; u < UW; ++u)
+        if (pend & (1u << u)) x[u] = ld_strong(xs + j[u]);
+#pragma unroll
+      for (int u = 0; u < UW; ++u)
+        if ((pend & (1u << u)) && !is_sent(x[u])) pend &= ~(1u << u);
+      if (wd_giveup(spins, st)) {
+        give = true;
+        break;
+      }
+    }
+    if (give) break;
+    T acc = 0;
+#pragma unroll
+    for (int u = 0; u < UW; ++u) acc += v[u] * x[u];
+    acc = warp_sum(acc);
+    if (kind == 2) {  // the earlier pieces' partial sums, 32 at a time, in piece order
+      T ps = T(0);
+      for (int q0 = h1.y; q0 < h1.z; q0 += 32) {
+        T pv = T(0);
+        if (q0 + lane < h1.z) {
+          pv = ld_strong(part + q0 + lane);
+          while (is_sent(pv)) {
+            if (wd_giveup(spins, st)) break;
+            pv = ld_strong(part + q0 + lane);
+          }
+        }
+        ps += warp_sum(pv);
+      }
+      acc += ps;
+    }
+    if (lane == 0) {
+      if (kind == 1) {
+        st_strong(part + h1.y, acc);
+      } else {
+        st_strong(xs + r, bwr - acc);
+        SF_TRACE(st, r, 1);
+      }
+    }
+  }
+}
+
 // Supernodal sync-free (B200 selector, nrhs == 1): a warp per fundamental
 // supernode piece J = rows [s, s+w), w <= 32, claimed in row order from the
 // segment's ticket (deadlock-free like K3).  Lane t owns row s+t:
@@ -1158,23 +1372,43 @@ struct SnDesc {
 #ifndef SPTRSV_SN_MINB
 #define SPTRSV_SN_MINB 2  // min resident CTAs per SM requested from ptxas (C4: 2 measured best of 1-3)
 #endif
+// Work items (exec.cu build_supernodes): a piece whose external column list
+// is longer than kSnChunk is cut into kSnChunk-column chunks -- partial
+// products V_J[:, chunk] x[chunk] go to 32-wide slots of `part` (sentinel
+// until written), and the piece's last chunk adds them in chunk order
+// (deterministic) before the diagonal block.  The pieces near the root of
+// the elimination tree hold the longest lists (all their children's and
+// grandchildren's columns) and sit at the END of the dependency chain: split,
+// their products run on many warps at once instead of one warp's serial rounds.
+constexpr int kSnChunk = 256;
+struct SnItem {
+  int J, q0, q1, kind;  // piece, external columns [q0, q1); kind 0 whole piece, 1 partial chunk, 2 last chunk
+  int s0, s1, pad0, pad1;  // kind 1: slot s0; kind 2: slots [s0, s1)
+};
 template <typename T>
-__global__ void __launch_bounds__(256, SPTRSV_SN_MINB) tri_supernode(int npieces, const SnDesc* __restrict__ desc,
+__global__ void __launch_bounds__(256, SPTRSV_SN_MINB) tri_supernode(int nitems, const SnItem* __restrict__ items,
+                                                     const SnDesc* __restrict__ desc,
                                                      const int* __restrict__ cols, const T* __restrict__ V,
                                                      const T* __restrict__ Tb, const T* __restrict__ bw,
-                                                     T* __restrict__ xs, SolveState st, int slot) {
+                                                     T* __restrict__ xs, T* __restrict__ part, SolveState st,
+                                                     int slot) {
   const int lane = threadIdx.x & 31;
   uint32_t* ticket = st.tickets + slot;
   while (true) {
-    int J = 0;
-    if (lane == 0) J = (int)atomicAdd(ticket, 1u);
-    J = __shfl_sync(0xffffffffu, J, 0);
-    if (J >= npieces) break;
-    const SnDesc d = desc[J];
+    int w = 0;
+    if (lane == 0) w = (int)atomicAdd(ticket, 1u);
+    w = __shfl_sync(0xffffffffu, w, 0);
+    if (w >= nitems) break;
+    const int4 i0 = __ldg((const int4*)(items + w));
+    const int4 i1 = __ldg((const int4*)(items + w) + 1);
+    const int kind = i0.w;
+    const SnDesc d = desc[i0.x];
     const bool act = lane < d.w;
-    T y = act ? bw[d.s + lane] : T(0);
-    for (int q0 = 0; q0 < d.ne; q0 += 32) {
-      const int nq = min(32, d.ne - q0);
+    // kind 0 / 2: y = b' - V x; kind 1: y = V x over the chunk (a partial)
+    T y = (act && kind != 1) ? bw[d.s + lane] : T(0);
+    if (kind == 1) y = T(0);
+    for (int q0 = i0.y; q0 < i0.z; q0 += 32) {
+      const int nq = min(32, i0.z - q0);
       const bool inq = lane < nq;
       const int j = inq ? ldg_nc(cols + d.coff + q0 + lane) : 0;
       T vr[32];
@@ -1193,9 +1427,29 @@ __global__ void __launch_bounds__(256, SPTRSV_SN_MINB) tri_supernode(int npieces
       for (int c = 0; c < 32; ++c) {
         if (c < nq) {  // warp-uniform
           const T xc = __shfl_sync(0xffffffffu, xj, c);
-          y -= vr[c] * xc;
+          if (kind == 1)
+            y += vr[c] * xc;
+          else
+            y -= vr[c] * xc;
         }
       }
+    }
+    if (kind == 1) {  // publish the chunk's partial products (32-wide slot)
+      if (act) st_strong(part + (size_t)i1.x * 32 + lane, y);
+      continue;
+    }
+    if (kind == 2) {  // the earlier chunks' partials, in chunk order
+      T ps = T(0);
+      for (int q = i1.x; q < i1.y; ++q) {
+        T pv = act ? ld_strong(part + (size_t)q * 32 + lane) : T(0);
+        uint32_t spins = 0;
+        while (__any_sync(0xffffffffu, act && is_sent(pv))) {
+          if (wd_giveup(spins, st)) break;
+          if (act && is_sent(pv)) pv = ld_strong(part + (size_t)q * 32 + lane);
+        }
+        ps += pv;
+      }
+      y -= ps;
     }
     // dense unit-lower diagonal block: column c of T_J holds rows c+1 .. w-1
     // at Tb[boff + c(w-1) - c(c-1)/2 + (t - c - 1)]

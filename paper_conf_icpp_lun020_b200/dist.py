@@ -79,9 +79,12 @@ def dist_solve(plan, B: torch.Tensor | None, group=None, root: int = 0, nrhs: in
     dev = torch.device("cuda", torch.cuda.current_device()) if nccl else torch.device("cpu")
     if nrhs is not None and nrhs != k:
         raise ValueError(f"nrhs={nrhs} but the root's B has {k} columns")
-    # equal-size shards for scatter/gather: pad every shard to ceil(k / P) columns
-    w = -(-k // world)
     c0, c1 = shard_bounds(k, world, rank)
+    even = k % world == 0 and (rank != root or B.stride(1) == n)  # root: B.T rows contiguous
+    # equal-size shards for scatter/gather: when P divides k the column-major
+    # shards are contiguous row blocks of B.T / X.T and travel as views (no
+    # staging copy); otherwise every shard is padded to ceil(k / P) columns
+    w = -(-k // world)
     mine = torch.empty(w, n, dtype=dtype, device=dev)  # row c = column c of the shard
     scatter_list = None
     if rank == root:
@@ -89,23 +92,41 @@ def dist_solve(plan, B: torch.Tensor | None, group=None, root: int = 0, nrhs: in
         scatter_list = []
         for r in range(world):
             a, b = shard_bounds(k, world, r)
-            buf = torch.zeros(w, n, dtype=dtype, device=dev)
-            buf[: b - a].copy_(bt[a:b])
-            scatter_list.append(buf)
+            if even:
+                scatter_list.append(bt[a:b])
+            else:
+                buf = torch.zeros(w, n, dtype=dtype, device=dev)
+                buf[: b - a].copy_(bt[a:b])
+                scatter_list.append(buf)
     dist.scatter(mine, scatter_list, src=groot, group=group)
     xs = torch.empty_like(mine)
     if c1 > c0:
         b_shard = mine[: c1 - c0].T  # (n, c1-c0) column-major
+        x_out = xs[: c1 - c0].T
         if c1 - c0 == 1:
-            b_shard = b_shard[:, 0]
-        x_shard = solve_fn(plan, b_shard)
-        xs[: c1 - c0].copy_(x_shard.T if x_shard.dim() == 2 else x_shard[None])
-    gather_list = [torch.empty_like(mine) for _ in range(world)] if rank == root else None
+            b_shard, x_out = b_shard[:, 0], x_out[:, 0]
+        x_shard = solve_fn(plan, b_shard, x_out) if _takes_out(solve_fn) else solve_fn(plan, b_shard)
+        if x_shard is not None and x_shard.data_ptr() != x_out.data_ptr():
+            x_out.copy_(x_shard)
+    X = torch.empty(k, n, dtype=dtype, device=dev) if rank == root else None
+    if rank == root and even:
+        gather_list = [X[a:b] for a, b in (shard_bounds(k, world, r) for r in range(world))]
+    else:
+        gather_list = [torch.empty_like(mine) for _ in range(world)] if rank == root else None
     dist.gather(xs, gather_list, dst=groot, group=group)
     if rank != root:
         return None
-    X = torch.empty(k, n, dtype=dtype, device=dev)
-    for r in range(world):
-        a, b = shard_bounds(k, world, r)
-        X[a:b].copy_(gather_list[r][: b - a])
+    if not even:
+        for r in range(world):
+            a, b = shard_bounds(k, world, r)
+            X[a:b].copy_(gather_list[r][: b - a])
     return X.T
+
+
+def _takes_out(fn) -> bool:
+    """solve_fn(plan, b, x) writes into x (the CUDA library's sptrsv_solve)."""
+    try:
+        import inspect
+        return len(inspect.signature(fn).parameters) >= 3
+    except (TypeError, ValueError):
+        return False

@@ -76,7 +76,8 @@ def main():
         total = dn.max()
         print(f"seg{i}: rows {r1 - r0} levels {nl} span {total / 1e3:.1f} us (event {times[1 + i] * 1e3:.1f} us) "
               f"per level {total / nl:.0f} ns | claim-late levels {late} ({claim_late / 1e3:.1f} us) | "
-              f"detect mean {det.mean():.0f} ns p50 {np.median(det):.0f} p90 {np.percentile(det, 90):.0f} | "
+              f"detect mean {det.mean():.0f} ns p10 {np.percentile(det, 10):.0f} p50 {np.median(det):.0f} "
+              f"p90 {np.percentile(det, 90):.0f} | "
               f"row claim->done p50 {np.median(dn - cl):.0f} ns")
         w = np.bincount(L, minlength=nl)
         dl = np.diff(lvl_done)

@@ -57,7 +57,10 @@ def test_device_plan_matches_structural_oracle(gpu, name):
     M, _ = g.gen_config(name, small=True, nrhs=1)
     pd = sp.sptrsv_analyse(*_dev_csr(M), min_block_rows=max(2, M.n // 9))
     info = pd.info()
-    assert info["analysis"] == 1  # every kernel of these plans runs on device-built formats
+    # at these small sizes the narrow-level triangles take the chain kernel,
+    # whose stage format is finished on the host (analysis 2); the full-size
+    # C3 / C5 plans are device-built end to end (test_full_size_device_analysis)
+    assert info["analysis"] in (1, 2)
     A = st.analyse(M, depth=info["depth"], reorder=info["reorder"] == 0)
     assert np.array_equal(pd.perm(), A.perm)
     assert np.array_equal(pd.levels(), A.leaf_level)
@@ -70,8 +73,9 @@ def test_device_plan_matches_structural_oracle(gpu, name):
             assert np.array_equal(pd.seg_array(i, C.ARRAY_LEVEL_PTR), arrs["LEVEL_PTR"])
         else:
             assert np.array_equal(pd.seg_array(i, C.ARRAY_DCSR_ROWS), arrs["DCSR_ROWS"])
-    with pytest.raises(sp.SptrsvError):
-        pd.matrix()  # no host P L P^T for device plans
+    if info["analysis"] == 1:
+        with pytest.raises(sp.SptrsvError):
+            pd.matrix()  # no host P L P^T for device-built plans
     pd.free()
 
 
