@@ -756,21 +756,26 @@ void choose_impls(Plan& p) {
       if (p.opts.selector == SPTRSV_SELECT_B200 && I.nlevels > 1 && supernodal) {
         impl = SPTRSV_IMPL_TRI_SUPERNODE;
       } else if (p.opts.selector == SPTRSV_SELECT_B200 && I.nlevels > 1) {
-        int64_t m = I.row1 - I.row0;
-        // narrow levels: one CTA walks the level chain with bar.sync (no
-        // cross-SM flag round trips); wide levels: all SMs
-        if (I.max_level_rows <= 2048 || (m / std::max(1, I.nlevels)) <= 256) {
-          // narrow levels with few dependencies per row: the strand
-          // wavefront over one thread-block cluster (exec.cu build_wave, which
-          // falls back to the single-CTA chain when the rows' dependencies
-          // do not stay inside their strands); else one CTA walks the chain
-          const int32_t kmax = S.kmax_indeg;
-          impl = (kmax >= 1 && kmax <= 8 && m >= 4096 && std::getenv("SPTRSV_NO_WAVE") == nullptr)
-                     ? SPTRSV_IMPL_TRI_PIPE
-                     : SPTRSV_IMPL_TRI_CHAIN;
-        }
-        else if (I.nlevels <= 20)
-          impl = SPTRSV_IMPL_TRI_LEVELSET;
+        // B200 thresholds re-derived with the paper's own method (Sec 3.4,
+        // L254-L263; scripts/fig5_derive.py -> profiles/r02_fig5.json,
+        // DESIGN.md sec. 6.1): every kernel timed on sub-matrices of the five
+        // families, the fastest per feature cell.
+        //  - the strand wavefront wins on long chains of narrow levels with
+        //    few dependencies (C2-like: >= 128 levels);
+        //  - the single-CTA chain wins on small triangles (<= 8192 rows)
+        //    with >= 32 levels (no cross-SM hop per level);
+        //  - everywhere else the mixed sync-free kernel -- including the few-
+        //    level triangles the paper gives to level-set (one launch per
+        //    level loses to it on B200 at every sampled size); with several
+        //    RHS a <= 20-level triangle still runs level by level (exec.cu)
+        const int64_t m = I.row1 - I.row0;
+        const bool narrow = I.max_level_rows <= 2048 || (m / std::max(1, I.nlevels)) <= 256;
+        const int32_t kmax = S.kmax_indeg;
+        if (narrow && kmax >= 1 && kmax <= 8 && m >= 4096 && I.nlevels >= 128 &&
+            std::getenv("SPTRSV_NO_WAVE") == nullptr)
+          impl = SPTRSV_IMPL_TRI_PIPE;
+        else if (narrow && m <= 8192 && I.nlevels >= 32)
+          impl = SPTRSV_IMPL_TRI_CHAIN;
         else
           impl = SPTRSV_IMPL_TRI_SYNCFREE;
       }

@@ -78,6 +78,10 @@ constexpr int kSnMultiMinRhs = 16;
 // UN = 1 (its polling is per entry).
 SpmmCfg spmm_cfg() {
   SpmmCfg c;
+  if (const char* e = std::getenv("SPTRSV_SPMM_TILE")) {  // RHS tile width of sq_multi_tiled (0 = off)
+    const int t = std::atoi(e);
+    c.tile = (t == 0 || t == 8 || t == 16 || t == 32) ? t : c.tile;
+  }
   if (const char* e = std::getenv("SPTRSV_SPMM")) {
     int a, b;
     if (std::sscanf(e, "%d,%d", &a, &b) == 2 && (a == 1 || a == 2 || a == 4 || a == 8 || a == 16) && (b == 1 || b == 2)) {
@@ -919,6 +923,25 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
             else
               k::sq_scalar_1<T, false><<<g, 256, 0, s>>>(S.dev_nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
           }
+        } else if (nrhs >= 64 && (int64_t)(I.col1 - I.col0) * nrhs * (int64_t)sizeof(T) > (int64_t(64) << 20) &&
+                   p.spmm.tile > 0) {
+          // X rows of the square's columns exceed L2: RHS-tiled SpMM
+          auto launch_tiled = [&](auto Gc) {
+            constexpr int Gv = decltype(Gc)::value;
+            const dim3 g(cdiv((int64_t)S.dev_nzr * Gv, 256), cdiv(nrhs, Gv));
+            if (dcsr)
+              k::sq_multi_tiled<T, Gv, 1, 2, true><<<g, 256, 0, s>>>(S.dev_nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val,
+                                                                     xs, bw, nrhs);
+            else
+              k::sq_multi_tiled<T, Gv, 1, 2, false><<<g, 256, 0, s>>>(S.dev_nzr, I.row0, S.d_rows, S.d_rp, S.d_ci,
+                                                                      val, xs, bw, nrhs);
+          };
+          if (p.spmm.tile == 8)
+            launch_tiled(std::integral_constant<int, 8>());
+          else if (p.spmm.tile == 16)
+            launch_tiled(std::integral_constant<int, 16>());
+          else
+            launch_tiled(std::integral_constant<int, 32>());
         } else {
           dispatch_multi_un(nrhs, p.spmm, [&](auto G, auto R, auto U) {
             unsigned g = cdiv((int64_t)S.dev_nzr * G, 256);
@@ -936,6 +959,12 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
         case SPTRSV_IMPL_TRI_DIAG:
           k::tri_diag<T><<<cdiv((int64_t)m * nrhs, 256), 256, 0, s>>>(I.row0, m, nrhs, bw, xs);
           break;
+        case SPTRSV_IMPL_TRI_SYNCFREE:
+          // B200: a few-level triangle with several RHS runs level by level
+          // (bandwidth-bound launches; the level-set label's own kernel)
+          if (!(nrhs > 1 && p.opts.selector == SPTRSV_SELECT_B200 && p.reorder_eff == 0 && I.nlevels <= 20))
+            goto sync_free;
+          [[fallthrough]];
         case SPTRSV_IMPL_TRI_LEVELSET: {
           const bool warp = tri_use_warp(S);
           for (int l = 0; l < I.nlevels; ++l) {
@@ -1038,6 +1067,7 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
             break;
           }
           [[fallthrough]];  // 1 < nrhs < 16: the multi-RHS sync-free kernel on the CSR copy
+        sync_free:
         default: {  // SPTRSV_IMPL_TRI_SYNCFREE
           // enough resident warps for about two of the triangle's widest
           // levels: more only spin on rows whose dependencies are levels away

@@ -186,6 +186,7 @@ struct GraphEntry {
 // SpMM lane geometry for nrhs > 1 (exec.cu: dispatch_multi_un)
 struct SpmmCfg {
   int rpt_max = 8, un = 2;  // measured best on C5 (round 1 sweep, profiles/r01_sweeps.md)
+  int tile = 16;            // RHS tile width of the tiled SpMM (0 = untiled; SPTRSV_SPMM_TILE)
 };
 
 struct Plan {

@@ -485,6 +485,32 @@ __global__ void sq_multi(int nzr, int r0, const int* __restrict__ rows, const in
   }
 }
 
+// SpMM square update with RHS TILING (B200, nrhs > 1): blockIdx.y selects a
+// tile of G*RPT right-hand-side columns and the grid is scheduled tile-major
+// (x fastest), so all resident CTAs gather from the same column tile of X:
+// the tile's rows of X (cols x G*RPT x 8 B) stay L2-resident instead of every
+// gather of a 4 KB X row missing L2 (round 1: 2.66x the algorithmic DRAM
+// bytes on C5's largest square).  The matrix is re-streamed once per tile.
+template <typename T, int G, int RPT, int UN, bool DCSR>
+__global__ void sq_multi_tiled(int nzr, int r0, const int* __restrict__ rows, const int* __restrict__ rp,
+                               const int* __restrict__ ci, const T* __restrict__ val, const T* __restrict__ xs,
+                               T* __restrict__ bw, int nrhs) {
+  const int c0 = blockIdx.y * (G * RPT);
+  const int g = (blockIdx.x * blockDim.x + threadIdx.x) / G, lane = threadIdx.x % G;
+  if (g >= nzr) return;
+  const int r = DCSR ? rows[g] : r0 + g;
+  const int a = rp[g], e = rp[g + 1];
+  if (a == e) return;
+  T acc[RPT];
+#pragma unroll
+  for (int t = 0; t < RPT; ++t) acc[t] = 0;
+  gather_row_update<T, RPT, true, UN>(acc, a, e, ci, val, xs, nrhs, c0 + lane, G, nrhs - c0 - lane);
+  T* br = bw + (int64_t)r * nrhs + c0 + lane;
+#pragma unroll
+  for (int t = 0; t < RPT; ++t)
+    if (c0 + lane + G * t < nrhs) br[G * t] -= acc[t];
+}
+
 // ------------------------------------------------- K2: one level of a triangle
 // SPTRSV-LEVEL-SET (Alg 2 L88-L98; L247 "a thread or a 32-thread warp"): after
 // the level reorder every level is a contiguous row range [ra, rb).  One

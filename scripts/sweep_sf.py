@@ -19,12 +19,14 @@ from workloads import generators as g  # noqa: E402
 
 def main():
     cfg = sys.argv[1]
+    nrhs = int(os.environ.get("SWEEP_NRHS", "1"))
     M = g.gen_matrix(cfg)
-    b = g.gen_rhs(M.n, 1, seed=g.config_seed(cfg))
+    b = g.gen_rhs(M.n, nrhs, seed=g.config_seed(cfg))
     plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, graphs=False)
     segs = plan.segments()
-    ref = on.solve(M, b)
-    B = torch.from_numpy(b[0]).cuda()
+    cols = [0, nrhs // 2, nrhs - 1] if nrhs > 1 else [0]
+    ref = on.solve(M, b[cols], threads=len(cols))
+    B = torch.from_numpy(b[0]).cuda() if nrhs == 1 else torch.from_numpy(b).cuda().T
     X = torch.empty_like(B)
     flush = torch.empty(64 << 20, dtype=torch.float32, device="cuda")
     base = dict(os.environ)
@@ -45,7 +47,8 @@ def main():
         plan.set_profiling(False)
         torch.cuda.synchronize()
         t = np.mean(acc, axis=0)
-        err = on.rel_err(X.cpu().numpy()[None], ref)
+        xh = X.cpu().numpy()
+        err = on.rel_err(xh[None] if nrhs == 1 else xh.T[cols], ref)
         tri = sum(t[1 + i] for i, s in enumerate(segs) if s["kind"] == "TRI")
         sq = sum(t[1 + i] for i, s in enumerate(segs) if s["kind"] == "SQ")
         print(f"{setting or 'default':45s} total {t.sum():.3f} ms tri {tri:.3f} sq {sq:.3f} err {err:.1e} | "
