@@ -203,6 +203,28 @@ sptrsv_status_t sptrsv_analyse(int32_t n, int64_t nnz, const int32_t* row_ptr, c
 sptrsv_status_t sptrsv_solve(sptrsv_plan_t plan, const void* b, int64_t ldb, void* x, int64_t ldx,
                              int32_t nrhs, sptrsv_layout_t layout, void* stream);
 
+/*
+ * Solve A^T x = b with the plan of A (the preconditioner's
+ * transposed sweep, PAPER.md:L33/L35 -- IC(0) applies L^{-T} L^{-1}), from
+ * the SAME plan: no second analysis, no transposed copy of the matrix.
+ * The plan stores L1 = D^-1 P A P^T (unit lower, R27), so
+ * A^T x = b  <=>  L1^T z = P b, x = P^T D^-1 z.  L1^T is solved over the
+ * plan's segments in reverse order with the push form of the sync-free solve
+ * (Alg 3: in-degree counters decremented with atomics, left_sum
+ * updated with atomicAdd; R32), squares as b_C -= S^T z_R with
+ * atomics.  Summation order therefore varies run to run (reading R22).
+ *   b, ldb, x, ldx, layout: as sptrsv_solve; nrhs must be 1 (NOT_SUPPORTED
+ *   otherwise); b and x are DEVICE pointers on the plan's device
+ *   (NOT_SUPPORTED for host pointers, INVALID_VALUE for another device).
+ *   b == x is allowed.  Stream-ordered and asynchronous; never captured into
+ *   a graph by the library.  The first call allocates 8n + 4*nseg bytes of
+ *   counters (through dev_alloc when given) and builds them on the device.
+ * A plan analysed with opts.transpose = 1 solves (A^T)^T = A here.
+ * Errors: INVALID_VALUE, NOT_SUPPORTED, ALLOC, CUDA, DEADLOCK.
+ */
+sptrsv_status_t sptrsv_solve_transposed(sptrsv_plan_t plan, const void* b, int64_t ldb, void* x, int64_t ldx,
+                                        int32_t nrhs, sptrsv_layout_t layout, void* stream);
+
 /* Release the plan.  Waits for the plan's last solve (an event recorded on
  * that solve's stream) -- not for the whole device -- then returns every
  * device allocation (through dev_free when given).  NULL is a no-op. */

@@ -279,12 +279,14 @@ def _layout(t, n):
     return None
 
 
-def sptrsv_solve(plan: Plan, b, x=None, stream=None):
+def sptrsv_solve(plan: Plan, b, x=None, stream=None, transposed: bool = False):
     """Solve with b of shape (n,) or (n, k) (any of column-/row-major strides).
 
     b on the GPU (torch): asynchronous on the given (or current torch) stream.
     b on the host (numpy or CPU torch): copied in, solved, copied back (blocking).
     Returns x (allocated like b when not given).  x may be b (in place).
+    transposed=True solves A^T x = b with the same plan (C ABI
+    sptrsv_solve_transposed: one RHS, device tensors only).
     """
     n = plan.n
     if b.shape[0] != n:
@@ -315,8 +317,9 @@ def sptrsv_solve(plan: Plan, b, x=None, stream=None):
     if lx is None or lx[0] != lb[0] or lx[1] != lb[1]:
         raise ValueError("x must have the shape and the layout of b")
     layout, nrhs, ldb = lb
-    st = C.lib().sptrsv_solve(plan._h, _ptr(b), ldb, _ptr(x), lx[2], nrhs, layout, _stream_handle(stream))
-    C.check(st, "sptrsv_solve")
+    fn = C.lib().sptrsv_solve_transposed if transposed else C.lib().sptrsv_solve
+    st = fn(plan._h, _ptr(b), ldb, _ptr(x), lx[2], nrhs, layout, _stream_handle(stream))
+    C.check(st, "sptrsv_solve_transposed" if transposed else "sptrsv_solve")
     return x
 
 

@@ -26,7 +26,7 @@ FORMATS = ["DIAG", "CSR", "DCSR"]
 IMPLS = ["TRI_DIAG", "TRI_LEVELSET", "TRI_SYNCFREE", "TRI_CHAIN", "SQ_SCALAR", "SQ_VECTOR", "TRI_SUPERNODE", "TRI_PIPE", "SQ_ADAPT"]
 ARRAY_IN_DEGREE, ARRAY_LEVEL_PTR, ARRAY_DCSR_ROWS = 0, 1, 2
 
-EXPORTS = ["sptrsv_opts_default", "sptrsv_analyse", "sptrsv_solve", "sptrsv_free", "sptrsv_plan_info",
+EXPORTS = ["sptrsv_opts_default", "sptrsv_analyse", "sptrsv_solve", "sptrsv_solve_transposed", "sptrsv_free", "sptrsv_plan_info",
            "sptrsv_plan_segments", "sptrsv_plan_perm", "sptrsv_plan_levels", "sptrsv_plan_seg_array",
            "sptrsv_plan_matrix", "sptrsv_plan_hash", "sptrsv_set_profiling", "sptrsv_seg_times", "sptrsv_status_string",
            "sptrsv_last_error", "sptrsv_version"]
@@ -84,6 +84,8 @@ def lib() -> ctypes.CDLL:
                                  ctypes.POINTER(vp)]
     L.sptrsv_solve.restype = ctypes.c_int
     L.sptrsv_solve.argtypes = [vp, vp, i64, vp, i64, i32, ctypes.c_int, vp]
+    L.sptrsv_solve_transposed.restype = ctypes.c_int
+    L.sptrsv_solve_transposed.argtypes = [vp, vp, i64, vp, i64, i32, ctypes.c_int, vp]
     L.sptrsv_free.restype = ctypes.c_int
     L.sptrsv_free.argtypes = [vp]
     L.sptrsv_plan_info.restype = ctypes.c_int

@@ -38,6 +38,7 @@ namespace sptrsv {
 Error upload(Plan& p, void* stream);
 int count_launches_public(const Plan& p);
 void build_sq_items(Segment& S);
+SpmmCfg spmm_cfg_public();
 void build_sf_items(Segment& S, int32_t& part_base, int selector);
 void fuse_square_items(Segment& T, Segment& Q);
 bool watchdog_word_acquire(int32_t** h, int32_t** d);
@@ -1034,7 +1035,7 @@ Error analyse_device(Plan& p, int32_t n, int64_t nnz, const int32_t* d_rp, const
   p.backoff_ns = 128;
   p.wd_spins = k::kWatchdogSpins;
   if (const char* e = std::getenv("SPTRSV_WATCHDOG_SPINS")) p.wd_spins = (uint32_t)std::max(1024, std::atoi(e));
-  p.spmm = SpmmCfg{};
+  p.spmm = spmm_cfg_public();
   if (p.dtype == SPTRSV_R64F)
     return analyse_device_t<double>(p, n, nnz, d_rp, d_ci, (const double*)d_val, (cudaStream_t)stream);
   return analyse_device_t<float>(p, n, nnz, d_rp, d_ci, (const float*)d_val, (cudaStream_t)stream);

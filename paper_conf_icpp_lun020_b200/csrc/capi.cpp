@@ -229,6 +229,20 @@ SPTRSV_EXPORT sptrsv_status_t sptrsv_solve(sptrsv_plan_t plan, const void* b, in
   return SPTRSV_SUCCESS;
 }
 
+SPTRSV_EXPORT sptrsv_status_t sptrsv_solve_transposed(sptrsv_plan_t plan, const void* b, int64_t ldb, void* x,
+                                                      int64_t ldx, int32_t nrhs, sptrsv_layout_t layout,
+                                                      void* stream) {
+  if (!plan) return fail(SPTRSV_ERROR_INVALID_VALUE, "plan is NULL");
+  Plan& p = plan->p;
+  if (p.opts.host_only) return fail(SPTRSV_ERROR_NOT_SUPPORTED, "plan was analysed with host_only=1");
+  if (nrhs < 0) return fail(SPTRSV_ERROR_INVALID_VALUE, "nrhs < 0");
+  if (layout != SPTRSV_COL_MAJOR && layout != SPTRSV_ROW_MAJOR) return fail(SPTRSV_ERROR_INVALID_VALUE, "bad layout");
+  if (nrhs > 0 && p.n > 0 && (!b || !x)) return fail(SPTRSV_ERROR_INVALID_VALUE, "b or x is NULL");
+  Error e = sptrsv::solve_T(p, b, ldb, x, ldx, nrhs, layout, stream);
+  if (e.status) return fail(e);
+  return SPTRSV_SUCCESS;
+}
+
 SPTRSV_EXPORT sptrsv_status_t sptrsv_free(sptrsv_plan_t plan) {
   if (!plan) return SPTRSV_SUCCESS;
   release(plan->p);

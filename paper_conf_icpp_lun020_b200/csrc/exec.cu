@@ -889,6 +889,28 @@ Error launch_sf_wrow(Plan& p, Segment& S, int nitem, const T* val, const T* bw, 
   return {SPTRSV_SUCCESS, ""};
 }
 
+// k::tri_level_cluster: one cluster of S.cl_size CTAs (non-portable above 8)
+template <typename T>
+Error launch_cluster(Plan& p, Segment& S, const T* bw, T* xs, k::SolveState st, cudaStream_t s) {
+  auto kern = k::tri_level_cluster<T>;
+  CUDA_TRY(ensure_smem_attr((const void*)kern, 0, S.cl_size > 8));
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(S.cl_size);
+  cfg.blockDim = dim3(SPTRSV_CL_NT);
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = S.cl_size;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  const int* ip = S.d_sf_items + (size_t)S.cl_nitem * 8;
+  CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, S.info.row0, S.info.nlevels, ip, (const k::SfItem*)S.d_sf_items, S.d_rp,
+                              S.d_ci, (const T*)S.d_val, bw, xs, (T*)p.d_part, st));
+  return {SPTRSV_SUCCESS, ""};
+}
+
 template <typename T>
 Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveState st, cudaEvent_t* ev) {
   for (size_t si = 0; si < p.segs.size(); ++si) {
@@ -1082,7 +1104,10 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
             if (const char* ev2 = std::getenv("SPTRSV_SF_CTAS")) c = std::max(1, std::atoi(ev2));
             return (unsigned)std::min<int64_t>({c, (int64_t)cap, (int64_t)cdiv(rows_total, rows_per_cta)});
           };
-          if (nrhs == 1 && !S.sf_items.empty()) {
+          if (nrhs == 1 && S.cl_size > 0) {
+            Error e = launch_cluster<T>(p, S, bw, xs, st, s);
+            if (e.status) return e;
+          } else if (nrhs == 1 && !S.sf_items.empty()) {
             const int nitem = (int)(S.sf_items.size() / 8);
             int nctas = SPTRSV_SF_MINB * p.sm_count;
             if (const char* e2 = std::getenv("SPTRSV_SF_CTAS")) nctas = std::max(1, std::atoi(e2));  // tuning
@@ -1422,11 +1447,64 @@ void build_sf_wrow(Segment& S, int32_t& part_base) {
     }
   }
 }
+// Items of the cluster level-set kernel (k::tri_level_cluster): the
+// tri_sf_mixed kinds, cut at level boundaries, then ip[nlevels + 1] (first
+// item of every level) appended to the same array.
+void build_cl_items(Segment& S, int32_t& part_base, int cs) {
+  const auto& I = S.info;
+  const std::vector<int32_t>& rp = S.rp;
+  const std::vector<int32_t>& lp = S.level_ptr;
+  auto push = [&](int t0, int t1, int p0, int p1, int kind, int s0, int s1) {
+    const int32_t rec[8] = {t0, t1, p0, p1, kind, s0, s1, 0};
+    S.sf_items.insert(S.sf_items.end(), rec, rec + 8);
+  };
+  std::vector<int32_t> ip(I.nlevels + 1, 0);
+  for (int l = 0; l < I.nlevels; ++l) {
+    ip[l] = (int32_t)(S.sf_items.size() / 8);
+    int t = lp[l];
+    const int tend = lp[l + 1];
+    while (t < tend) {
+      const int len = rp[t + 1] - rp[t];
+      if (len > k::kSfLong) {
+        if (len <= k::kSfNB) {
+          push(t, t + 1, rp[t], rp[t + 1], 3, 0, 0);
+        } else {
+          const int np = (len + k::kSfNB - 1) / k::kSfNB;
+          const int first = part_base;
+          for (int q = 0; q < np; ++q) {
+            const int a = rp[t] + q * k::kSfNB, b = std::min(a + k::kSfNB, rp[t + 1]);
+            if (q < np - 1)
+              push(t, t + 1, a, b, 1, part_base++, 0);
+            else
+              push(t, t + 1, a, b, 2, first, part_base);
+          }
+        }
+        ++t;
+        continue;
+      }
+      const int start = t;
+      while (t < tend && t - start < 32 && rp[t + 1] - rp[t] <= k::kSfLong) ++t;
+      push(start, t, rp[start], rp[t], 0, 0, 0);
+    }
+  }
+  ip[I.nlevels] = (int32_t)(S.sf_items.size() / 8);
+  S.cl_nitem = ip[I.nlevels];
+  S.sf_items.insert(S.sf_items.end(), ip.begin(), ip.end());
+  S.cl_size = cs;
+}
+
 void build_sf_items(Segment& S, int32_t& part_base, int selector) {
   S.sf_items.clear();
   S.sf_mixed = S.sf_wrow = false;
+  S.cl_size = 0;
+  S.cl_nitem = 0;
   const auto& I = S.info;
   if (I.kind != 0 || I.impl != SPTRSV_IMPL_TRI_SYNCFREE || selector != SPTRSV_SELECT_B200) return;
+  if (const char* e = std::getenv("SPTRSV_SF_CLUSTER")) {  // experiment: level-set on one cluster
+    const int cs = std::atoi(e);
+    if (cs >= 1 && cs <= 16 && (int)S.level_ptr.size() == I.nlevels + 1 && I.nlevels > 1)
+      return build_cl_items(S, part_base, cs);
+  }
   // default (B200): the mixed-granularity kernel; SPTRSV_SF_V1 = the round-1
   // thread / warp-per-row kernels (kept for comparison)
   S.sf_mixed = std::getenv("SPTRSV_SF_V1") == nullptr && std::getenv("SPTRSV_SF_WROW") == nullptr &&
@@ -2082,6 +2160,106 @@ Error solve(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t n
   return {SPTRSV_SUCCESS, ""};
 }
 
+// ------------------------------------------- A^T x = b from the same plan
+// (reading R32; kernels: k::perm_in_T / tri_push_T /
+// sq_push_T / perm_out_T).  First call: the in-degree counters of L1^T
+// (column counts of every triangle's CSR) and, for wave triangles whose
+// device row order is not the level order, the reverse-level claim order.
+Error prepare_T(Plan& p, cudaStream_t s) {
+  if (p.d_tcnt0) return {SPTRSV_SUCCESS, ""};
+  const int n = p.n;
+  const size_t ns = p.segs.size();
+  p.d_tcnt0 = (int32_t*)dalloc(p, (size_t)std::max(1, n) * 4, s);
+  p.d_tcnt = (int32_t*)dalloc(p, (size_t)std::max(1, n) * 4, s);
+  p.d_tticket = (uint32_t*)dalloc(p, std::max<size_t>(1, ns) * 4, s);
+  if (!p.d_tcnt0 || !p.d_tcnt || !p.d_tticket) return {SPTRSV_ERROR_ALLOC, "transposed-solve workspace"};
+  CUDA_TRY(cudaMemsetAsync(p.d_tcnt0, 0, (size_t)std::max(1, n) * 4, s));
+  p.d_torder.assign(ns, nullptr);
+  for (size_t i = 0; i < ns; ++i) {
+    Segment& S = p.segs[i];
+    if (S.info.kind != 0) continue;
+    const int m = S.info.row1 - S.info.row0;
+    const int64_t ne = S.rp.empty() ? (int64_t)S.info.nnz - m : (int64_t)S.rp.back();
+    if (ne > 0)
+      k::count_cols<<<(unsigned)std::min<int64_t>(cdiv(ne, 256), (int64_t)p.sm_count * 16), 256, 0, s>>>(
+          ne, S.d_ci, p.d_tcnt0);
+    if (S.wave_K > 0 && (int)S.wave_tau.size() == m) {  // device position q of plan row t: tau^-1
+      std::vector<int32_t> inv(m), ord(m);
+      for (int q = 0; q < m; ++q) inv[S.wave_tau[q]] = q;
+      for (int i2 = 0; i2 < m; ++i2) ord[i2] = inv[m - 1 - i2];
+      p.d_torder[i] = (int32_t*)dalloc(p, (size_t)m * 4, s);
+      if (!p.d_torder[i]) return {SPTRSV_ERROR_ALLOC, "transposed-solve claim order"};
+      CUDA_TRY(cudaMemcpyAsync(p.d_torder[i], ord.data(), (size_t)m * 4, cudaMemcpyHostToDevice, s));
+      CUDA_TRY(cudaStreamSynchronize(s));  // ord is a host temporary
+    }
+  }
+  CUDA_TRY(cudaGetLastError());
+  return {SPTRSV_SUCCESS, ""};
+}
+
+template <typename T>
+Error solve_T_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, sptrsv_layout_t layout, cudaStream_t s) {
+  const int n = p.n;
+  T* bw = (T*)p.ws.bw;
+  T* xs = (T*)p.ws.xs;
+  k::SolveState st{p.d_tickets, p.nticket, p.d_error, nullptr, p.d_epoch, 0u, 0u, p.backoff_ns, p.d_derr, p.wd_spins,
+                   nullptr};
+  const int64_t sb = layout == SPTRSV_ROW_MAJOR ? ldb : 1, sx = layout == SPTRSV_ROW_MAJOR ? ldx : 1;
+  const int nseg = (int)p.segs.size();
+  k::perm_in_T<T><<<std::max(1u, cdiv(n, 256)), 256, 0, s>>>(n, p.d_perm, b, sb, bw, p.d_tcnt0, p.d_tcnt,
+                                                             p.d_tticket, nseg);
+  CUDA_TRY(cudaGetLastError());
+  for (int si = nseg - 1; si >= 0; --si) {  // segments in reverse order
+    Segment& S = p.segs[si];
+    const auto& I = S.info;
+    const T* val = (const T*)S.d_val;
+    if (I.kind == 1) {
+      if (S.dev_nzr > 0 && I.nnz > 0) {
+        const unsigned g = cdiv(S.dev_nzr, 128);
+        if (S.dev_dcsr)
+          k::sq_push_T<T, true><<<g, 128, 0, s>>>(S.dev_nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
+        else
+          k::sq_push_T<T, false><<<g, 128, 0, s>>>(S.dev_nzr, I.row0, S.d_rows, S.d_rp, S.d_ci, val, xs, bw);
+      }
+    } else {
+      const int m = I.row1 - I.row0;
+      if (m > 0) {
+        const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>(cdiv(m, 256), (int64_t)p.sm_count * 2));
+        k::tri_push_T<T><<<g, 256, 0, s>>>(I.row0, m, p.d_torder.empty() ? nullptr : p.d_torder[si], S.d_rp, S.d_ci,
+                                           val, bw, xs, p.d_tcnt, p.d_tticket + si, st);
+      }
+    }
+    CUDA_TRY(cudaGetLastError());
+  }
+  k::perm_out_T<T><<<std::max(1u, cdiv(n, 256)), 256, 0, s>>>(n, p.d_perm, (const T*)p.d_rdiag, xs, x, sx);
+  CUDA_TRY(cudaGetLastError());
+  return {SPTRSV_SUCCESS, ""};
+}
+
+Error solve_T(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t nrhs, sptrsv_layout_t layout,
+              void* stream_v) {
+  cudaStream_t s = (cudaStream_t)stream_v;
+  int cur = -1;
+  if (cudaGetDevice(&cur) != cudaSuccess || cur != p.device) CUDA_TRY(cudaSetDevice(p.device));
+  if (take_deadlock(p, s))
+    return {SPTRSV_ERROR_DEADLOCK, "a spin-wait watchdog tripped during an earlier solve on this plan"};
+  if (nrhs == 0 || p.n == 0) return {SPTRSV_SUCCESS, ""};
+  if (nrhs != 1) return {SPTRSV_ERROR_NOT_SUPPORTED, "the transposed solve from the same plan takes one RHS"};
+  int bdev = -1, xdev = -1;
+  const int bd = ptr_kind(b, &bdev), xd = ptr_kind(x, &xdev);
+  if (!bd || !xd) return {SPTRSV_ERROR_NOT_SUPPORTED, "the transposed solve takes device pointers"};
+  if (bdev != p.device || xdev != p.device)
+    return {SPTRSV_ERROR_INVALID_VALUE, "b / x live on another device than the plan"};
+  Error e = prepare_solve(p, 1, s);
+  if (e.status) return e;
+  e = prepare_T(p, s);
+  if (e.status) return e;
+  e = p.dtype == SPTRSV_R64F ? solve_T_device<double>(p, (const double*)b, ldb, (double*)x, ldx, layout, s)
+                             : solve_T_device<float>(p, (const float*)b, ldb, (float*)x, ldx, layout, s);
+  if (e.status) return e;
+  return record_done(p, s);
+}
+
 void release(Plan& p) {
   if (p.device >= 0) {
     cudaSetDevice(p.device);
@@ -2097,6 +2275,13 @@ void release(Plan& p) {
   dfree(p, p.ws.stage_b, nullptr);
   dfree(p, p.ws.stage_x, nullptr);
   dfree(p, p.ws.flags, nullptr);
+  dfree(p, p.d_tcnt0, nullptr);
+  dfree(p, p.d_tcnt, nullptr);
+  dfree(p, p.d_tticket, nullptr);
+  for (auto* q : p.d_torder) dfree(p, q, nullptr);
+  p.d_tcnt0 = p.d_tcnt = nullptr;
+  p.d_tticket = nullptr;
+  p.d_torder.clear();
   if (p.ws.h2d) cudaStreamDestroy((cudaStream_t)p.ws.h2d);
   if (p.ws.d2h) cudaStreamDestroy((cudaStream_t)p.ws.d2h);
   for (void* e : p.ws.ev)
@@ -2142,6 +2327,7 @@ Error device_info(int* sm_count, int* major, int* minor) {
 }
 
 int count_launches_public(const Plan& p) { return count_launches(p); }
+SpmmCfg spmm_cfg_public() { return spmm_cfg(); }
 Error prepare_solve_public(Plan& p, int nrhs, cudaStream_t s) { return prepare_solve(p, nrhs, s); }
 
 }  // namespace sptrsv

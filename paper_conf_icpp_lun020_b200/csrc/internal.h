@@ -139,6 +139,9 @@ struct Segment {
   int32_t fused_sq = -1;  // TRI (mixed sync-free): index of the square fused as trailing items
   bool fused = false;     // SQ: computed inside the preceding triangle's kernel at nrhs == 1
   bool sf_wrow = false;
+  int32_t cl_size = 0;    // TRI: > 0 = level-set on one cluster of cl_size CTAs (k::tri_level_cluster);
+                          // sf_items then holds the level-cut items followed by ip[nlevels + 1]
+  int32_t cl_nitem = 0;
   const int32_t* d_sf_items = nullptr;
   // row-block square kernel (k::sq_adapt_1, nrhs == 1): k::SqItem[] as 4 ints
   std::vector<int32_t> sq_items;
@@ -186,7 +189,8 @@ struct GraphEntry {
 // SpMM lane geometry for nrhs > 1 (exec.cu: dispatch_multi_un)
 struct SpmmCfg {
   int rpt_max = 8, un = 2;  // measured best on C5 (round 1 sweep, profiles/r01_sweeps.md)
-  int tile = 16;            // RHS tile width of the tiled SpMM (0 = untiled; SPTRSV_SPMM_TILE)
+  int tile = 0;             // RHS tile width of the tiled SpMM (0 = untiled, the default: re-streaming
+                            // the matrix per tile measured 1.6-1.75x slower on C5; SPTRSV_SPMM_TILE)
 };
 
 struct Plan {
@@ -251,6 +255,13 @@ struct Plan {
   bool done_ev_recorded = false;
   int launches_per_solve = 0;
 
+  // transposed solve from the same plan (f-4, reading R32; exec.cu solve_T):
+  // built at the first A^T solve
+  int32_t* d_tcnt0 = nullptr;        // in-degree of L1^T per row: column counts inside its triangle
+  int32_t* d_tcnt = nullptr;         // working counters, reset from d_tcnt0 by permute-in
+  uint32_t* d_tticket = nullptr;     // per-segment claim tickets
+  std::vector<int32_t*> d_torder;    // per segment: claim order (wave triangles), else nullptr
+
   // profiling
   bool profiling = false;
   std::vector<void*> events;  // cudaEvent_t
@@ -288,6 +299,9 @@ void dfree(Plan& p, void* q, cudaStream_t s);
 Error upload(Plan& p, void* stream);
 Error solve(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t nrhs,
             sptrsv_layout_t layout, void* stream);
+// A^T x = b with the plan of A (nrhs == 1, device pointers)
+Error solve_T(Plan& p, const void* b, int64_t ldb, void* x, int64_t ldx, int32_t nrhs,
+              sptrsv_layout_t layout, void* stream);
 void release(Plan& p);
 
 }  // namespace sptrsv

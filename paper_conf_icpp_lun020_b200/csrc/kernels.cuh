@@ -357,6 +357,10 @@ __global__ void __launch_bounds__(256) sq_adapt_1(int nitem, int r0, const SqIte
                                                   const int* __restrict__ rows, const int* __restrict__ rp,
                                                   const int* __restrict__ ci, const T* __restrict__ val,
                                                   const T* __restrict__ xs, T* __restrict__ bw) {
+  // One item per warp.  Every load that does not depend on x (entries, row
+  // bounds, DCSR row ids, the b' values) is issued together with the entry
+  // loads, so the item's dependent chain is header -> entries -> x gathers.
+  // (A persistent grid with next-item prefetch measured slower on C3.)
   __shared__ T prod[8][kSqNB];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int w = blockIdx.x * 8 + warp;
@@ -402,6 +406,15 @@ __global__ void __launch_bounds__(256) sq_adapt_1(int nitem, int r0, const SqIte
       v[u] = ldg_nc(val + p);
     }
   }
+  const int t = t0 + lane;
+  int q0 = 0, q1 = 0, r = 0;
+  T br = T(0);
+  if (t < t1) {
+    q0 = __ldg(rp + t) - a;
+    q1 = __ldg(rp + t + 1) - a;
+    r = DCSR ? __ldg(rows + t) : r0 + t;
+    if (q1 > q0) br = bw[r];  // this item is the only writer of row r
+  }
 #pragma unroll
   for (int u = 0; u < kSqNB / 32; ++u)
     if (a + 32 * u + lane < e) x[u] = ldg_nc(xs + j[u]);
@@ -409,15 +422,10 @@ __global__ void __launch_bounds__(256) sq_adapt_1(int nitem, int r0, const SqIte
   for (int u = 0; u < kSqNB / 32; ++u)
     if (a + 32 * u + lane < e) pr[32 * u + lane] = v[u] * x[u];
   __syncwarp();
-  const int t = t0 + lane;
-  if (t < t1) {
-    const int q0 = rp[t] - a, q1 = rp[t + 1] - a;
-    if (q1 > q0) {
-      T sum = 0;
-      for (int q = q0; q < q1; ++q) sum += pr[q];
-      const int r = DCSR ? rows[t] : r0 + t;
-      bw[r] -= sum;
-    }
+  if (q1 > q0) {
+    T sum = 0;
+    for (int q = q0; q < q1; ++q) sum += pr[q];
+    bw[r] = br - sum;
   }
 }
 
@@ -1667,6 +1675,10 @@ __global__ void __launch_bounds__(256) tri_syncfree_multi(int r0, int m, const i
     const int r = r0 + k;
     const int a = rp[k], e = rp[k + 1];
     for (int c0 = 0; c0 < nrhs; c0 += G * RPT) {
+      // a whole pass of columns in range: with one predicate per column the
+      // 7 predicate registers run out and ptxas interleaves FMAs with the
+      // gathers (9 of 16 in flight; C5 seg0 3.5 -> 8.3 ms in round 2)
+      const bool full = c0 + G * RPT <= nrhs;
       T acc[RPT];
 #pragma unroll
       for (int t = 0; t < RPT; ++t)
@@ -1684,12 +1696,19 @@ __global__ void __launch_bounds__(256) tri_syncfree_multi(int r0, int m, const i
         }
         const T* xr = xs + (int64_t)j * nrhs + c0 + lane;
         T x[RPT];
+        if (full) {  // no per-column predicates: all RPT gathers issue before the first FMA
 #pragma unroll
-        for (int t = 0; t < RPT; ++t)
-          if (c0 + lane + G * t < nrhs) x[t] = ld_strong(xr + G * t);
+          for (int t = 0; t < RPT; ++t) x[t] = ld_strong(xr + G * t);
 #pragma unroll
-        for (int t = 0; t < RPT; ++t)
-          if (c0 + lane + G * t < nrhs) acc[t] -= v * x[t];
+          for (int t = 0; t < RPT; ++t) acc[t] -= v * x[t];
+        } else {
+#pragma unroll
+          for (int t = 0; t < RPT; ++t)
+            if (c0 + lane + G * t < nrhs) x[t] = ld_strong(xr + G * t);
+#pragma unroll
+          for (int t = 0; t < RPT; ++t)
+            if (c0 + lane + G * t < nrhs) acc[t] -= v * x[t];
+        }
       }
       T* xo = xs + (int64_t)r * nrhs + c0 + lane;
 #pragma unroll
@@ -2597,6 +2616,283 @@ __global__ void __launch_bounds__(288, 1)
   }
   __syncthreads();
   cluster_sync_all();  // no CTA leaves while a peer may still push into it
+}
+
+
+// ----------------------------------- K2 on one cluster: level-set, no launches
+// Level-set (Alg 2 L88-L98) for a triangle whose levels are narrow but many
+// (B200 selector, nrhs == 1): the whole triangle runs in ONE thread-block
+// cluster (CS CTAs, one per SM), and Alg 2's barrier between levels (L96) is
+// the cluster barrier (barrier.cluster.arrive.release / wait.acquire, ~400
+// cycles on-chip) instead of a kernel boundary (~2-3 us) or the sync-free
+// kernel's per-dependency polls through L2 (Alg 3; on B200 a level of
+// ~10^3 rows ends with the slowest of its detections, ~1 us).  No flags, no
+// sentinels, no tickets: after the barrier every x of earlier levels is
+// visible, so a row's dependencies are plain loads.
+//
+// Work of level l = the items [ip[l], ip[l+1]) (exec.cu build_cl_items; the
+// tri_sf_mixed item kinds, cut at level boundaries): kind 0 = <= 32
+// consecutive rows with <= kSfLong entries, lane per row; kind 3 = one row
+// of <= kSfNB entries, warp; kind 1/2 = kSfNB-entry pieces of a longer row
+// (partial sums to `part` slots, the last piece adds them in piece order).
+// Warp gw of the cluster takes items ip[l] + gw, + NW, ...  Between
+// barrier.cluster.arrive and .wait each warp already loads the header,
+// indices, values and b' of its first item of the next level (they do not
+// depend on x), so after the wait only the x gathers remain on the chain.
+template <typename T>
+struct ClPre {
+  int4 h0, h1;
+  int p, e, cnt;
+  T s;
+  int j[kSfNB / 32];
+  T v[kSfNB / 32];
+};
+
+template <typename T>
+__device__ __forceinline__ void cl_load(ClPre<T>& q, const SfItem* __restrict__ items, int w, int r0,
+                                        const int* __restrict__ rp, const int* __restrict__ ci,
+                                        const T* __restrict__ val, const T* __restrict__ bw, int lane) {
+  constexpr int UW = kSfNB / 32;
+  q.h0 = __ldg((const int4*)(items + w));
+  q.h1 = __ldg((const int4*)(items + w) + 1);
+  if (q.h1.x == 0) {
+    const int k = q.h0.x + lane;
+    q.p = q.e = 0;
+    q.s = T(0);
+    if (k < q.h0.y) {
+      q.p = __ldg(rp + k);
+      q.e = __ldg(rp + k + 1);
+      q.s = ldg_nc(bw + r0 + k);
+    }
+    q.cnt = min(UW, q.e - q.p);
+#pragma unroll
+    for (int u = 0; u < UW; ++u)
+      if (u < q.cnt) {
+        q.j[u] = __ldg(ci + q.p + u);
+        q.v[u] = ldg_nc(val + q.p + u);
+      }
+  } else {
+    const int ne = q.h0.w - q.h0.z;
+    q.s = (q.h1.x != 1 && lane == 0) ? ldg_nc(bw + r0 + q.h0.x) : T(0);
+#pragma unroll
+    for (int u = 0; u < UW; ++u)
+      if (lane + 32 * u < ne) {
+        q.j[u] = __ldg(ci + q.h0.z + lane + 32 * u);
+        q.v[u] = ldg_nc(val + q.h0.z + lane + 32 * u);
+      }
+  }
+}
+
+template <typename T>
+__device__ __forceinline__ bool cl_compute(ClPre<T>& q, int r0, const int* __restrict__ ci,
+                                           const T* __restrict__ val, T* __restrict__ xs, T* __restrict__ part,
+                                           const SolveState& st, uint32_t& spins, int lane) {
+  constexpr int UW = kSfNB / 32;
+  if (q.h1.x == 0) {
+    if (q.h0.x + lane < q.h0.y) {
+      T x[UW];
+#pragma unroll
+      for (int u = 0; u < UW; ++u)
+        if (u < q.cnt) x[u] = xs[q.j[u]];
+      T s = q.s;
+#pragma unroll
+      for (int u = 0; u < UW; ++u)
+        if (u < q.cnt) s -= q.v[u] * x[u];
+      for (int p = q.p + q.cnt; p < q.e; p += UW) {  // rows longer than UW (<= kSfLong)
+        const int cnt = min(UW, q.e - p);
+#pragma unroll
+        for (int u = 0; u < UW; ++u)
+          if (u < cnt) {
+            q.j[u] = __ldg(ci + p + u);
+            q.v[u] = ldg_nc(val + p + u);
+          }
+#pragma unroll
+        for (int u = 0; u < UW; ++u)
+          if (u < cnt) x[u] = xs[q.j[u]];
+#pragma unroll
+        for (int u = 0; u < UW; ++u)
+          if (u < cnt) s -= q.v[u] * x[u];
+      }
+      xs[r0 + q.h0.x + lane] = s;
+    }
+    return true;
+  }
+  const int kind = q.h1.x, ne = q.h0.w - q.h0.z;
+  T acc = 0;
+  {
+    T x[UW];
+#pragma unroll
+    for (int u = 0; u < UW; ++u)
+      if (lane + 32 * u < ne) x[u] = xs[q.j[u]];
+#pragma unroll
+    for (int u = 0; u < UW; ++u)
+      if (lane + 32 * u < ne) acc += q.v[u] * x[u];
+  }
+  acc = warp_sum(acc);
+  bool ok = true;
+  if (kind == 2) {  // the earlier pieces' partial sums (same level), in piece order
+    const int np = q.h1.z - q.h1.y;
+    T pv = T(0);
+    if (lane < np) {
+      pv = ld_strong(part + q.h1.y + lane);
+      while (is_sent(pv)) {
+        if (wd_giveup(spins, st)) {
+          ok = false;
+          break;
+        }
+        pv = ld_strong(part + q.h1.y + lane);
+      }
+    }
+    acc += warp_sum(pv);
+  }
+  if (lane == 0) {
+    if (kind == 1)
+      st_strong(part + q.h1.y, acc);
+    else
+      xs[r0 + q.h0.x] = q.s - acc;
+  }
+  return __all_sync(0xffffffffu, ok);
+}
+
+#ifndef SPTRSV_CL_NT
+#define SPTRSV_CL_NT 512
+#endif
+template <typename T>
+__global__ void __launch_bounds__(SPTRSV_CL_NT, 1)
+    tri_level_cluster(int r0, int nlev, const int* __restrict__ ip, const SfItem* __restrict__ items,
+                      const int* __restrict__ rp, const int* __restrict__ ci, const T* __restrict__ val,
+                      const T* __restrict__ bw, T* __restrict__ xs, T* __restrict__ part, SolveState st) {
+  const int lane = threadIdx.x & 31;
+  const int nw = gridDim.x * (blockDim.x >> 5);
+  const int gw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  uint32_t spins = 0;
+  bool alive = true;
+  ClPre<T> q;
+  int i0 = __ldg(ip), i1 = __ldg(ip + 1);
+  bool have = gw < i1 - i0;
+  if (have) cl_load(q, items, i0 + gw, r0, rp, ci, val, bw, lane);
+  for (int l = 0; l < nlev; ++l) {
+    const int i2 = l + 2 <= nlev ? __ldg(ip + l + 2) : i1;
+    if (have && alive) alive = cl_compute(q, r0, ci, val, xs, part, st, spins, lane);
+    for (int w = i0 + gw + nw; w < i1 && alive; w += nw) {
+      cl_load(q, items, w, r0, rp, ci, val, bw, lane);
+      alive = cl_compute(q, r0, ci, val, xs, part, st, spins, lane);
+    }
+    __syncwarp();
+    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+    have = i1 + gw < i2;
+    if (have) cl_load(q, items, i1 + gw, r0, rp, ci, val, bw, lane);
+    __syncwarp();
+    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+    i0 = i1;
+    i1 = i2;
+  }
+}
+
+
+// ------------------------------ transposed solve from the same plan (f-4, R32)
+// A^T x = b with the plan of A.  The plan stores L1 = D^-1 P A P^T (unit
+// lower, values scaled by 1/d, R27), so A = P^T D L1 P and
+//     A^T x = b  <=>  L1^T z = P b,   x = P^T D^-1 z.
+// L1^T is unit UPPER: it is solved over the plan's segments in REVERSE order
+// with the PUSH form of the sync-free solve, Alg 3 (L105-L125) as the paper
+// states it: a component waits until its in-degree counter (here the number
+// of not-yet-solved rows whose L1 row references it, i.e. its column count
+// inside the triangle) reaches zero, takes z_i = b'_i, then for every entry
+// (i, j) of its L1 row adds -l'_ij z_i into b'_j with atomicAdd and
+// decrements in_degree[j] (release after a fence).  A square (rows R, cols C)
+// of L1 becomes b'_C -= S^T z_R: every stored row pushes its entries with
+// atomics.  The same CSR arrays serve both directions: no second plan, no
+// transpose of the matrix.
+
+// b'[k] = b[perm[k]] (no 1/d: it moves to permute-out); counters from cnt0;
+// block 0 zeroes the per-segment claim tickets
+template <typename T>
+__global__ void perm_in_T(int n, const int* __restrict__ perm, const T* __restrict__ b, int64_t stride,
+                          T* __restrict__ bw, const int* __restrict__ cnt0, int* __restrict__ cnt,
+                          uint32_t* __restrict__ tickets, int nticket) {
+  if (blockIdx.x == 0)
+    for (int t = threadIdx.x; t < nticket; t += blockDim.x) tickets[t] = 0;
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k < n) {
+    bw[k] = b[(int64_t)perm[k] * stride];
+    cnt[k] = cnt0[k];
+  }
+}
+
+// x[perm[k]] = z_k / d_k
+template <typename T>
+__global__ void perm_out_T(int n, const int* __restrict__ perm, const T* __restrict__ rd, const T* __restrict__ xs,
+                           T* __restrict__ x, int64_t stride) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k < n) x[(int64_t)perm[k] * stride] = xs[k] * rd[k];
+}
+
+// in-degree of the transposed triangle: column counts of its CSR entries
+static __global__ void count_cols(int64_t nnz, const int* __restrict__ ci, int* __restrict__ cnt0) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < nnz; p += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(cnt0 + ci[p], 1);
+}
+
+__device__ __forceinline__ int ld_acquire(const int* p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// Transposed triangle (unit upper L1^T), push form.  Warps claim groups of
+// 32 components through a ticket in REVERSE topological order (order[i], or
+// local row m-1-i when the device row order is the level order), so every
+// component a claimed one waits for was claimed earlier and is running: no
+// deadlock under any CTA schedule (the argument of the forward kernel).
+template <typename T>
+__global__ void __launch_bounds__(256) tri_push_T(int r0, int m, const int* __restrict__ order,
+                                                  const int* __restrict__ rp, const int* __restrict__ ci,
+                                                  const T* __restrict__ val, T* __restrict__ bw, T* __restrict__ xs,
+                                                  int* __restrict__ cnt, uint32_t* __restrict__ ticket,
+                                                  SolveState st) {
+  const int lane = threadIdx.x & 31;
+  uint32_t spins = 0;
+  for (;;) {
+    int base = 0;
+    if (lane == 0) base = (int)atomicAdd(ticket, 32u);
+    base = __shfl_sync(0xffffffffu, base, 0);
+    if (base >= m) break;
+    const int i = base + lane;
+    bool done = i >= m;
+    int q = 0;
+    if (!done) q = order ? __ldg(order + i) : m - 1 - i;
+    const int r = r0 + q;
+    int a = 0, e = 0;
+    if (!done) {
+      a = __ldg(rp + q);
+      e = __ldg(rp + q + 1);
+    }
+    while (!__all_sync(0xffffffffu, done)) {
+      if (!done && ld_acquire(cnt + r) == 0) {
+        const T z = ld_strong(bw + r);  // every push into b'_r happened before its counter release
+        xs[r] = z;
+        for (int p = a; p < e; ++p) atomicAdd(bw + __ldg(ci + p), -ldg_nc(val + p) * z);
+        __threadfence();
+        for (int p = a; p < e; ++p) atomicSub(cnt + __ldg(ci + p), 1);
+        done = true;
+      }
+      if (!done && wd_giveup(spins, st)) done = true;  // garbage result, DEADLOCK reported
+    }
+  }
+}
+
+// Transposed square: b'_c -= sum_r s'_rc z_r, one lane per stored row
+template <typename T, bool DCSR>
+__global__ void sq_push_T(int nzr, int r0, const int* __restrict__ rows, const int* __restrict__ rp,
+                          const int* __restrict__ ci, const T* __restrict__ val, const T* __restrict__ xs,
+                          T* __restrict__ bw) {
+  const int t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= nzr) return;
+  const int r = DCSR ? __ldg(rows + t) : r0 + t;
+  const T z = xs[r];
+  const int a = __ldg(rp + t), e = __ldg(rp + t + 1);
+  for (int p = a; p < e; ++p) atomicAdd(bw + __ldg(ci + p), -ldg_nc(val + p) * z);
 }
 
 }  // namespace k
