@@ -421,8 +421,15 @@ def main():
             dep = {"nlevels": dseg["nlevels"], "ns_per_level": ns_lvl}
             tl = load_tlvl()
             if tl:
-                dep["t_lvl_floor_ns"] = tl.get("smem_chain_bar_ns")
-                dep["t_lvl_source"] = "profiles/t_lvl.json (bar.sync + ld.shared/DFMA/st.shared chain, 1 SM)"
+                # the floor of ONE dependent level for the kernel family: an
+                # on-SM barrier chain for the single-SM / one-cluster kernels,
+                # a cross-SM store -> poll hop through L2 for the multi-SM ones
+                on_sm = dimpl in ("TRI_CHAIN", "TRI_PIPE")
+                fl = tl.get("smem_chain_bar_ns") if on_sm else tl.get("cross_sm_hop_ns")
+                dep["t_lvl_floor_ns"] = fl
+                dep["floor_frac"] = fl / ns_lvl if fl else None
+                dep["t_lvl_source"] = ("profiles/t_lvl.json: " + ("bar.sync + ld.shared/DFMA/st.shared chain, 1 SM"
+                                       if on_sm else "cross-SM flag ping-pong through L2 (st/ld.relaxed.gpu)"))
     else:
         dbytes = M.n * 4 + 2 * M.n * nrhs * vb
         dimpl = "PERMUTE"

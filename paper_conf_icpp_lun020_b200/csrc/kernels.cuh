@@ -1269,17 +1269,20 @@ __global__ void __launch_bounds__(256, SPTRSV_SFM_MINB) tri_sf_mixed(int r0, int
 #pragma unroll
     for (int u = 0; u < UW; ++u) acc += v[u] * x[u];
     acc = warp_sum(acc);
-    if (kind == 2) {  // add the earlier pieces' partial sums, in piece order
-      const int np = h1.z - h1.y;
-      T pv = T(0);
-      if (lane < np) {
-        pv = ld_strong(part + h1.y + lane);
-        while (is_sent(pv)) {
-          if (wd_giveup(spins, st)) break;
-          pv = ld_strong(part + h1.y + lane);
+    if (kind == 2) {  // add the earlier pieces' partial sums, 32 at a time, in piece order
+      T ps = T(0);   // (a row of > 32 * kSfNB entries has > 32 pieces: the hub columns of
+      for (int q0 = h1.y; q0 < h1.z; q0 += 32) {  // C3 become rows of 258K entries in C3^T)
+        T pv = T(0);
+        if (q0 + lane < h1.z) {
+          pv = ld_strong(part + q0 + lane);
+          while (is_sent(pv)) {
+            if (wd_giveup(spins, st)) break;
+            pv = ld_strong(part + q0 + lane);
+          }
         }
+        ps += warp_sum(pv);
       }
-      acc += warp_sum(pv);
+      acc += ps;
     }
     if (lane == 0) {
       if (kind == 1) {
@@ -2730,20 +2733,23 @@ __device__ __forceinline__ bool cl_compute(ClPre<T>& q, int r0, const int* __res
   }
   acc = warp_sum(acc);
   bool ok = true;
-  if (kind == 2) {  // the earlier pieces' partial sums (same level), in piece order
-    const int np = q.h1.z - q.h1.y;
-    T pv = T(0);
-    if (lane < np) {
-      pv = ld_strong(part + q.h1.y + lane);
-      while (is_sent(pv)) {
-        if (wd_giveup(spins, st)) {
-          ok = false;
-          break;
+  if (kind == 2) {  // the earlier pieces' partial sums (same level), 32 at a time, in piece order
+    T ps = T(0);
+    for (int q0 = q.h1.y; q0 < q.h1.z; q0 += 32) {
+      T pv = T(0);
+      if (q0 + lane < q.h1.z) {
+        pv = ld_strong(part + q0 + lane);
+        while (is_sent(pv)) {
+          if (wd_giveup(spins, st)) {
+            ok = false;
+            break;
+          }
+          pv = ld_strong(part + q0 + lane);
         }
-        pv = ld_strong(part + q.h1.y + lane);
       }
+      ps += warp_sum(pv);
     }
-    acc += warp_sum(pv);
+    acc += ps;
   }
   if (lane == 0) {
     if (kind == 1)
@@ -2845,6 +2851,48 @@ __device__ __forceinline__ int ld_acquire(const int* p) {
 // local row m-1-i when the device row order is the level order), so every
 // component a claimed one waits for was claimed earlier and is running: no
 // deadlock under any CTA schedule (the argument of the forward kernel).
+// Pushes of one row (entries [a, e), value z): a row of <= kPushShort
+// entries is pushed by its own lane; longer rows (supernodal panels, hubs)
+// by the whole warp, lanes over the entries, one ready row after another.
+// Every lane fences (acq_rel) between its own adds and its own decrements:
+// the release pattern of Alg 3's "atomicAdd(left_sum) then atomicSub
+// (in_degree)" (L118-L123), without a sequentially consistent fence.
+constexpr int kPushShort = 8;
+__device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+
+template <typename T, bool CNT>
+__device__ __forceinline__ void push_rows(bool ready, int a, int e, T z, const int* __restrict__ ci,
+                                          const T* __restrict__ val, T* __restrict__ bw, int* __restrict__ cnt,
+                                          int lane) {
+  const bool shortr = ready && e - a <= kPushShort;
+  if (shortr)
+    for (int p = a; p < e; ++p) atomicAdd(bw + __ldg(ci + p), -ldg_nc(val + p) * z);
+  unsigned lm = __ballot_sync(0xffffffffu, ready && !shortr);
+  unsigned lm2 = lm;
+  while (lm) {
+    const int src = __ffs(lm) - 1;
+    lm &= lm - 1;
+    const int pa = __shfl_sync(0xffffffffu, a, src), pe = __shfl_sync(0xffffffffu, e, src);
+    const T pz = __shfl_sync(0xffffffffu, z, src);
+    for (int p = pa + lane; p < pe; p += 32) atomicAdd(bw + __ldg(ci + p), -ldg_nc(val + p) * pz);
+  }
+  if (!CNT) return;
+  if (__any_sync(0xffffffffu, ready)) fence_acq_rel_gpu();
+  if (shortr)
+    for (int p = a; p < e; ++p) atomicSub(cnt + __ldg(ci + p), 1);
+  while (lm2) {
+    const int src = __ffs(lm2) - 1;
+    lm2 &= lm2 - 1;
+    const int pa = __shfl_sync(0xffffffffu, a, src), pe = __shfl_sync(0xffffffffu, e, src);
+    for (int p = pa + lane; p < pe; p += 32) atomicSub(cnt + __ldg(ci + p), 1);
+  }
+}
+
+// Transposed triangle (unit upper L1^T), push form.  Warps claim groups of
+// 32 components through a ticket in REVERSE topological order (order[i], or
+// local row m-1-i when the device row order is the level order), so every
+// component a claimed one waits for was claimed earlier and is running: no
+// deadlock under any CTA schedule (the argument of the forward kernel).
 template <typename T>
 __global__ void __launch_bounds__(256) tri_push_T(int r0, int m, const int* __restrict__ order,
                                                   const int* __restrict__ rp, const int* __restrict__ ci,
@@ -2868,31 +2916,42 @@ __global__ void __launch_bounds__(256) tri_push_T(int r0, int m, const int* __re
       a = __ldg(rp + q);
       e = __ldg(rp + q + 1);
     }
+    bool give = false;
     while (!__all_sync(0xffffffffu, done)) {
-      if (!done && ld_acquire(cnt + r) == 0) {
-        const T z = ld_strong(bw + r);  // every push into b'_r happened before its counter release
+      const bool ready = !done && ld_acquire(cnt + r) == 0;
+      T z = T(0);
+      if (ready) {
+        z = ld_strong(bw + r);  // every push into b'_r happened before its counter release
         xs[r] = z;
-        for (int p = a; p < e; ++p) atomicAdd(bw + __ldg(ci + p), -ldg_nc(val + p) * z);
-        __threadfence();
-        for (int p = a; p < e; ++p) atomicSub(cnt + __ldg(ci + p), 1);
-        done = true;
       }
-      if (!done && wd_giveup(spins, st)) done = true;  // garbage result, DEADLOCK reported
+      push_rows<T, true>(ready, a, e, z, ci, val, bw, cnt, lane);
+      done = done || ready;
+      if (!done && wd_giveup(spins, st)) give = true;
+      if (__any_sync(0xffffffffu, give)) break;  // garbage result, DEADLOCK reported
     }
+    if (__any_sync(0xffffffffu, give)) break;
   }
 }
 
-// Transposed square: b'_c -= sum_r s'_rc z_r, one lane per stored row
+// Transposed square: b'_c -= sum_r s'_rc z_r, one lane per stored row (long
+// rows pushed by the whole warp)
 template <typename T, bool DCSR>
 __global__ void sq_push_T(int nzr, int r0, const int* __restrict__ rows, const int* __restrict__ rp,
                           const int* __restrict__ ci, const T* __restrict__ val, const T* __restrict__ xs,
                           T* __restrict__ bw) {
   const int t = blockIdx.x * blockDim.x + threadIdx.x;
-  if (t >= nzr) return;
-  const int r = DCSR ? __ldg(rows + t) : r0 + t;
-  const T z = xs[r];
-  const int a = __ldg(rp + t), e = __ldg(rp + t + 1);
-  for (int p = a; p < e; ++p) atomicAdd(bw + __ldg(ci + p), -ldg_nc(val + p) * z);
+  const int lane = threadIdx.x & 31;
+  if (t - lane >= nzr) return;  // whole warp out of range
+  const bool live = t < nzr;
+  int a = 0, e = 0;
+  T z = T(0);
+  if (live) {
+    const int r = DCSR ? __ldg(rows + t) : r0 + t;
+    z = xs[r];
+    a = __ldg(rp + t);
+    e = __ldg(rp + t + 1);
+  }
+  push_rows<T, false>(live && e > a, a, e, z, ci, val, bw, nullptr, lane);
 }
 
 }  // namespace k

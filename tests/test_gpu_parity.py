@@ -201,7 +201,7 @@ def test_transpose(gpu, name, uplo, nrhs):
     _check64(g.transpose(M), b, x)
 
 
-@pytest.mark.parametrize("name", ["C2", "C4"])
+@pytest.mark.parametrize("name", ["C2", "C3", "C4"])
 def test_full_size_transpose(gpu, name):
     """Full BASELINE sizes, default options: L^T x = b (the backward sweep of
     an IC(0) / supernodal preconditioner application)."""
@@ -421,6 +421,18 @@ def test_square_row_blocks(gpu, depth, dtype, reorder):
         _check64(M, b, x)
     else:
         assert on.rel_err(x, on.solve(M, b)) <= TOL32
+
+
+@pytest.mark.parametrize("transpose", [False, True])
+@pytest.mark.parametrize("n", [9000, 20000])
+def test_row_with_more_than_32_pieces(gpu, n, transpose):
+    """A row longer than 32 * kSfNB (8,192) entries is cut into > 32 pieces;
+    its last piece adds the partial sums 32 at a time (C3^T has rows of 258K
+    entries: the round-2 bug summed only the first 32 pieces)."""
+    M = g.shape_arrow(n)
+    b = g.gen_rhs(M.n, 1)
+    x, plan = _solve(M, b, depth=0, force_tri_impl="TRI_SYNCFREE", transpose=transpose)
+    _check64(g.transpose(M) if transpose else M, b, x)
 
 
 def test_full_size_c2_default_plan(gpu):
