@@ -33,6 +33,13 @@ def _stale(out: str, deps: list[str]) -> bool:
 
 def build(force: bool = False, verbose: bool = False) -> str:
     os.makedirs(BUILD, exist_ok=True)
+    # a change of the compile flags (SPTRSV_NVCC_FLAGS) rebuilds everything
+    stamp = os.path.join(BUILD, "flags.txt")
+    flags = " ".join(COMMON)
+    if not os.path.exists(stamp) or open(stamp).read() != flags:
+        force = True
+        with open(stamp, "w") as f:
+            f.write(flags)
     hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [os.path.join(INCLUDE, "sptrsv.h")]
     objs = []
     for src in SOURCES:

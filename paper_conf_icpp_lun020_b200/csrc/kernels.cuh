@@ -1523,6 +1523,20 @@ __global__ void __launch_bounds__(256, SPTRSV_SN_MINB) tri_supernode(int nitems,
 // In fp64 on B200 the DMMA tensor-core rate is not above the DFMA rate, so
 // the dense tiles run on the FMA pipes (f-3).
 constexpr int kSnmCols = 64;
+constexpr int kSnmXld = kSnmCols + 4;
+#ifndef SPTRSV_SNM_DMMA
+#define SPTRSV_SNM_DMMA 1
+#endif
+
+// fp64 tensor-core MMA (DMMA, mma.sync m8n8k4 .f64 -- tcgen05 has no f64
+// kind, so this is sm_100a's f64 tensor-core path): D = A(8x4, row) x
+// B(4x8, col) + C.  Fragments (g = lane >> 2, q = lane & 3): a = A[g][q],
+// b = B[q][g], c/d = {C[g][2q], C[g][2q+1]}.
+__device__ __forceinline__ void dmma_8x8x4(double& d0, double& d1, double a, double b) {
+  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
+               : "+d"(d0), "+d"(d1)
+               : "d"(a), "d"(b));
+}
 template <typename T>
 __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const SnDesc* __restrict__ desc,
                                                            const int* __restrict__ cols, const T* __restrict__ V,
@@ -1530,10 +1544,11 @@ __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const
                                                            T* __restrict__ xs, SolveState st, int slot, int nrhs,
                                                            int c_lo, int c_hi) {
   __shared__ __align__(16) T Vs[32][32];
-  __shared__ __align__(16) T Xs[32][kSnmCols];
+  __shared__ __align__(16) T Xs[32][kSnmXld];  // row pad: the DMMA B fragments read 4 rows x 8 columns
   __shared__ __align__(16) T Ys[32][kSnmCols + 1];
   __shared__ int Js[2][32];
   __shared__ int Jsh;
+  constexpr bool kSnmDmma = sizeof(T) == 8 && SPTRSV_SNM_DMMA;  // fp64 product on the tensor cores
   const int tid = threadIdx.x, lane = tid & 31, wi = tid >> 5;
   uint32_t* ticket = st.tickets + slot;
   const uint32_t epoch = solve_epoch(st);
@@ -1545,12 +1560,16 @@ __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const
     if (J >= npieces) break;
     const SnDesc d = desc[J];
     for (int c0 = c_lo; c0 < c_hi; c0 += kSnmCols) {
+      // fp64: warp wi owns the 8 x 8 DMMA tiles (row block wi & 3, column
+      // blocks 4 (wi >> 2) .. +3); acc[i][u] = C[t = 8 rb + g][c = 8 cb_i + 2 q + u].
+      // fp32: warp wi owns rows 4 wi .. 4 wi + 3, lane columns lane, lane + 32.
       T acc[4][2];
 #pragma unroll
       for (int i = 0; i < 4; ++i)
 #pragma unroll
         for (int u = 0; u < 2; ++u) {
-          const int t = wi * 4 + i, c = c0 + lane + 32 * u;
+          const int t = kSnmDmma ? 8 * (wi & 3) + (lane >> 2) : wi * 4 + i;
+          const int c = c0 + (kSnmDmma ? 8 * (4 * (wi >> 2) + i) + 2 * (lane & 3) + u : lane + 32 * u);
           acc[i][u] = (t < d.w && c < nrhs) ? bw[(int64_t)(d.s + t) * nrhs + c] : T(0);
         }
       // round prologue for external columns [q0, q0+32): one thread per
@@ -1603,23 +1622,41 @@ __global__ void __launch_bounds__(256, 4) tri_supernode_multi(int npieces, const
           Xs[idx / kSnmCols][idx % kSnmCols] = xr[k];
         }
         __syncthreads();
-        for (int q = 0; q < nq; ++q) {
-          const T x0 = Xs[q][lane], x1 = Xs[q][lane + 32];
+        if constexpr (kSnmDmma) {
+          // C -= V_J^T[rows, q0..q0+32) X[q0..q0+32, cols] on the fp64 tensor
+          // cores: 8 k-steps of 4 external columns (rounds are zero-padded)
+          const int g = lane >> 2, qq = lane & 3, rb = wi & 3, cb = 4 * (wi >> 2);
 #pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const T v = Vs[q][wi * 4 + i];
-            acc[i][0] -= v * x0;
-            acc[i][1] -= v * x1;
+          for (int k0 = 0; k0 < 32; k0 += 4) {
+            if (k0 < nq) {  // CTA-uniform
+              const double a = -Vs[k0 + qq][8 * rb + g];
+#pragma unroll
+              for (int i = 0; i < 4; ++i) dmma_8x8x4(acc[i][0], acc[i][1], a, Xs[k0 + qq][8 * (cb + i) + g]);
+            }
+          }
+        } else {
+          for (int q = 0; q < nq; ++q) {
+            const T x0 = Xs[q][lane], x1 = Xs[q][lane + 32];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+              const T v = Vs[q][wi * 4 + i];
+              acc[i][0] -= v * x0;
+              acc[i][1] -= v * x1;
+            }
           }
         }
         if (q0 + 32 < d.ne) prep(q0 + 32, buf ^ 1);
         __syncthreads();  // Vs / Xs are restaged next round, Js[buf ^ 1] is ready
       }
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        Ys[wi * 4 + i][lane] = acc[i][0];
-        Ys[wi * 4 + i][lane + 32] = acc[i][1];
-      }
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+          if constexpr (kSnmDmma)
+            Ys[8 * (wi & 3) + (lane >> 2)][8 * (4 * (wi >> 2) + i) + 2 * (lane & 3) + u] = acc[i][u];
+          else
+            Ys[wi * 4 + i][lane + 32 * u] = acc[i][u];
+        }
       // T_J column-major in shared memory (aliasing Xs, free after the
       // product): column c holds rows c+1 .. w-1 (packed as in tri_supernode)
       T(*Ts)[32] = reinterpret_cast<T(*)[32]>(&Xs[0][0]);
