@@ -103,7 +103,8 @@ typedef struct {
                                min_block_rows 0, a root whose levels are all <= 2048 rows with
                                1..8 dependencies per row stays one triangle (R30);
                                >= 0 forces a uniform depth                                     */
-  int64_t min_block_rows;   /* depth-rule threshold; 0 = 20 * SMs * 128 (378,880 on 148 SMs)   */
+  int64_t min_block_rows;   /* depth-rule threshold; 0 = 20 * SMs * 128 (378,880 on 148 SMs),
+                               and 4x that under selector B200 with depth = -1 (DESIGN R33)   */
   int32_t reorder;          /* 0 = level-set reordering of every triangle (L231), 1 = none,
                                2 = auto (default): none when the input is supernodal (mean width of
                                its fundamental supernodes >= 8, R29), else level        */
@@ -241,7 +242,8 @@ typedef struct {
   double analyse_ms;          /* host wall time of sptrsv_analyse, upload included          */
   int64_t device_bytes;       /* device memory owned by the plan (arena, excl. workspace)  */
   int32_t depth_rule;         /* 0 = the paper's rule (L299), 1 = B200 retune (a root with
-                                 only narrow levels stays whole: DESIGN.md R30), 2 = caller's */
+                                 only narrow levels stays whole: DESIGN.md R30), 2 = caller's,
+                                 3 = the B200 threshold (R33) gave a shallower tree          */
   int32_t analysis;           /* where the analysis ran: 0 host, 1 device (f-2), 2 device levels /
                                  reorder / P L P^T + host-built kernel formats                */
 } sptrsv_plan_info_t;

@@ -185,6 +185,20 @@ void to_lower_transposed(LowerCSR& L, int32_t n, const int32_t* rp, const int32_
 }
 
 // Reading R2: largest d with d == 0 or floor(n / 2^d) >= T.
+// The depth-rule threshold T of L299 ("20 x CUDA cores"; reading R2).
+// Under the B200 selector with neither depth nor min_block_rows given, T is
+// 4x the paper's (reading R33): re-derived on B200 by the depth sweep of
+// DESIGN.md 5.8 (C3 depth 3 -> 1: -2.5%; C5 2 -> 0: -11% at 512 RHS, -13%
+// at one RHS; C1 / C2 / C4 unchanged), the L299 experiment redone on this
+// GPU with its kernels.  SPTRSV_NO_DEPTH_RETUNE keeps the paper's T.
+int64_t min_block_rows_rule(const Plan& p) {
+  if (p.opts.min_block_rows > 0) return p.opts.min_block_rows;
+  const int64_t T = (int64_t)20 * p.sm_count * 128;
+  if (p.opts.selector == SPTRSV_SELECT_B200 && p.opts.depth < 0 && std::getenv("SPTRSV_NO_DEPTH_RETUNE") == nullptr)
+    return 4 * T;
+  return T;
+}
+
 int32_t depth_rule(int64_t n, int64_t T) {
   int32_t d = 0;
   while ((n >> (d + 1)) >= T) ++d;
@@ -384,11 +398,16 @@ Error analyse_host(Plan& p, int32_t n, int64_t nnz, const int32_t* row_ptr, cons
   p.nnz = nnz;
 
   // ---- depth (L299) ----
-  p.min_block_rows = p.opts.min_block_rows > 0 ? p.opts.min_block_rows : (int64_t)20 * p.sm_count * 128;
+  p.min_block_rows = min_block_rows_rule(p);
   if (p.opts.depth >= 0)
     p.depth = clamp_depth(n, p.opts.depth);
   else
     p.depth = n ? depth_rule(n, p.min_block_rows) : 0;
+  // reading R33: the B200 threshold is 4x the paper's; report when it chose
+  // a shallower tree than the paper's T would have
+  if (p.opts.depth < 0 && n && p.min_block_rows != (int64_t)20 * p.sm_count * 128 && p.opts.min_block_rows == 0 &&
+      p.depth < depth_rule(n, (int64_t)20 * p.sm_count * 128))
+    p.depth_retuned = 3;
 
   // ---- recursive reordering: every node, root and leaves (reading R3) ----
   // Siblings are independent once their parent is reordered (each only reads
@@ -804,5 +823,7 @@ void choose_impls(Plan& p) {
     }
   }
 }
+
+int64_t default_min_block_rows(const Plan& p) { return min_block_rows_rule(p); }
 
 }  // namespace sptrsv

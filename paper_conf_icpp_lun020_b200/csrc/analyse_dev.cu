@@ -39,6 +39,7 @@ Error upload(Plan& p, void* stream);
 int count_launches_public(const Plan& p);
 void build_sq_items(Segment& S);
 SpmmCfg spmm_cfg_public();
+int64_t default_min_block_rows(const Plan& p);
 void build_sf_items(Segment& S, int32_t& part_base, int selector);
 void fuse_square_items(Segment& T, Segment& Q);
 bool watchdog_word_acquire(int32_t** h, int32_t** d);
@@ -563,7 +564,7 @@ Error analyse_device_t(Plan& p, int32_t n, int64_t nnz, const int32_t* d_rp, con
     Lval = lval;
   }
   // ---- depth (L299) ----
-  p.min_block_rows = p.opts.min_block_rows > 0 ? p.opts.min_block_rows : (int64_t)20 * p.sm_count * 128;
+  p.min_block_rows = default_min_block_rows(p);
   auto depth_rule = [](int64_t nn2, int64_t T2) {
     int32_t d = 0;
     while ((nn2 >> (d + 1)) >= T2) ++d;
@@ -576,6 +577,9 @@ Error analyse_device_t(Plan& p, int32_t n, int64_t nnz, const int32_t* d_rp, con
     return std::min(d, lg);
   };
   p.depth = p.opts.depth >= 0 ? clamp_depth(n, p.opts.depth) : (n ? depth_rule(n, p.min_block_rows) : 0);
+  if (p.opts.depth < 0 && n && p.min_block_rows != (int64_t)20 * p.sm_count * 128 && p.opts.min_block_rows == 0 &&
+      p.depth < depth_rule(n, (int64_t)20 * p.sm_count * 128))
+    p.depth_retuned = 3;  // reading R33, as the host does
   int* d_a = S.take<int>(nn + 1);
   int* d_l = S.take<int>(nn + 1);
   // ---- reorder AUTO (R29): mean fundamental-supernode width of the input ----

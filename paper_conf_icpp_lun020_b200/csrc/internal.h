@@ -284,6 +284,7 @@ std::vector<SegGeo> segment_geometry(int32_t n, int32_t depth, int32_t variant,
 Error build_segments_host(Plan& p, const std::vector<std::pair<int32_t, int32_t>>& leaves,
                           const std::vector<int32_t>& leaf_nl, int threads);
 int32_t select_tri(int32_t nlevels, int32_t npr);
+int64_t default_min_block_rows(const Plan& p);  // reading R2 / R33
 int32_t select_sq(int32_t npr, int64_t empty, int64_t m);
 
 // device-resident analysis (analyse_dev.cu): CSR given as

@@ -141,24 +141,50 @@ def test_structure_parity_c2_full_size():
 
 def test_b200_depth_retune_keeps_narrow_root_whole():
     """Reading R30: with the library's defaults (selector B200, depth and
-    min_block_rows unset) C2's root -- every level <= 1,000 rows, <= 2
-    dependencies per row -- stays one triangle (the wavefront solves it
-    whole); the structure is then the oracle's at depth 0.  An explicit
-    min_block_rows (or depth) restores the paper's rule; so does PAPER."""
-    M, _ = g.gen_config("C2")
+    min_block_rows unset) a 2-D stencil IC(0) root -- every level <= 2,048
+    rows, <= 2 dependencies per row -- stays one triangle (the wavefront
+    solves it whole); the structure is then the oracle's at depth 0.  On a
+    4M-row grid the B200 threshold (R33) alone would still split once, so
+    R30 is what keeps it whole.  An explicit min_block_rows (or depth)
+    restores the paper's rule; so does PAPER."""
+    M = g.c2_laplacian_ic0(2000)  # n = 4M: R33's T (1.5M rows) gives depth 1
     plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, host_only=True)
     info = plan.info()
     assert info["depth"] == 0 and info["depth_rule"] == 1
     assert [s["impl"] for s in plan.segments()] == ["TRI_PIPE"]
+    paper = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, host_only=True, selector="PAPER")
+    assert paper.info()["depth"] == 3 and paper.info()["depth_rule"] == 0
+    M, _ = g.gen_config("C2")
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, host_only=True)
+    assert plan.info()["depth"] == 0 and plan.info()["depth_rule"] in (1, 3)
     _compare(M, plan, st.analyse(M, depth=0))
     paper = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, host_only=True, selector="PAPER")
     assert paper.info()["depth"] == 1 and paper.info()["depth_rule"] == 0
     forced = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, host_only=True, depth=1)
     assert forced.info()["depth_rule"] == 2
-    # a wide-level root keeps the paper's depth (C5 shape, 150K rows, T small)
+    # a wide-level root keeps the paper's depth (C5 shape, 150K rows: 0 either way)
     M5 = g.c5_random_multirhs(n=150_001)
     p5 = sp.sptrsv_analyse(M5.row_ptr, M5.col_idx, M5.val, host_only=True)
     assert p5.info()["depth_rule"] == 0
+
+
+def test_b200_depth_threshold_r33():
+    """Reading R33: under the B200 selector with depth / min_block_rows unset,
+    the L299 threshold is 4 x 20 x SMs x 128; a C5-shaped root of 800K rows
+    (paper: depth 1) stays whole, reported as depth_rule 3, and its structure
+    is the oracle's at that depth; the PAPER selector and an explicit
+    min_block_rows keep the paper's threshold."""
+    M = g.c5_random_multirhs(n=800_000)
+    plan = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, host_only=True)
+    info = plan.info()
+    T = 20 * info["sm_count"] * 128
+    assert info["min_block_rows"] == 4 * T
+    assert info["depth"] == st.depth_rule(M.n, 4 * T) == 0 and info["depth_rule"] == 3
+    _compare(M, plan, st.analyse(M, depth=0))
+    paper = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, host_only=True, selector="PAPER")
+    assert paper.info()["depth"] == st.depth_rule(M.n, T) == 1 and paper.info()["depth_rule"] == 0
+    explicit = sp.sptrsv_analyse(M.row_ptr, M.col_idx, M.val, host_only=True, min_block_rows=T)
+    assert explicit.info()["depth"] == 1 and explicit.info()["depth_rule"] == 0
 
 
 @pytest.mark.parametrize("shape", ["diag", "chain", "dense", "arrow", "fig1", "n1", "n2", "empty"])
