@@ -416,7 +416,10 @@ def main():
         dseg = segs[dom - 1]
         dbytes = seg_alg_bytes(dseg, nrhs, vb)
         dimpl = run_impl(dseg)
-        if dseg["kind"] == "TRI" and dseg["nlevels"] > 1:
+        # a dependency floor applies to a one-RHS triangle solved row by row
+        # (the supernodal kernels take one hop per piece of up to 32 rows, and
+        # many-RHS triangles are bound by their X-row gathers, DESIGN 5.7)
+        if dseg["kind"] == "TRI" and dseg["nlevels"] > 1 and nrhs == 1 and not dimpl.startswith("TRI_SUPERNODE"):
             ns_lvl = seg_mean[dom] * 1e6 / dseg["nlevels"]
             dep = {"nlevels": dseg["nlevels"], "ns_per_level": ns_lvl}
             tl = load_tlvl()
