@@ -46,18 +46,26 @@ def laplacian_csr(nx: int, ny: int, device) -> torch.Tensor:
 
 
 class IC0:
-    """M^-1 = L^-T L^-1 from two plans analysed once (forward and transposed)."""
+    """M^-1 = L^-T L^-1.  same_plan=False (default): two plans analysed once
+    (forward, and the analysed transpose, R31: the fast pull-form kernels for
+    both sweeps).  same_plan=True: ONE plan; the L^-T sweep is the same
+    plan's push-form transposed solve (R32: no second analysis or copy)."""
 
-    def __init__(self, L):
+    def __init__(self, L, same_plan: bool = False):
         self.fwd = sp.sptrsv_analyse(L.row_ptr, L.col_idx, L.val)
-        self.bwd = sp.sptrsv_analyse(L.row_ptr, L.col_idx, L.val, transpose=True)
+        self.same = same_plan
+        self.bwd = None if same_plan else sp.sptrsv_analyse(L.row_ptr, L.col_idx, L.val, transpose=True)
 
     def __call__(self, r: torch.Tensor) -> torch.Tensor:
-        return sp.sptrsv_solve(self.bwd, sp.sptrsv_solve(self.fwd, r))
+        y = sp.sptrsv_solve(self.fwd, r)
+        if self.same:
+            return sp.sptrsv_solve(self.fwd, y, transposed=True)
+        return sp.sptrsv_solve(self.bwd, y)
 
     def free(self):
         self.fwd.free()
-        self.bwd.free()
+        if self.bwd is not None:
+            self.bwd.free()
 
 
 def pcg(A: torch.Tensor, b: torch.Tensor, M=None, tol: float = 1e-8, maxiter: int = 10000):

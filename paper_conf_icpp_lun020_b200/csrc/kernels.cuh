@@ -1417,7 +1417,10 @@ struct SnDesc {
 // the elimination tree hold the longest lists (all their children's and
 // grandchildren's columns) and sit at the END of the dependency chain: split,
 // their products run on many warps at once instead of one warp's serial rounds.
-constexpr int kSnChunk = 256;
+#ifndef SPTRSV_SN_CHUNK
+#define SPTRSV_SN_CHUNK 256
+#endif
+constexpr int kSnChunk = SPTRSV_SN_CHUNK;
 struct SnItem {
   int J, q0, q1, kind;  // piece, external columns [q0, q1); kind 0 whole piece, 1 partial chunk, 2 last chunk
   int s0, s1, pad0, pad1;  // kind 1: slot s0; kind 2: slots [s0, s1)

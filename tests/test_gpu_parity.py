@@ -226,6 +226,10 @@ def test_ic0_pcg_driver(gpu):
     z = M(torch.from_numpy(r).cuda()).cpu().numpy()
     ref = on.solve(g.transpose(L), on.solve(L, r))
     assert on.rel_err(z[None], ref[None]) <= TOL64
+    Ms = ex.IC0(L, same_plan=True)  # the L^-T sweep from the forward plan (R32)
+    zs = Ms(torch.from_numpy(r).cuda()).cpu().numpy()
+    assert on.rel_err(zs[None], ref[None]) <= TOL64
+    Ms.free()
     A = ex.laplacian_csr(nx, nx, torch.device("cuda"))
     b = torch.from_numpy(g.gen_rhs(L.n, 1, seed=6)[0]).cuda()
     x0, it_cg, h0 = ex.pcg(A, b, None, 1e-10)
