@@ -2175,6 +2175,16 @@ Error prepare_T(Plan& p, cudaStream_t s) {
   if (!p.d_tcnt0 || !p.d_tcnt || !p.d_tticket) return {SPTRSV_ERROR_ALLOC, "transposed-solve workspace"};
   CUDA_TRY(cudaMemsetAsync(p.d_tcnt0, 0, (size_t)std::max(1, n) * 4, s));
   p.d_torder.assign(ns, nullptr);
+  p.d_tpos.assign(ns, nullptr);
+  p.d_tlvs.assign(ns, nullptr);
+  p.d_ttpos.assign(ns, nullptr);
+  auto upload_ints = [&](const std::vector<int32_t>& h, int32_t** d) -> Error {
+    *d = (int32_t*)dalloc(p, std::max<size_t>(1, h.size()) * 4, s);
+    if (!*d) return {SPTRSV_ERROR_ALLOC, "transposed-solve index arrays"};
+    CUDA_TRY(cudaMemcpyAsync(*d, h.data(), h.size() * 4, cudaMemcpyHostToDevice, s));
+    CUDA_TRY(cudaStreamSynchronize(s));  // h is a host temporary
+    return {SPTRSV_SUCCESS, ""};
+  };
   for (size_t i = 0; i < ns; ++i) {
     Segment& S = p.segs[i];
     if (S.info.kind != 0) continue;
@@ -2183,14 +2193,35 @@ Error prepare_T(Plan& p, cudaStream_t s) {
     if (ne > 0)
       k::count_cols<<<(unsigned)std::min<int64_t>(cdiv(ne, 256), (int64_t)p.sm_count * 16), 256, 0, s>>>(
           ne, S.d_ci, p.d_tcnt0);
-    if (S.wave_K > 0 && (int)S.wave_tau.size() == m) {  // device position q of plan row t: tau^-1
-      std::vector<int32_t> inv(m), ord(m);
+    const bool wave = S.wave_K > 0 && (int)S.wave_tau.size() == m;
+    if (wave) {  // device position q of plan row t: tau^-1
+      std::vector<int32_t> inv(m), ord(m), pos(m);
       for (int q = 0; q < m; ++q) inv[S.wave_tau[q]] = q;
       for (int i2 = 0; i2 < m; ++i2) ord[i2] = inv[m - 1 - i2];
-      p.d_torder[i] = (int32_t*)dalloc(p, (size_t)m * 4, s);
-      if (!p.d_torder[i]) return {SPTRSV_ERROR_ALLOC, "transposed-solve claim order"};
-      CUDA_TRY(cudaMemcpyAsync(p.d_torder[i], ord.data(), (size_t)m * 4, cudaMemcpyHostToDevice, s));
-      CUDA_TRY(cudaStreamSynchronize(s));  // ord is a host temporary
+      for (int q = 0; q < m; ++q) pos[q] = m - 1 - S.wave_tau[q];
+      Error e = upload_ints(ord, &p.d_torder[i]);
+      if (e.status) return e;
+      e = upload_ints(pos, &p.d_tpos[i]);
+      if (e.status) return e;
+    }
+    // narrow-level triangle (levels contiguous in plan order, every level <=
+    // kPcMaxW rows, enough levels to be latency-bound): one-CTA reverse chain
+    const int nl = S.info.nlevels;
+    if (p.reorder_eff == 0 && nl >= 32 && (int)S.level_ptr.size() == nl + 1 &&
+        std::getenv("SPTRSV_NO_PUSHCHAIN") == nullptr) {
+      int wmax = 0;
+      for (int l = 0; l < nl; ++l) wmax = std::max(wmax, S.level_ptr[l + 1] - S.level_ptr[l]);
+      if (wmax <= k::kPcMaxW) {
+        std::vector<int32_t> lvs(nl + 1);
+        for (int l = 0; l <= nl; ++l) lvs[l] = m - S.level_ptr[nl - l];
+        Error e = upload_ints(lvs, &p.d_tlvs[i]);
+        if (e.status) return e;
+        p.d_ttpos[i] = (int32_t*)dalloc(p, (size_t)std::max<int64_t>(1, ne) * 4, s);
+        if (!p.d_ttpos[i]) return {SPTRSV_ERROR_ALLOC, "transposed-solve target positions"};
+        if (ne > 0)
+          k::pc_tpos<<<(unsigned)std::min<int64_t>(cdiv(ne, 256), (int64_t)p.sm_count * 16), 256, 0, s>>>(
+              ne, S.info.row0, m, S.d_ci, p.d_tpos[i], p.d_ttpos[i]);
+      }
     }
   }
   CUDA_TRY(cudaGetLastError());
@@ -2223,7 +2254,14 @@ Error solve_T_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, sptrsv
       }
     } else {
       const int m = I.row1 - I.row0;
-      if (m > 0) {
+      if (m > 0 && p.d_tlvs[si]) {  // narrow levels: one-CTA reverse chain, shared-memory ring
+        constexpr int XW = 2 * k::kPcMaxW * 2;  // >= 2 levels of kPcMaxW rows, a power of two
+        const uint32_t smem = (uint32_t)(XW * sizeof(T));
+        auto kern = k::tri_pushchain_T<T>;
+        CUDA_TRY(ensure_smem_attr((const void*)kern, smem, false));
+        kern<<<1, k::kPcNT, smem, s>>>(I.row0, m, I.nlevels, p.d_tlvs[si], p.d_torder[si], p.d_ttpos[si], S.d_rp,
+                                       S.d_ci, val, bw, xs, XW);
+      } else if (m > 0) {
         const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>(cdiv(m, 256), (int64_t)p.sm_count * 2));
         k::tri_push_T<T><<<g, 256, 0, s>>>(I.row0, m, p.d_torder.empty() ? nullptr : p.d_torder[si], S.d_rp, S.d_ci,
                                            val, bw, xs, p.d_tcnt, p.d_tticket + si, st);
@@ -2279,6 +2317,12 @@ void release(Plan& p) {
   dfree(p, p.d_tcnt, nullptr);
   dfree(p, p.d_tticket, nullptr);
   for (auto* q : p.d_torder) dfree(p, q, nullptr);
+  for (auto* q : p.d_tpos) dfree(p, q, nullptr);
+  for (auto* q : p.d_tlvs) dfree(p, q, nullptr);
+  for (auto* q : p.d_ttpos) dfree(p, q, nullptr);
+  p.d_ttpos.clear();
+  p.d_tpos.clear();
+  p.d_tlvs.clear();
   p.d_tcnt0 = p.d_tcnt = nullptr;
   p.d_tticket = nullptr;
   p.d_torder.clear();

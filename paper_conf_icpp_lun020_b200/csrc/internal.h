@@ -261,6 +261,10 @@ struct Plan {
   int32_t* d_tcnt = nullptr;         // working counters, reset from d_tcnt0 by permute-in
   uint32_t* d_tticket = nullptr;     // per-segment claim tickets
   std::vector<int32_t*> d_torder;    // per segment: claim order (wave triangles), else nullptr
+  std::vector<int32_t*> d_tpos;      // per segment: device row -> claim position (wave triangles)
+  std::vector<int32_t*> d_ttpos;     // per segment: claim position of every CSR entry's target
+  std::vector<int32_t*> d_tlvs;      // per segment: claim-position level starts (narrow-level
+                                     // triangles solved by k::tri_pushchain_T), else nullptr
 
   // profiling
   bool profiling = false;

@@ -2973,6 +2973,117 @@ __global__ void __launch_bounds__(256) tri_push_T(int r0, int m, const int* __re
   }
 }
 
+// Transposed triangle with narrow levels (every level <= kPcMaxW rows, the
+// C2 stencil factor's anti-diagonals): ONE CTA walks the levels in reverse
+// with a __syncthreads per level (Alg 2's barrier, L96, on-chip), so the
+// push of Alg 3 needs no counters.  Positions p = 0 .. m-1 are the claim
+// order (reverse level order); a push into a target within XW positions of
+// the current level's start goes into a shared-memory ring slot (atomicAdd
+// on shared memory), a farther one into b' in global memory (then the
+// pushing thread fences before the level's barrier).  A row's value is its
+// global b' (initial b' plus far pushes, read a level ahead) plus its ring
+// slot.  The next level's rows, row bounds, first kPcE entries and global b'
+// are loaded during the current level, so the per-level chain is
+// barrier -> LDS ring -> FMA -> shared atomics -> barrier.
+constexpr int kPcMaxW = 2048, kPcNT = 1024, kPcR = kPcMaxW / kPcNT, kPcE = 2;
+template <typename T>
+struct PcRow {
+  int q, a, e;
+  T g;
+  int tp[kPcE];  // claim positions of the first kPcE push targets
+  T v[kPcE];
+};
+template <typename T>
+__device__ __forceinline__ void pc_load(PcRow<T>& R, int p, int m, const int* __restrict__ order,
+                                        const int* __restrict__ rp, const int* __restrict__ tpos,
+                                        const T* __restrict__ val, const T* __restrict__ bw, int r0) {
+  R.q = order ? __ldg(order + p) : m - 1 - p;
+  R.a = __ldg(rp + R.q);
+  R.e = __ldg(rp + R.q + 1);
+  R.g = ld_strong(bw + r0 + R.q);
+#pragma unroll
+  for (int u = 0; u < kPcE; ++u)
+    if (R.a + u < R.e) {
+      R.tp[u] = __ldg(tpos + R.a + u);
+      R.v[u] = ldg_nc(val + R.a + u);
+    }
+}
+
+// claim position of every entry's target (k::tri_pushchain_T reads it
+// instead of chaining ci -> pos loads): tpos[e] = pos[ci[e] - r0] or m-1-(ci[e]-r0)
+static __global__ void pc_tpos(int64_t ne, int r0, int m, const int* __restrict__ ci, const int* __restrict__ pos,
+                               int* __restrict__ tpos) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < ne; e += (int64_t)gridDim.x * blockDim.x) {
+    const int lj = ci[e] - r0;
+    tpos[e] = pos ? pos[lj] : m - 1 - lj;
+  }
+}
+
+template <typename T>
+__global__ void __launch_bounds__(kPcNT, 1)
+    tri_pushchain_T(int r0, int m, int nlev, const int* __restrict__ lvs, const int* __restrict__ order,
+                    const int* __restrict__ tpos, const int* __restrict__ rp, const int* __restrict__ ci,
+                    const T* __restrict__ val, T* __restrict__ bw, T* __restrict__ xs, int XW) {
+  extern __shared__ __align__(16) unsigned char pc_smem[];
+  T* ring = (T*)pc_smem;
+  const int tid = threadIdx.x;
+  for (int i = tid; i < XW; i += kPcNT) ring[i] = T(0);
+  PcRow<T> R[kPcR];
+  int s = __ldg(lvs), e = __ldg(lvs + 1);
+#pragma unroll
+  for (int k = 0; k < kPcR; ++k)
+    if (s + tid + k * kPcNT < e) pc_load(R[k], s + tid + k * kPcNT, m, order, rp, tpos, val, bw, r0);
+  __syncthreads();
+  const uint32_t xm = (uint32_t)XW - 1;  // XW is a power of two
+  for (int l = 0; l < nlev; ++l) {
+    const int en = l + 2 <= nlev ? __ldg(lvs + l + 2) : e;
+    // next level's rows, bounds, entries and global b', loaded while this
+    // level computes (far pushes into them came from levels <= l - 1, fenced
+    // before those levels' barriers: a level is <= XW / 2 rows)
+    PcRow<T> Rn[kPcR];
+#pragma unroll
+    for (int k = 0; k < kPcR; ++k)
+      if (e + tid + k * kPcNT < en) pc_load(Rn[k], e + tid + k * kPcNT, m, order, rp, tpos, val, bw, r0);
+    bool far = false;
+#pragma unroll
+    for (int k = 0; k < kPcR; ++k) {
+      const int p = s + tid + k * kPcNT;
+      if (p < e) {
+        const T z = R[k].g + ring[(uint32_t)p & xm];
+        ring[(uint32_t)p & xm] = T(0);
+        xs[r0 + R[k].q] = z;
+        for (int u = 0; u < R[k].e - R[k].a; ++u) {
+          int tp = 0;
+          T vv = T(0);
+          if (u < kPcE) {
+#pragma unroll
+            for (int w2 = 0; w2 < kPcE; ++w2)  // run-time index into registers
+              if (w2 == u) {
+                tp = R[k].tp[w2];
+                vv = R[k].v[w2];
+              }
+          } else {
+            tp = __ldg(tpos + R[k].a + u);
+            vv = ldg_nc(val + R[k].a + u);
+          }
+          if (tp < s + XW) {
+            atomicAdd(ring + ((uint32_t)tp & xm), -vv * z);
+          } else {
+            atomicAdd(bw + __ldg(ci + R[k].a + u), -vv * z);
+            far = true;
+          }
+        }
+      }
+    }
+    if (far) __threadfence();
+    __syncthreads();  // this level's pushes are in the ring (and far ones in L2)
+#pragma unroll
+    for (int k = 0; k < kPcR; ++k) R[k] = Rn[k];
+    s = e;
+    e = en;
+  }
+}
+
 // Transposed square: b'_c -= sum_r s'_rc z_r, one lane per stored row (long
 // rows pushed by the whole warp)
 template <typename T, bool DCSR>

@@ -114,3 +114,22 @@ def test_full_size_transposed_same_plan(gpu, name):
     x, _ = _solve_T(M, b[0])
     MT = g.transpose(M)
     assert on.rel_err(x[None], on.solve(MT, b)) <= TOL64
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C3"])
+@pytest.mark.parametrize("chain", [True, False])
+def test_transposed_narrow_level_chain(gpu, name, chain, monkeypatch):
+    """Narrow-level triangles (every level <= 2,048 rows, >= 32 levels) take
+    the one-CTA reverse chain with the shared-memory ring (k::tri_pushchain_T);
+    SPTRSV_NO_PUSHCHAIN forces the multi-CTA counter kernel.  Both against
+    the oracle, with the wavefront's strand-ordered device rows (C2) and a
+    deep bidiagonal chain whose every level is one row."""
+    if not chain:
+        monkeypatch.setenv("SPTRSV_NO_PUSHCHAIN", "1")
+    M, b = g.gen_config(name, small=True, nrhs=1)
+    x, _ = _solve_T(M, b[0], depth=1)
+    _check(M, b[0], x)
+    Mb = g.shape_bidiagonal(3000)
+    bb = g.gen_rhs(Mb.n, 1)
+    x, _ = _solve_T(Mb, bb[0])
+    _check(Mb, bb[0], x)
