@@ -56,8 +56,8 @@ cudaError_t ensure_smem_attr(const void* f, uint32_t smem, bool cluster) {
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
-  char key[64];
-  std::snprintf(key, sizeof(key), "%p/%d", f, dev);
+  char key[64];  // the non-portable cluster attribute is part of the key
+  std::snprintf(key, sizeof(key), "%p/%d/%d", f, dev, cluster ? 1 : 0);
   std::lock_guard<std::mutex> g(attr_mu);
   auto it = attr_set.find(key);
   if (it != attr_set.end() && it->second >= smem) return cudaSuccess;

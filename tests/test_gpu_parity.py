@@ -449,3 +449,19 @@ def test_full_size_c2_default_plan(gpu):
     assert info["depth"] == 0 and info["depth_rule"] in (1, 3)
     assert [s["impl"] for s in plan.segments()] == ["TRI_PIPE"]
     _check64(M, b, x)
+
+
+@pytest.mark.parametrize("cs", [4, 16])
+def test_cluster_level_set_experiment(gpu, cs, monkeypatch):
+    """DESIGN 5.5: the level-set on one thread-block cluster (k::tri_level_cluster,
+    SPTRSV_SF_CLUSTER, not selected by default: measured slower) stays correct,
+    including rows cut into pieces within a level."""
+    monkeypatch.setenv("SPTRSV_SF_CLUSTER", str(cs))
+    M, b = g.gen_config("C3", small=True, nrhs=1)
+    x, _ = _solve(M, b, depth=2)
+    _check64(M, b, x)
+    A = g.shape_arrow(12000)
+    bA = g.gen_rhs(A.n, 1)
+    x, _ = _solve(A, bA, depth=0, force_tri_impl="TRI_SYNCFREE")
+    _check64(A, bA, x)
+
