@@ -1121,7 +1121,7 @@ Error run_segments(Plan& p, T* bw, T* xs, int nrhs, cudaStream_t s, k::SolveStat
                 const Segment& Q = p.segs[S.fused_sq];
                 sq = k::SqDesc{Q.d_rows, Q.d_rp, Q.d_ci, Q.d_val, Q.info.row0, Q.dev_dcsr ? 1 : 0};
               }
-              k::tri_sf_mixed<T, 4><<<std::max(1u, ctas(256, m)), 256, 0, s>>>(
+              k::tri_sf_mixed<T, SPTRSV_SF_U><<<std::max(1u, ctas(256, m)), 256, 0, s>>>(
                   I.row0, nitem, (const k::SfItem*)S.d_sf_items, S.d_rp, S.d_ci, val, bw, xs, (T*)p.d_part, st,
                   S.ticket_slot, sq);
             }

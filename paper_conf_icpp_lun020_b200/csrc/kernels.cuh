@@ -865,9 +865,12 @@ __global__ void __launch_bounds__(256) tri_syncfree_warp(int r0, int m, const in
 #endif
 constexpr int kSfNB = SPTRSV_SF_NB;
 #ifndef SPTRSV_SF_LONG
-#define SPTRSV_SF_LONG 32
+#define SPTRSV_SF_LONG 64  // round-2 sweep on C3 (16 / 32 / 64 / 96 / 128): 3.48 / 3.10 / 2.95 / 2.95 / 2.97 ms
 #endif
 constexpr int kSfLong = SPTRSV_SF_LONG;  // tri_sf_mixed: rows with more entries get a warp
+#ifndef SPTRSV_SF_U
+#define SPTRSV_SF_U 4  // tri_sf_mixed: loads a lane of a row group issues per batch
+#endif
 #ifndef SPTRSV_SF_POLLS
 #define SPTRSV_SF_POLLS 1
 #endif
