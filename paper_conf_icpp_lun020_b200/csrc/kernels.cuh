@@ -129,7 +129,10 @@ __device__ __forceinline__ void watchdog_trip(const SolveState& st) {
 
 // One more unsuccessful poll: true = give up (this poll's watchdog tripped,
 // or another one already did -- checked every 1024 polls, so the chunk
-// launches after a trip do not each spin kWatchdogSpins again).
+// launches after a trip do not each spin kWatchdogSpins again).  The lanes'
+// counters can differ (per-lane loops), so a loop whose condition is a
+// full-warp vote takes the decision with __any_sync: a lane that left such a
+// loop alone would leave the others blocked in the next vote.
 __device__ __forceinline__ bool wd_giveup(uint32_t& spins, const SolveState& st) {
   if (++spins > st.wd_spins) {
     watchdog_trip(st);
@@ -1007,7 +1010,7 @@ __global__ void __launch_bounds__(256, SPTRSV_SF_MINB) tri_sf_items(int r0, int 
       if (__any_sync(0xffffffffu, prog)) {
         ns = 0;
       } else {
-        if (wd_giveup(spins, st)) break;
+        if (__any_sync(0xffffffffu, wd_giveup(spins, st))) break;
         ns = backoff(ns, st.backoff_ns);
       }
       __syncwarp();
@@ -1137,7 +1140,7 @@ __global__ void __launch_bounds__(256, SPTRSV_SFM_MINB) tri_sf_mixed(int r0, int
         // -- sets the level time)
         bool give = false;
         while (!__any_sync(0xffffffffu, !done && !is_sent(xb))) {
-          if (wd_giveup(spins, st)) {
+          if (__any_sync(0xffffffffu, wd_giveup(spins, st))) {
             give = true;
             break;
           }
@@ -1192,7 +1195,7 @@ __global__ void __launch_bounds__(256, SPTRSV_SFM_MINB) tri_sf_mixed(int r0, int
         }
       bool give = false;
       while (__any_sync(0xffffffffu, pend != 0)) {
-        if (wd_giveup(spins, st)) {
+        if (__any_sync(0xffffffffu, wd_giveup(spins, st))) {
           give = true;
           break;
         }
@@ -1256,7 +1259,7 @@ __global__ void __launch_bounds__(256, SPTRSV_SFM_MINB) tri_sf_mixed(int r0, int
       }
     bool give = false;
     while (__any_sync(0xffffffffu, pend != 0)) {
-      if (wd_giveup(spins, st)) {
+      if (__any_sync(0xffffffffu, wd_giveup(spins, st))) {
         give = true;
         break;
       }
@@ -1355,7 +1358,7 @@ __global__ void __launch_bounds__(256) tri_sf_wrow(int r0, int nitem, const SfIt
 #pragma unroll
       for (int u = 0; u < UW; ++u)
         if ((pend & (1u << u)) && !is_sent(x[u])) pend &= ~(1u << u);
-      if (wd_giveup(spins, st)) {
+      if (__any_sync(0xffffffffu, wd_giveup(spins, st))) {
         give = true;
         break;
       }
@@ -1462,7 +1465,7 @@ __global__ void __launch_bounds__(256, SPTRSV_SN_MINB) tri_supernode(int nitems,
       uint32_t spins = 0;
       unsigned ns = 0;
       while (__any_sync(0xffffffffu, inq && is_sent(xj))) {
-        if (wd_giveup(spins, st)) break;
+        if (__any_sync(0xffffffffu, wd_giveup(spins, st))) break;
         ns = backoff(ns, st.backoff_ns);
         if (inq && is_sent(xj)) xj = ld_strong(xs + j);
       }
@@ -1487,7 +1490,7 @@ __global__ void __launch_bounds__(256, SPTRSV_SN_MINB) tri_supernode(int nitems,
         T pv = act ? ld_strong(part + (size_t)q * 32 + lane) : T(0);
         uint32_t spins = 0;
         while (__any_sync(0xffffffffu, act && is_sent(pv))) {
-          if (wd_giveup(spins, st)) break;
+          if (__any_sync(0xffffffffu, wd_giveup(spins, st))) break;
           if (act && is_sent(pv)) pv = ld_strong(part + (size_t)q * 32 + lane);
         }
         ps += pv;
