@@ -104,6 +104,14 @@ class ClockSampler:
         self._t = threading.Thread(target=self._run, daemon=True)
         self._t.start()
 
+    def wait_first(self, timeout: float = 3.0):
+        """Block until the first sample landed: the first nvidia-smi call
+        (process start + driver queries) then falls before the timed steps,
+        where it made the first step of short runs an outlier."""
+        t0 = time.time()
+        while not self.rows and time.time() - t0 < timeout:
+            time.sleep(0.01)
+
     def stop(self):
         self._stop.set()
         if self._t:
@@ -322,6 +330,11 @@ def main():
     stream = torch.cuda.current_stream(dev)
 
     assert args.warmup >= 3, "W >= 3: the 2nd solve captures the CUDA graph, the timed ones replay it"
+    # clocks are sampled from before the warm-up to the end of the timed
+    # region (every 0.2 s); the first sample is taken before any solve
+    clocks = ClockSampler(local)
+    clocks.start()
+    clocks.wait_first()
     for _ in range(args.warmup):
         if not args.no_flush:
             flush.zero_()
@@ -330,8 +343,6 @@ def main():
 
     # ---------------- timed region: K solves (graph replays), CUDA events on
     # the solve stream, no host synchronisation between steps
-    clocks = ClockSampler(local)
-    clocks.start()
     if ws > 1:
         dist.barrier()
     torch.cuda.synchronize()
