@@ -2178,6 +2178,7 @@ Error prepare_T(Plan& p, cudaStream_t s) {
   p.d_tpos.assign(ns, nullptr);
   p.d_tlvs.assign(ns, nullptr);
   p.d_ttpos.assign(ns, nullptr);
+  p.d_tpc.assign(ns, PcSeg{});
   auto upload_ints = [&](const std::vector<int32_t>& h, int32_t** d) -> Error {
     *d = (int32_t*)dalloc(p, std::max<size_t>(1, h.size()) * 4, s);
     if (!*d) return {SPTRSV_ERROR_ALLOC, "transposed-solve index arrays"};
@@ -2194,8 +2195,10 @@ Error prepare_T(Plan& p, cudaStream_t s) {
       k::count_cols<<<(unsigned)std::min<int64_t>(cdiv(ne, 256), (int64_t)p.sm_count * 16), 256, 0, s>>>(
           ne, S.d_ci, p.d_tcnt0);
     const bool wave = S.wave_K > 0 && (int)S.wave_tau.size() == m;
+    std::vector<int32_t> ord;
     if (wave) {  // device position q of plan row t: tau^-1
-      std::vector<int32_t> inv(m), ord(m), pos(m);
+      std::vector<int32_t> inv(m), pos(m);
+      ord.resize(m);
       for (int q = 0; q < m; ++q) inv[S.wave_tau[q]] = q;
       for (int i2 = 0; i2 < m; ++i2) ord[i2] = inv[m - 1 - i2];
       for (int q = 0; q < m; ++q) pos[q] = m - 1 - S.wave_tau[q];
@@ -2221,6 +2224,24 @@ Error prepare_T(Plan& p, cudaStream_t s) {
         if (ne > 0)
           k::pc_tpos<<<(unsigned)std::min<int64_t>(cdiv(ne, 256), (int64_t)p.sm_count * 16), 256, 0, s>>>(
               ne, S.info.row0, m, S.d_ci, p.d_tpos[i], p.d_ttpos[i]);
+        // claim-position records: row, entry count, first kPcE (target, value) pairs; b' buffer
+        std::vector<int32_t> pq(m);
+        for (int q2 = 0; q2 < m; ++q2) pq[q2] = wave ? ord[q2] : m - 1 - q2;
+        PcSeg& C = p.d_tpc[i];
+        e = upload_ints(pq, &C.pq);
+        if (e.status) return e;
+        C.ecnt = (int32_t*)dalloc(p, (size_t)m * 4, s);
+        C.etp = (int32_t*)dalloc(p, (size_t)m * k::kPcE * 4, s);
+        C.ev = dalloc(p, (size_t)m * k::kPcE * p.vbytes, s);
+        C.gpos = dalloc(p, (size_t)m * p.vbytes, s);
+        if (!C.ecnt || !C.etp || !C.ev || !C.gpos) return {SPTRSV_ERROR_ALLOC, "transposed-solve chain records"};
+        if (p.vbytes == 8)
+          k::pc_build<double><<<cdiv(m, 256), 256, 0, s>>>(m, C.pq, S.d_rp, p.d_ttpos[i], (const double*)S.d_val,
+                                                           C.ecnt, C.etp, (double*)C.ev);
+        else
+          k::pc_build<float><<<cdiv(m, 256), 256, 0, s>>>(m, C.pq, S.d_rp, p.d_ttpos[i], (const float*)S.d_val,
+                                                          C.ecnt, C.etp, (float*)C.ev);
+        CUDA_TRY(cudaGetLastError());
       }
     }
   }
@@ -2259,8 +2280,10 @@ Error solve_T_device(Plan& p, const T* b, int64_t ldb, T* x, int64_t ldx, sptrsv
         const uint32_t smem = (uint32_t)(XW * sizeof(T));
         auto kern = k::tri_pushchain_T<T>;
         CUDA_TRY(ensure_smem_attr((const void*)kern, smem, false));
-        kern<<<1, k::kPcNT, smem, s>>>(I.row0, m, I.nlevels, p.d_tlvs[si], p.d_torder[si], p.d_ttpos[si], S.d_rp,
-                                       S.d_ci, val, bw, xs, XW);
+        const PcSeg& C = p.d_tpc[si];
+        k::pc_gather<T><<<cdiv(m, 256), 256, 0, s>>>(m, I.row0, C.pq, bw, (T*)C.gpos);
+        kern<<<1, k::kPcNT, smem, s>>>(I.row0, I.nlevels, p.d_tlvs[si], C.pq, C.ecnt, C.etp, (const T*)C.ev,
+                                       (T*)C.gpos, S.d_rp, p.d_ttpos[si], val, xs, XW);
       } else if (m > 0) {
         const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>(cdiv(m, 256), (int64_t)p.sm_count * 2));
         k::tri_push_T<T><<<g, 256, 0, s>>>(I.row0, m, p.d_torder.empty() ? nullptr : p.d_torder[si], S.d_rp, S.d_ci,
@@ -2320,6 +2343,14 @@ void release(Plan& p) {
   for (auto* q : p.d_tpos) dfree(p, q, nullptr);
   for (auto* q : p.d_tlvs) dfree(p, q, nullptr);
   for (auto* q : p.d_ttpos) dfree(p, q, nullptr);
+  for (auto& C : p.d_tpc) {
+    dfree(p, C.pq, nullptr);
+    dfree(p, C.ecnt, nullptr);
+    dfree(p, C.etp, nullptr);
+    dfree(p, C.ev, nullptr);
+    dfree(p, C.gpos, nullptr);
+  }
+  p.d_tpc.clear();
   p.d_ttpos.clear();
   p.d_tpos.clear();
   p.d_tlvs.clear();

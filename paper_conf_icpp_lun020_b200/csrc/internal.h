@@ -193,6 +193,16 @@ struct SpmmCfg {
                             // the matrix per tile measured 1.6-1.75x slower on C5; SPTRSV_SPMM_TILE)
 };
 
+// claim-position records of a narrow-level triangle's transposed chain
+// (k::pc_build / pc_gather / tri_pushchain_T)
+struct PcSeg {
+  int32_t* pq = nullptr;    // claim position -> local device row
+  int32_t* ecnt = nullptr;  // entries of that row
+  int32_t* etp = nullptr;   // first kPcE target positions
+  void* ev = nullptr;       // their values
+  void* gpos = nullptr;     // b' in claim-position order (per solve)
+};
+
 struct Plan {
   sptrsv_opts_t opts{};
   int32_t n = 0;
@@ -263,6 +273,7 @@ struct Plan {
   std::vector<int32_t*> d_torder;    // per segment: claim order (wave triangles), else nullptr
   std::vector<int32_t*> d_tpos;      // per segment: device row -> claim position (wave triangles)
   std::vector<int32_t*> d_ttpos;     // per segment: claim position of every CSR entry's target
+  std::vector<PcSeg> d_tpc;          // per segment: claim-position records (k::tri_pushchain_T)
   std::vector<int32_t*> d_tlvs;      // per segment: claim-position level starts (narrow-level
                                      // triangles solved by k::tri_pushchain_T), else nullptr
 

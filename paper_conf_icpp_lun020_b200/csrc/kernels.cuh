@@ -2994,29 +2994,30 @@ __global__ void __launch_bounds__(256) tri_push_T(int r0, int m, const int* __re
 constexpr int kPcMaxW = 2048, kPcNT = 1024, kPcR = kPcMaxW / kPcNT, kPcE = 2;
 template <typename T>
 struct PcRow {
-  int q, a, e;
-  T g;
+  int q, n;      // local device row, entry count
+  T g;           // b' of the row (global part)
   int tp[kPcE];  // claim positions of the first kPcE push targets
   T v[kPcE];
 };
+// Every load of a position's record is independent of the others (no
+// order -> row pointer -> entry chain): the record is laid out by claim
+// position at the first transposed solve (k::pc_build), and b' is gathered
+// into claim-position order before the kernel (k::pc_gather).
 template <typename T>
-__device__ __forceinline__ void pc_load(PcRow<T>& R, int p, int m, const int* __restrict__ order,
-                                        const int* __restrict__ rp, const int* __restrict__ tpos,
-                                        const T* __restrict__ val, const T* __restrict__ bw, int r0) {
-  R.q = order ? __ldg(order + p) : m - 1 - p;
-  R.a = __ldg(rp + R.q);
-  R.e = __ldg(rp + R.q + 1);
-  R.g = ld_strong(bw + r0 + R.q);
+__device__ __forceinline__ void pc_load(PcRow<T>& R, int p, const int* __restrict__ pq,
+                                        const int* __restrict__ ecnt, const int* __restrict__ etp,
+                                        const T* __restrict__ ev, const T* __restrict__ gpos) {
+  R.q = __ldg(pq + p);
+  R.n = __ldg(ecnt + p);
+  R.g = ld_strong(gpos + p);
 #pragma unroll
-  for (int u = 0; u < kPcE; ++u)
-    if (R.a + u < R.e) {
-      R.tp[u] = __ldg(tpos + R.a + u);
-      R.v[u] = ldg_nc(val + R.a + u);
-    }
+  for (int u = 0; u < kPcE; ++u) {
+    R.tp[u] = __ldg(etp + (size_t)p * kPcE + u);
+    R.v[u] = ldg_nc(ev + (size_t)p * kPcE + u);
+  }
 }
 
-// claim position of every entry's target (k::tri_pushchain_T reads it
-// instead of chaining ci -> pos loads): tpos[e] = pos[ci[e] - r0] or m-1-(ci[e]-r0)
+// claim position of every entry's target: tpos[e] = pos[ci[e] - r0] or m-1-(ci[e]-r0)
 static __global__ void pc_tpos(int64_t ne, int r0, int m, const int* __restrict__ ci, const int* __restrict__ pos,
                                int* __restrict__ tpos) {
   for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < ne; e += (int64_t)gridDim.x * blockDim.x) {
@@ -3025,11 +3026,34 @@ static __global__ void pc_tpos(int64_t ne, int r0, int m, const int* __restrict_
   }
 }
 
+// per claim position p: entry count and the first kPcE (target position, value) pairs
+template <typename T>
+__global__ void pc_build(int m, const int* __restrict__ pq, const int* __restrict__ rp, const int* __restrict__ tpos,
+                         const T* __restrict__ val, int* __restrict__ ecnt, int* __restrict__ etp, T* __restrict__ ev) {
+  const int p = blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= m) return;
+  const int q = pq[p], a = rp[q], e = rp[q + 1];
+  ecnt[p] = e - a;
+#pragma unroll
+  for (int u = 0; u < kPcE; ++u) {
+    etp[(size_t)p * kPcE + u] = a + u < e ? tpos[a + u] : p;
+    ev[(size_t)p * kPcE + u] = a + u < e ? val[a + u] : T(0);
+  }
+}
+
+// b' of the segment's rows in claim-position order
+template <typename T>
+__global__ void pc_gather(int m, int r0, const int* __restrict__ pq, const T* __restrict__ bw, T* __restrict__ gpos) {
+  const int p = blockIdx.x * blockDim.x + threadIdx.x;
+  if (p < m) gpos[p] = bw[r0 + pq[p]];
+}
+
 template <typename T>
 __global__ void __launch_bounds__(kPcNT, 1)
-    tri_pushchain_T(int r0, int m, int nlev, const int* __restrict__ lvs, const int* __restrict__ order,
-                    const int* __restrict__ tpos, const int* __restrict__ rp, const int* __restrict__ ci,
-                    const T* __restrict__ val, T* __restrict__ bw, T* __restrict__ xs, int XW) {
+    tri_pushchain_T(int r0, int nlev, const int* __restrict__ lvs, const int* __restrict__ pq,
+                    const int* __restrict__ ecnt, const int* __restrict__ etp, const T* __restrict__ ev,
+                    T* __restrict__ gpos, const int* __restrict__ rp, const int* __restrict__ tpos,
+                    const T* __restrict__ val, T* __restrict__ xs, int XW) {
   extern __shared__ __align__(16) unsigned char pc_smem[];
   T* ring = (T*)pc_smem;
   const int tid = threadIdx.x;
@@ -3038,18 +3062,18 @@ __global__ void __launch_bounds__(kPcNT, 1)
   int s = __ldg(lvs), e = __ldg(lvs + 1);
 #pragma unroll
   for (int k = 0; k < kPcR; ++k)
-    if (s + tid + k * kPcNT < e) pc_load(R[k], s + tid + k * kPcNT, m, order, rp, tpos, val, bw, r0);
+    if (s + tid + k * kPcNT < e) pc_load(R[k], s + tid + k * kPcNT, pq, ecnt, etp, ev, gpos);
   __syncthreads();
   const uint32_t xm = (uint32_t)XW - 1;  // XW is a power of two
   for (int l = 0; l < nlev; ++l) {
     const int en = l + 2 <= nlev ? __ldg(lvs + l + 2) : e;
-    // next level's rows, bounds, entries and global b', loaded while this
-    // level computes (far pushes into them came from levels <= l - 1, fenced
-    // before those levels' barriers: a level is <= XW / 2 rows)
+    // next level's records, loaded while this level computes (far pushes
+    // into them came from levels <= l - 1, fenced before those levels'
+    // barriers: a level is <= XW / 2 rows)
     PcRow<T> Rn[kPcR];
 #pragma unroll
     for (int k = 0; k < kPcR; ++k)
-      if (e + tid + k * kPcNT < en) pc_load(Rn[k], e + tid + k * kPcNT, m, order, rp, tpos, val, bw, r0);
+      if (e + tid + k * kPcNT < en) pc_load(Rn[k], e + tid + k * kPcNT, pq, ecnt, etp, ev, gpos);
     bool far = false;
 #pragma unroll
     for (int k = 0; k < kPcR; ++k) {
@@ -3058,7 +3082,8 @@ __global__ void __launch_bounds__(kPcNT, 1)
         const T z = R[k].g + ring[(uint32_t)p & xm];
         ring[(uint32_t)p & xm] = T(0);
         xs[r0 + R[k].q] = z;
-        for (int u = 0; u < R[k].e - R[k].a; ++u) {
+        const int a = R[k].n > kPcE ? __ldg(rp + R[k].q) : 0;  // long rows: the CSR for the rest
+        for (int u = 0; u < R[k].n; ++u) {
           int tp = 0;
           T vv = T(0);
           if (u < kPcE) {
@@ -3069,13 +3094,13 @@ __global__ void __launch_bounds__(kPcNT, 1)
                 vv = R[k].v[w2];
               }
           } else {
-            tp = __ldg(tpos + R[k].a + u);
-            vv = ldg_nc(val + R[k].a + u);
+            tp = __ldg(tpos + a + u);
+            vv = ldg_nc(val + a + u);
           }
           if (tp < s + XW) {
             atomicAdd(ring + ((uint32_t)tp & xm), -vv * z);
           } else {
-            atomicAdd(bw + __ldg(ci + R[k].a + u), -vv * z);
+            atomicAdd(gpos + tp, -vv * z);
             far = true;
           }
         }
